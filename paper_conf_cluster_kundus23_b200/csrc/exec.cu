@@ -1,0 +1,706 @@
+// exec.cu -- lowering of a schedule Q to per-GPU stage programs and
+// their replay as CUDA graphs.
+//
+//   * each logical GPU i executes Q_i stage by stage; the ops of one
+//     stage fork onto up to w streams and join before the next stage
+//   * every op output has a location on each logical GPU that consumes it;
+//     a producer writes straight into the channel slice of a consumer concat
+//     (zero-copy concat) -- on its own GPU or, for a cross-GPU edge, in the
+//     consumer GPU's memory over NVLink (fused into the epilogue for conv /
+//     pool / add, else a peer-store push kernel), then releases an epoch flag
+//   * a stage waits device-side (acquire spin on the flag) for its remote
+//     inputs: no host round trip between a transfer and the next kernel,
+//     which is what the paper's MPI engine lacked
+//   * stages of different GPUs are not synchronised otherwise
+#include <algorithm>
+#include <cstring>
+#include <numeric>
+#include <set>
+
+#include "exec.h"
+
+namespace hios {
+
+void ck(cudaError_t e, const char* what) {
+  if (e != cudaSuccess) fail(HIOS_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+static inline int rup(int x, int m) { return (x + m - 1) / m * m; }
+static inline int64_t rup64(int64_t x, int64_t m) { return (x + m - 1) / m * m; }
+
+Executor::Executor(Schedule& sch) : s(sch), g(*sch.g), M(sch.M) {
+  esz = g.dtype == HIOS_BF16 ? 2 : 4;
+  int ndev = 0;
+  ck(cudaGetDeviceCount(&ndev), "cudaGetDeviceCount");
+  if (ndev <= 0) fail(HIOS_E_CUDA, "no CUDA device");
+  lg.resize(M);
+  for (int i = 0; i < M; ++i) {
+    lg[i].dev = s.devices.empty() ? i % ndev : s.devices[i];
+    if (lg[i].dev < 0 || lg[i].dev >= ndev) fail(HIOS_E_INVALID, "device out of range");
+    lg[i].local = s.owner.empty() || s.owner[i] == s.rank;
+  }
+  n_streams = 1;
+  for (auto& q : s.Q)
+    for (auto& S : q) n_streams = std::max(n_streams, (int)S.size());
+}
+
+Executor::~Executor() {
+  for (int i = 0; i < M; ++i) {
+    LGpu& L = lg[i];
+    if (!L.local && !L.ipc_mapped) continue;
+    cudaSetDevice(L.dev);
+    if (L.ipc_mapped) {
+      if (L.arena) cudaIpcCloseMemHandle(L.arena);
+      if (L.sync) cudaIpcCloseMemHandle(L.sync);
+      continue;
+    }
+    if (L.gexec) cudaGraphExecDestroy(L.gexec);
+    if (L.gexec_timed) cudaGraphExecDestroy(L.gexec_timed);
+    for (auto st : L.streams) cudaStreamDestroy(st);
+    if (L.ev_fork) cudaEventDestroy(L.ev_fork);
+    for (auto e : L.ev_join) cudaEventDestroy(e);
+    if (L.ev_start) cudaEventDestroy(L.ev_start);
+    if (L.ev_done) cudaEventDestroy(L.ev_done);
+    if (L.arena) cudaFree(L.arena);
+    if (L.sync) cudaFree(L.sync);
+    for (void* p : L.allocs) cudaFree(p);
+  }
+  for (auto e : op_ev0) if (e) cudaEventDestroy(e);
+  for (auto e : op_ev1) if (e) cudaEventDestroy(e);
+  if (d_in_stage) cudaFree(d_in_stage);
+  if (d_out_stage) cudaFree(d_out_stage);
+}
+
+// ----------------------------------------------------------------- plan
+void Executor::plan() {
+  const int n = g.n;
+  std::vector<std::vector<char>> need(n, std::vector<char>(M, 0));
+  for (int u = 0; u < n; ++u) {
+    need[u][s.gpu_of[u]] = 1;
+    for (int e : g.ops[u].out_edges) need[u][s.gpu_of[g.edges[e].dst]] = 1;
+  }
+  loc.assign(n, std::vector<Loc>(M));
+  inplace.assign(g.edges.size(), 0);
+  std::vector<int64_t> cursor(M, 0);
+  auto alloc = [&](int l, int64_t bytes) {
+    int64_t off = cursor[l];
+    cursor[l] += rup64(std::max<int64_t>(bytes, 16), 256);
+    return off;
+  };
+  // reverse topological order: a concat consumer's buffer exists before its producers are placed
+  for (int k = n - 1; k >= 0; --k) {
+    const int u = g.topo[k];
+    const Op& o = g.ops[u];
+    for (int l = 0; l < M; ++l) {
+      if (!need[u][l]) continue;
+      bool placed = false;
+      for (int e : o.out_edges) {
+        const int v = g.edges[e].dst;
+        const Op& ov = g.ops[v];
+        if (ov.kind != HIOS_OP_CONCAT || s.gpu_of[v] != l || loc[v][l].off < 0) continue;
+        int c_off = 0;
+        for (int e2 : ov.in_edges) {
+          if (g.edges[e2].slot >= g.edges[e].slot) break;
+          c_off += g.ops[g.edges[e2].src].C;
+        }
+        if (c_off % 8 || loc[v][l].ldc % 8) continue;  // 16-byte aligned slices only
+        loc[u][l] = Loc{loc[v][l].off + (int64_t)c_off * esz, loc[v][l].ldc};
+        inplace[e] = 1;
+        placed = true;
+        break;
+      }
+      if (!placed) {
+        const int ldc = rup(o.C, 8);
+        loc[u][l] = Loc{alloc(l, (int64_t)o.H * o.W * ldc * esz), ldc};
+      }
+    }
+  }
+  ox.assign(n, OpExec());
+  for (int v = 0; v < n; ++v) {
+    const Op& o = g.ops[v];
+    const int l = s.gpu_of[v];
+    if (o.kind == HIOS_OP_SEPCONV) {
+      OpExec& x = ox[v];
+      x.dw_ldc = rup(std::max(o.in_c, o.out_c), 8);
+      x.dwbuf = alloc(l, (int64_t)o.H * o.W * x.dw_ldc * esz);
+      if (o.reps > 1) {
+        x.mid_ldc = rup(o.out_c, 8);
+        x.midbuf = alloc(l, (int64_t)o.H * o.W * x.mid_ldc * esz);
+      }
+    }
+  }
+  // remote deliveries and flags
+  flag_index.assign(n, std::vector<int>(M, -1));
+  std::vector<int> nflags(M, 0);
+  for (int u = 0; u < n; ++u) {
+    const int home = s.gpu_of[u];
+    const int kind = g.ops[u].kind;
+    const bool can_fuse = kind == HIOS_OP_CONV || kind == HIOS_OP_MAXPOOL || kind == HIOS_OP_AVGPOOL ||
+                          kind == HIOS_OP_ADD;
+    bool fused_used = false;
+    for (int l = 0; l < M; ++l) {
+      if (l == home || !need[u][l]) continue;
+      flag_index[u][l] = nflags[l]++;
+      const bool fuse = can_fuse && !fused_used;
+      fused_used = fused_used || fuse;
+      ox[u].remote.push_back({l, fuse});
+    }
+  }
+  for (int l = 0; l < M; ++l) {
+    lg[l].arena_bytes = (size_t)std::max<int64_t>(cursor[l], 256);
+    lg[l].sync_words = 1 + M + nflags[l];
+  }
+}
+
+// ------------------------------------------------------------- allocate
+template <typename T> static T to_dev_t(float x);
+template <> float to_dev_t<float>(float x) { return x; }
+template <> bf16 to_dev_t<bf16>(float x) { return __float2bfloat16(x); }
+
+template <typename T>
+static void* upload(LGpu& L, const std::vector<T>& h) {
+  void* d = nullptr;
+  ck(cudaMalloc(&d, std::max<size_t>(h.size() * sizeof(T), 16)), "cudaMalloc weights");
+  L.allocs.push_back(d);
+  if (!h.empty()) ck(cudaMemcpy(d, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice), "upload");
+  return d;
+}
+
+// conv weights W[k][c][r][s] -> tensor-core layout [k][r*S+s][Cp] (Cp = C rounded to 8, zero pad)
+//                             -> SIMT layout [k][r][s][c]
+template <typename T>
+static std::vector<T> conv_layout(const float* W, int K, int C, int R, int S, int Cp) {
+  std::vector<T> out((size_t)K * R * S * Cp, to_dev_t<T>(0.f));
+  for (int k = 0; k < K; ++k)
+    for (int c = 0; c < C; ++c)
+      for (int r = 0; r < R; ++r)
+        for (int s2 = 0; s2 < S; ++s2)
+          out[((size_t)k * R * S + r * S + s2) * Cp + c] = to_dev_t<T>(W[(((size_t)k * C + c) * R + r) * S + s2]);
+  return out;
+}
+
+template <typename T>
+static void upload_weights_T(Executor& ex, int v) {
+  const Op& o = ex.g.ops[v];
+  LGpu& L = ex.lg[ex.s.gpu_of[v]];
+  OpExec& x = ex.ox[v];
+  const bool tc = ex.g.dtype == HIOS_BF16;
+  switch (o.kind) {
+    case HIOS_OP_CONV: {
+      const int Cp = tc ? rup(o.in_c, 8) : o.in_c;
+      x.w = upload(L, conv_layout<T>(o.weight.data(), o.out_c, o.in_c, o.kh, o.kw, Cp));
+      x.scale.push_back((float*)upload(L, o.scale));
+      x.shift.push_back((float*)upload(L, o.shift));
+      break;
+    }
+    case HIOS_OP_SEPCONV: {
+      size_t off = 0;
+      for (int r = 0; r < o.reps; ++r) {
+        const int c = r == 0 ? o.in_c : o.out_c;
+        const int RS = o.kh * o.kw;
+        std::vector<float> dw((size_t)RS * c);
+        for (int ch = 0; ch < c; ++ch)
+          for (int rs = 0; rs < RS; ++rs) dw[(size_t)rs * c + ch] = o.weight[off + (size_t)ch * RS + rs];
+        off += (size_t)c * RS;
+        x.dw.push_back((float*)upload(L, dw));
+        const int Cp = tc ? rup(c, 8) : c;
+        x.pw.push_back(upload(L, conv_layout<T>(o.weight.data() + off, o.out_c, c, 1, 1, Cp)));
+        off += (size_t)o.out_c * c;
+        std::vector<float> sc(o.scale.begin() + (size_t)r * o.out_c, o.scale.begin() + (size_t)(r + 1) * o.out_c);
+        std::vector<float> sh(o.shift.begin() + (size_t)r * o.out_c, o.shift.begin() + (size_t)(r + 1) * o.out_c);
+        x.scale.push_back((float*)upload(L, sc));
+        x.shift.push_back((float*)upload(L, sh));
+      }
+      break;
+    }
+    case HIOS_OP_LINEAR: {
+      // weight columns follow the NCHW flatten order; the input is NHWC:
+      // only C x 1 x 1 inputs (flatten orders coincide) are supported
+      const int in_op = ex.g.edges[o.in_edges[0]].src;
+      const Op& xi = ex.g.ops[in_op];
+      if (xi.H * xi.W != 1) fail(HIOS_E_UNSUPPORTED, "linear on a spatial input (insert a GAP)");
+      x.ldw = rup(o.in_c, 8);
+      std::vector<T> w((size_t)o.out_c * x.ldw, to_dev_t<T>(0.f));
+      for (int k = 0; k < o.out_c; ++k)
+        for (int c = 0; c < o.in_c; ++c) w[(size_t)k * x.ldw + c] = to_dev_t<T>(o.weight[(size_t)k * o.in_c + c]);
+      x.w = upload(L, w);
+      x.bias = (float*)upload(L, o.shift);
+      break;
+    }
+    default:
+      break;
+  }
+}
+
+void Executor::allocate() {
+  // peer access between distinct local devices
+  std::set<int> devs;
+  for (auto& L : lg) if (L.local) devs.insert(L.dev);
+  for (int a : devs)
+    for (int b : devs) {
+      if (a == b) continue;
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, a, b);
+      if (can) {
+        cudaSetDevice(a);
+        cudaError_t e = cudaDeviceEnablePeerAccess(b, 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled)
+          ck(e, "cudaDeviceEnablePeerAccess");
+        cudaGetLastError();
+      }
+    }
+  for (int l = 0; l < M; ++l) {
+    LGpu& L = lg[l];
+    if (!L.local) continue;
+    ck(cudaSetDevice(L.dev), "cudaSetDevice");
+    ck(cudaMalloc(&L.arena, L.arena_bytes), "cudaMalloc arena");
+    ck(cudaMemset(L.arena, 0, L.arena_bytes), "memset arena");
+    ck(cudaMalloc(&L.sync, L.sync_words * sizeof(unsigned)), "cudaMalloc sync");
+    ck(cudaMemset(L.sync, 0, L.sync_words * sizeof(unsigned)), "memset sync");
+    L.streams.resize(n_streams);
+    for (auto& st : L.streams) ck(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking), "stream");
+    ck(cudaEventCreateWithFlags(&L.ev_fork, cudaEventDisableTiming), "event");
+    L.ev_join.resize(n_streams);
+    for (auto& e : L.ev_join) ck(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
+    ck(cudaEventCreate(&L.ev_start), "event");
+    ck(cudaEventCreate(&L.ev_done), "event");
+  }
+  for (int v = 0; v < g.n; ++v) {
+    const int l = s.gpu_of[v];
+    if (!lg[l].local) continue;
+    ck(cudaSetDevice(lg[l].dev), "cudaSetDevice");
+    if (g.dtype == HIOS_BF16) upload_weights_T<bf16>(*this, v);
+    else upload_weights_T<float>(*this, v);
+  }
+  lowered = true;
+}
+
+// --------------------------------------------------------------- closures
+struct ConvPlan {
+  int th, tw, tiles_q, tiles_m, n_tile, tiles_n, stages;
+  size_t smem;
+};
+
+static ConvPlan plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh, int sw) {
+  ConvPlan c{};
+  int64_t best = -1;
+  for (int tw : {128, 64, 32, 16, 8}) {
+    const int th = 128 / tw;
+    if (tw * sw > 256 || th * sh > 256) continue;
+    const int64_t cost = (int64_t)((P + th - 1) / th) * th * ((Q + tw - 1) / tw) * tw;
+    if (best < 0 || cost < best) { best = cost; c.th = th; c.tw = tw; }
+  }
+  if (best < 0) fail(HIOS_E_UNSUPPORTED, "conv stride too large for the TMA box");
+  c.tiles_q = (Q + c.tw - 1) / c.tw;
+  c.tiles_m = ((P + c.th - 1) / c.th) * c.tiles_q;
+  const int nb = (K + 255) / 256;
+  c.n_tile = rup((K + nb - 1) / nb, 16);
+  while ((int64_t)c.tiles_m * ((K + c.n_tile - 1) / c.n_tile) < 148 && c.n_tile > 32)
+    c.n_tile = rup(c.n_tile / 2, 16);
+  c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
+  const int KI = R * S * ((C + 63) / 64);
+  const size_t stage_bytes = 16384 + (size_t)c.n_tile * 128;
+  c.stages = (int)std::min<size_t>(8, (200 * 1024 - 2048) / stage_bytes);
+  c.stages = std::max(2, std::min(c.stages, std::max(KI, 2)));
+  c.smem = conv_tc_smem_bytes(c.n_tile, c.stages);
+  return c;
+}
+
+struct View {
+  char* p;
+  int ldc;
+};
+
+template <typename T>
+static std::function<void(cudaStream_t)> conv_closure(Executor& ex, const View& in, int H, int W, int C,
+                                                      const void* w, float* scale, float* shift, int K, int R,
+                                                      int S, int sh, int sw, int ph, int pw, int dh, int dw,
+                                                      int P, int Q, int relu, const View& out, const View* out2,
+                                                      int& nk);
+
+template <>
+std::function<void(cudaStream_t)> conv_closure<bf16>(Executor&, const View& in, int H, int W, int C, const void* w,
+                                                     float* scale, float* shift, int K, int R, int S, int sh, int sw,
+                                                     int ph, int pw, int dh, int dw, int P, int Q, int relu,
+                                                     const View& out, const View* out2, int& nk) {
+  ConvPlan cp = plan_conv_tc(P, Q, K, C, R, S, sh, sw);
+  CUtensorMap mx, mw;
+  if (!make_tmap_3d(&mx, in.p, C, W, H, (uint64_t)in.ldc * 2, (uint64_t)W * in.ldc * 2, 64, cp.tw * sw, cp.th * sh,
+                    sw, sh))
+    fail(HIOS_E_CUDA, "tensor map (activation)");
+  const int Cp = rup(C, 8);
+  if (!make_tmap_3d(&mw, w, Cp, R * S, K, (uint64_t)Cp * 2, (uint64_t)R * S * Cp * 2, 64, 1, cp.n_tile, 1, 1))
+    fail(HIOS_E_CUDA, "tensor map (weights)");
+  ConvTcArgs a{};
+  a.P = P; a.Q = Q; a.K = K; a.C = C; a.R = R; a.S = S; a.sh = sh; a.sw = sw; a.ph = ph; a.pw = pw;
+  a.dh = dh; a.dw = dw; a.th = cp.th; a.tw = cp.tw; a.tiles_q = cp.tiles_q; a.n_tile = cp.n_tile;
+  a.c_chunks = (C + 63) / 64; a.stages = cp.stages; a.relu = relu; a.scale = scale; a.shift = shift;
+  a.out = (bf16*)out.p; a.ldo = out.ldc;
+  a.out2 = out2 ? (bf16*)out2->p : nullptr; a.ldo2 = out2 ? out2->ldc : 0;
+  nk += 1;
+  return [mx, mw, a, cp](cudaStream_t st) { launch_conv_tc(mx, mw, a, cp.tiles_m, cp.tiles_n, cp.smem, st); };
+}
+
+template <>
+std::function<void(cudaStream_t)> conv_closure<float>(Executor&, const View& in, int H, int W, int C, const void* w,
+                                                      float* scale, float* shift, int K, int R, int S, int sh,
+                                                      int sw, int ph, int pw, int dh, int dw, int P, int Q, int relu,
+                                                      const View& out, const View* out2, int& nk) {
+  ConvSimtArgs a{};
+  a.x = (const float*)in.p; a.H = H; a.W = W; a.C = C; a.ldx = in.ldc;
+  a.w = (const float*)w; a.P = P; a.Q = Q; a.K = K; a.R = R; a.S = S; a.sh = sh; a.sw = sw; a.ph = ph;
+  a.pw = pw; a.dh = dh; a.dw = dw; a.relu = relu; a.scale = scale; a.shift = shift;
+  a.out = (float*)out.p; a.ldo = out.ldc;
+  a.out2 = out2 ? (float*)out2->p : nullptr; a.ldo2 = out2 ? out2->ldc : 0;
+  nk += 1;
+  return [a](cudaStream_t st) { launch_conv_simt(a, st); };
+}
+
+template <typename T>
+static void build_op(Executor& ex, int v) {
+  Graph& g = ex.g;
+  const Op& o = g.ops[v];
+  const int l = ex.s.gpu_of[v];
+  OpExec& x = ex.ox[v];
+  auto view_of = [&](int u, int on) { return View{ex.ptr(on, ex.loc[u][on].off), ex.loc[u][on].ldc}; };
+  auto in_op = [&](int k) { return g.edges[o.in_edges[k]].src; };
+  const View out = view_of(v, l);
+  // fused remote destination (first remote consumer GPU of a fusable op)
+  View out2v{nullptr, 0};
+  const View* out2 = nullptr;
+  for (auto& r : x.remote)
+    if (r.second) {
+      out2v = view_of(v, r.first);
+      out2 = &out2v;
+    }
+  std::vector<std::function<void(cudaStream_t)>> fns;
+  int nk = 0;
+  switch (o.kind) {
+    case HIOS_OP_INPUT:
+      break;  // staged before the graph (hios_run_device)
+    case HIOS_OP_CONV: {
+      const int u = in_op(0);
+      const Op& xi = g.ops[u];
+      fns.push_back(conv_closure<T>(ex, view_of(u, l), xi.H, xi.W, xi.C, x.w, x.scale[0], x.shift[0], o.out_c, o.kh,
+                                    o.kw, o.sh, o.sw, o.ph, o.pw, o.dh, o.dw, o.H, o.W, o.relu, out, out2, nk));
+      break;
+    }
+    case HIOS_OP_SEPCONV: {
+      const Op& x0 = g.ops[in_op(0)];
+      View dwv{ex.ptr(l, x.dwbuf), x.dw_ldc};
+      View midv{x.midbuf >= 0 ? ex.ptr(l, x.midbuf) : nullptr, x.mid_ldc};
+      for (int r = 0; r < o.reps; ++r) {
+        DwArgs<T> d{};
+        const int c = r == 0 ? o.in_c : o.out_c;
+        const int Hi = r == 0 ? x0.H : o.H, Wi = r == 0 ? x0.W : o.W;
+        if (r == 0) {
+          const int nin = (int)o.in_edges.size();
+          if (nin > HIOS_MAX_IN) fail(HIOS_E_UNSUPPORTED, "sepconv with more than 16 inputs");
+          for (int k = 0; k < nin; ++k) {
+            View iv = view_of(in_op(k), l);
+            d.x[k] = (const T*)iv.p;
+            d.ldx[k] = iv.ldc;
+            d.agg[k] = o.agg.empty() ? 1.f : o.agg[k];
+          }
+          d.n_in = nin;
+        } else {
+          d.x[0] = (const T*)midv.p; d.ldx[0] = midv.ldc; d.agg[0] = 1.f; d.n_in = 1;
+        }
+        d.H = Hi; d.W = Wi; d.C = c; d.P = o.H; d.Q = o.W; d.R = o.kh; d.S = o.kw;
+        d.sh = r == 0 ? o.sh : 1; d.sw = r == 0 ? o.sw : 1; d.ph = o.ph; d.pw = o.pw;
+        d.pre_relu = o.pre_relu; d.w = x.dw[r]; d.out = (T*)dwv.p; d.ldo = dwv.ldc;
+        fns.push_back([d](cudaStream_t st) { launch_dw<T>(d, st); });
+        ++nk;
+        const bool last = r == o.reps - 1;
+        fns.push_back(conv_closure<T>(ex, dwv, o.H, o.W, c, x.pw[r], x.scale[r], x.shift[r], o.out_c, 1, 1, 1, 1, 0,
+                                      0, 1, 1, o.H, o.W, last ? o.relu : 0, last ? out : midv,
+                                      last ? nullptr : nullptr, nk));
+      }
+      break;
+    }
+    case HIOS_OP_MAXPOOL:
+    case HIOS_OP_AVGPOOL: {
+      const int u = in_op(0);
+      const Op& xi = g.ops[u];
+      View iv = view_of(u, l);
+      PoolArgs<T> p{};
+      p.x = (const T*)iv.p; p.H = xi.H; p.W = xi.W; p.C = xi.C; p.ldx = iv.ldc;
+      p.P = o.H; p.Q = o.W; p.kh = o.kh; p.kw = o.kw; p.sh = o.sh; p.sw = o.sw; p.ph = o.ph; p.pw = o.pw;
+      p.is_max = o.kind == HIOS_OP_MAXPOOL; p.cip = o.cip;
+      p.out = (T*)out.p; p.ldo = out.ldc;
+      p.out2 = out2 ? (T*)out2->p : nullptr; p.ldo2 = out2 ? out2->ldc : 0;
+      fns.push_back([p](cudaStream_t st) { launch_pool<T>(p, st); });
+      ++nk;
+      break;
+    }
+    case HIOS_OP_GAP: {
+      const int u = in_op(0);
+      const Op& xi = g.ops[u];
+      View iv = view_of(u, l);
+      const T* xp = (const T*)iv.p;
+      const int HW = xi.H * xi.W, C = xi.C, ldx = iv.ldc;
+      T* op = (T*)out.p;
+      fns.push_back([=](cudaStream_t st) { launch_gap<T>(xp, HW, C, ldx, op, st); });
+      ++nk;
+      break;
+    }
+    case HIOS_OP_LINEAR: {
+      View iv = view_of(in_op(0), l);
+      const T* xp = (const T*)iv.p;
+      const T* w = (const T*)x.w;
+      const int Cin = o.in_c, K = o.out_c, ldw = x.ldw;
+      const float* b = x.bias;
+      T* op = (T*)out.p;
+      fns.push_back([=](cudaStream_t st) { launch_linear<T>(xp, Cin, w, ldw, b, K, op, st); });
+      ++nk;
+      break;
+    }
+    case HIOS_OP_CONCAT: {
+      int c_off = 0;
+      for (int e : o.in_edges) {
+        const int u = g.edges[e].src;
+        const Op& xu = g.ops[u];
+        if (!ex.inplace[e]) {
+          View iv = view_of(u, l);
+          CopyArgs<T> c{(const T*)iv.p, iv.ldc, o.H * o.W, xu.C, (T*)(out.p + (size_t)c_off * ex.esz), out.ldc};
+          fns.push_back([c](cudaStream_t st) { launch_copy<T>(c, st); });
+          ++nk;
+        }
+        c_off += xu.C;
+      }
+      break;
+    }
+    case HIOS_OP_ADD: {
+      const int nin = (int)o.in_edges.size();
+      if (nin > HIOS_MAX_IN) fail(HIOS_E_UNSUPPORTED, "add with more than 16 inputs");
+      AddArgs<T> a{};
+      for (int k = 0; k < nin; ++k) {
+        View iv = view_of(in_op(k), l);
+        a.x[k] = (const T*)iv.p; a.ldx[k] = iv.ldc; a.agg[k] = o.agg[k];
+      }
+      a.n_in = nin; a.HW = o.H * o.W; a.C = o.C; a.relu = o.relu;
+      a.out = (T*)out.p; a.ldo = out.ldc;
+      a.out2 = out2 ? (T*)out2->p : nullptr; a.ldo2 = out2 ? out2->ldc : 0;
+      fns.push_back([a](cudaStream_t st) { launch_add<T>(a, st); });
+      ++nk;
+      break;
+    }
+    case HIOS_OP_IDENTITY: {
+      View iv = view_of(in_op(0), l);
+      CopyArgs<T> c{(const T*)iv.p, iv.ldc, o.H * o.W, o.C, (T*)out.p, out.ldc};
+      fns.push_back([c](cudaStream_t st) { launch_copy<T>(c, st); });
+      ++nk;
+      break;
+    }
+  }
+  x.run = [fns](cudaStream_t st) {
+    for (auto& f : fns) f(st);
+  };
+  x.n_kernels = nk;
+}
+
+void Executor::build_closures() {
+  for (int v = 0; v < g.n; ++v) {
+    const int l = s.gpu_of[v];
+    if (!lg[l].local) continue;
+    ck(cudaSetDevice(lg[l].dev), "cudaSetDevice");
+    if (g.dtype == HIOS_BF16) build_op<bf16>(*this, v);
+    else build_op<float>(*this, v);
+  }
+}
+
+// deliveries of op u's output to other logical GPUs: push (unless fused) + flag release
+static int enqueue_deliver(Executor& ex, int u, cudaStream_t st) {
+  const int l = ex.s.gpu_of[u];
+  const Op& o = ex.g.ops[u];
+  int nk = 0;
+  for (auto& r : ex.ox[u].remote) {
+    const int d = r.first;
+    if (!r.second) {
+      const Loc& src = ex.loc[u][l];
+      const Loc& dst = ex.loc[u][d];
+      if (ex.g.dtype == HIOS_BF16) {
+        CopyArgs<bf16> c{(const bf16*)ex.ptr(l, src.off), src.ldc, o.H * o.W, o.C, (bf16*)ex.ptr(d, dst.off), dst.ldc};
+        launch_copy<bf16>(c, st);
+      } else {
+        CopyArgs<float> c{(const float*)ex.ptr(l, src.off), src.ldc, o.H * o.W, o.C, (float*)ex.ptr(d, dst.off),
+                          dst.ldc};
+        launch_copy<float>(c, st);
+      }
+      ++nk;
+    }
+    launch_signal(ex.lg[l].sync, ex.lg[d].sync + 1 + ex.M + ex.flag_index[u][d], st);
+    ++nk;
+  }
+  return nk;
+}
+
+void Executor::enqueue_stage_program(int l, bool timed) {
+  LGpu& L = lg[l];
+  cudaStream_t s0 = L.streams[0];
+  int64_t nk = 0;
+  launch_epoch(L.sync, s0);
+  ++nk;
+  // back-pressure: do not overwrite a consumer GPU's buffers before it finished the previous run
+  std::set<int> consumers, producers;
+  for (int v = 0; v < g.n; ++v) {
+    if (s.gpu_of[v] == l)
+      for (auto& r : ox[v].remote) consumers.insert(r.first);
+    else
+      for (int m = 0; m < M; ++m)
+        if (m == l && flag_index[v][l] >= 0) producers.insert(s.gpu_of[v]);
+  }
+  for (int c : consumers) {
+    launch_wait(L.sync, L.sync + 1 + c, 1, s0);
+    ++nk;
+  }
+  for (auto& S : s.Q[l]) {
+    std::set<int> waits;
+    for (int v : S)
+      for (int e : g.ops[v].in_edges) {
+        const int u = g.edges[e].src;
+        if (s.gpu_of[u] != l) waits.insert(u);
+      }
+    for (int u : waits) {
+      launch_wait(L.sync, L.sync + 1 + M + flag_index[u][l], 0, s0);
+      ++nk;
+    }
+    auto run_one = [&](int v, cudaStream_t st) {
+      if (timed) ck(cudaEventRecordWithFlags(op_ev0[v], st, cudaEventRecordExternal), "event record");
+      ox[v].run(st);
+      if (timed) ck(cudaEventRecordWithFlags(op_ev1[v], st, cudaEventRecordExternal), "event record");
+      nk += ox[v].n_kernels;
+      nk += enqueue_deliver(*this, v, st);
+    };
+    if (S.size() == 1) {
+      run_one(S[0], s0);
+    } else {
+      ck(cudaEventRecord(L.ev_fork, s0), "fork");
+      for (size_t k = 1; k < S.size(); ++k) ck(cudaStreamWaitEvent(L.streams[k], L.ev_fork, 0), "fork wait");
+      for (size_t k = 0; k < S.size(); ++k) run_one(S[k], L.streams[k]);
+      for (size_t k = 1; k < S.size(); ++k) {
+        ck(cudaEventRecord(L.ev_join[k], L.streams[k]), "join");
+        ck(cudaStreamWaitEvent(s0, L.ev_join[k], 0), "join wait");
+      }
+    }
+  }
+  for (int p : producers) {
+    launch_signal(L.sync, lg[p].sync + 1 + l, s0);
+    ++nk;
+  }
+  if (!timed) kernels_per_run += nk;
+}
+
+void Executor::capture() {
+  if (op_ev0.empty()) {
+    op_ev0.assign(g.n, nullptr);
+    op_ev1.assign(g.n, nullptr);
+  }
+  kernels_per_run = 0;
+  for (int l = 0; l < M; ++l) {
+    LGpu& L = lg[l];
+    if (!L.local) continue;
+    ck(cudaSetDevice(L.dev), "cudaSetDevice");
+    for (int v = 0; v < g.n; ++v)
+      if (s.gpu_of[v] == l && !op_ev0[v]) {
+        ck(cudaEventCreate(&op_ev0[v]), "event");
+        ck(cudaEventCreate(&op_ev1[v]), "event");
+      }
+    for (int timed = 0; timed < 2; ++timed) {
+      cudaGraph_t graph;
+      ck(cudaStreamBeginCapture(L.streams[0], cudaStreamCaptureModeRelaxed), "begin capture");
+      enqueue_stage_program(l, timed != 0);
+      ck(cudaStreamEndCapture(L.streams[0], &graph), "end capture");
+      cudaGraphExec_t ge;
+      ck(cudaGraphInstantiate(&ge, graph, 0), "graph instantiate");
+      cudaGraphDestroy(graph);
+      (timed ? L.gexec_timed : L.gexec) = ge;
+    }
+  }
+  captured = true;
+}
+
+void Executor::run_device(const void* d_in, void* d_out, cudaStream_t user, bool timed) {
+  if (!lowered) {
+    plan();
+    allocate();
+  }
+  if (!captured) {
+    build_closures();
+    capture();
+  }
+  int cur = 0;
+  ck(cudaGetDevice(&cur), "cudaGetDevice");
+  cudaEvent_t ev_user = nullptr;
+  if (user) {
+    ck(cudaEventCreateWithFlags(&ev_user, cudaEventDisableTiming), "event");
+    ck(cudaEventRecord(ev_user, user), "record user");
+  }
+  const int li = s.gpu_of[g.input_op], ls = s.gpu_of[g.sink_op];
+  for (int l = 0; l < M; ++l) {
+    LGpu& L = lg[l];
+    if (!L.local) continue;
+    ck(cudaSetDevice(L.dev), "cudaSetDevice");
+    if (ev_user) ck(cudaStreamWaitEvent(L.streams[0], ev_user, 0), "wait user");
+    ck(cudaEventRecord(L.ev_start, L.streams[0]), "record start");
+    if (l == li && d_in) {
+      const Loc& lc = loc[g.input_op][l];
+      if (g.dtype == HIOS_BF16)
+        launch_input<bf16>((const float*)d_in, g.in_c, g.in_h, g.in_w, (bf16*)ptr(l, lc.off), lc.ldc, L.streams[0]);
+      else
+        launch_input<float>((const float*)d_in, g.in_c, g.in_h, g.in_w, (float*)ptr(l, lc.off), lc.ldc,
+                            L.streams[0]);
+    }
+  }
+  for (int l = 0; l < M; ++l) {
+    LGpu& L = lg[l];
+    if (!L.local) continue;
+    ck(cudaSetDevice(L.dev), "cudaSetDevice");
+    ck(cudaGraphLaunch(timed ? L.gexec_timed : L.gexec, L.streams[0]), "graph launch");
+  }
+  for (int l = 0; l < M; ++l) {
+    LGpu& L = lg[l];
+    if (!L.local) continue;
+    ck(cudaSetDevice(L.dev), "cudaSetDevice");
+    if (l == ls && d_out) {
+      const Op& o = g.ops[g.sink_op];
+      const Loc& lc = loc[g.sink_op][l];
+      if (g.dtype == HIOS_BF16)
+        launch_output<bf16>((const bf16*)ptr(l, lc.off), o.C, o.H, o.W, lc.ldc, (float*)d_out, L.streams[0]);
+      else
+        launch_output<float>((const float*)ptr(l, lc.off), o.C, o.H, o.W, lc.ldc, (float*)d_out, L.streams[0]);
+    }
+    ck(cudaEventRecord(L.ev_done, L.streams[0]), "record done");
+  }
+  ck(cudaSetDevice(cur), "cudaSetDevice");
+  for (int l = 0; l < M; ++l) {
+    LGpu& L = lg[l];
+    if (!L.local) continue;
+    if (user) ck(cudaStreamWaitEvent(user, L.ev_done, 0), "user wait");
+    else ck(cudaEventSynchronize(L.ev_done), "synchronize");
+  }
+  if (ev_user) cudaEventDestroy(ev_user);
+  ck(cudaGetLastError(), "run");
+}
+
+void Executor::read_output(int op, float* host, int64_t n) {
+  const int l = s.gpu_of[op];
+  if (!lg[l].local) fail(HIOS_E_INVALID, "op not executed by this process");
+  const Op& o = g.ops[op];
+  if (n < (int64_t)o.C * o.H * o.W) fail(HIOS_E_INVALID, "output buffer too small");
+  ck(cudaSetDevice(lg[l].dev), "cudaSetDevice");
+  float* tmp = nullptr;
+  const size_t bytes = (size_t)o.C * o.H * o.W * sizeof(float);
+  ck(cudaMalloc(&tmp, bytes), "cudaMalloc");
+  const Loc& lc = loc[op][l];
+  cudaStream_t st = lg[l].streams[0];
+  if (g.dtype == HIOS_BF16)
+    launch_output<bf16>((const bf16*)ptr(l, lc.off), o.C, o.H, o.W, lc.ldc, tmp, st);
+  else
+    launch_output<float>((const float*)ptr(l, lc.off), o.C, o.H, o.W, lc.ldc, tmp, st);
+  ck(cudaStreamSynchronize(st), "sync");
+  ck(cudaMemcpy(host, tmp, bytes, cudaMemcpyDeviceToHost), "D2H");
+  cudaFree(tmp);
+}
+
+}  // namespace hios

@@ -1,0 +1,83 @@
+// exec.h -- per-GPU stage executor.
+#pragma once
+#include <functional>
+#include <vector>
+
+#include "internal.h"
+#include "kernels.cuh"
+
+namespace hios {
+
+struct Loc {
+  int64_t off = -1;  // byte offset in the owning logical GPU's arena
+  int ldc = 0;       // pixel stride in elements
+};
+
+struct OpExec {
+  // device weights (home logical GPU)
+  void* w = nullptr;       // conv / linear weights (T) or sepconv pw weights per rep
+  std::vector<void*> pw;   // sepconv: per-rep pointwise weights
+  std::vector<float*> dw;  // sepconv: per-rep depthwise weights [RS][C] fp32
+  std::vector<float*> scale, shift;
+  float* bias = nullptr;
+  int ldw = 0;
+  // sepconv scratch (arena offsets)
+  int64_t dwbuf = -1, midbuf = -1;
+  int dw_ldc = 0, mid_ldc = 0;
+  // remote deliveries of this op's output: (consumer lgpu, fused-into-epilogue?)
+  std::vector<std::pair<int, bool>> remote;
+  std::function<void(cudaStream_t)> run;  // enqueue the op's kernels (incl. fused out2)
+  int n_kernels = 0;
+};
+
+struct LGpu {
+  int dev = 0;
+  bool local = true;
+  std::vector<cudaStream_t> streams;
+  cudaEvent_t ev_fork = nullptr;
+  std::vector<cudaEvent_t> ev_join;
+  cudaEvent_t ev_start = nullptr, ev_done = nullptr;
+  cudaGraphExec_t gexec = nullptr, gexec_timed = nullptr;
+  char* arena = nullptr;       // local: owned; remote (rank mode): IPC-mapped
+  size_t arena_bytes = 0;
+  unsigned* sync = nullptr;    // [0] epoch, [1 .. 1+M) acks, then flags
+  size_t sync_words = 0;
+  std::vector<void*> allocs;   // weights etc. (owned)
+  bool ipc_mapped = false;
+};
+
+struct Executor {
+  Schedule& s;
+  Graph& g;
+  int M;
+  int esz;  // element size
+  std::vector<LGpu> lg;
+  std::vector<std::vector<Loc>> loc;   // loc[op][lgpu]
+  std::vector<char> inplace;           // per edge: producer writes into the concat slice
+  std::vector<OpExec> ox;
+  std::vector<std::vector<int>> flag_index;  // [op][lgpu] flag slot on that lgpu (-1 none)
+  int n_streams = 1;
+  bool lowered = false, captured = false;
+  int64_t kernels_per_run = 0;
+  // timed-graph events: per op (start, end) on its home lgpu
+  std::vector<cudaEvent_t> op_ev0, op_ev1;
+  // staging for hios_run (host pointers)
+  float* d_in_stage = nullptr;
+  float* d_out_stage = nullptr;
+
+  explicit Executor(Schedule& sch);
+  ~Executor();
+  void plan();             // locations, flags (host only)
+  void allocate();         // arenas, sync words, weights (local lgpus)
+  void build_closures();   // per-op kernel launchers
+  void capture();          // per-lgpu CUDA graphs
+  void run_device(const void* d_in, void* d_out, cudaStream_t user, bool timed);
+  char* ptr(int lgpu, int64_t off) const { return lg[lgpu].arena + off; }
+  bool is_local(int l) const { return lg[l].local; }
+  void read_output(int op, float* host, int64_t n);
+  void enqueue_stage_program(int l, bool timed);
+};
+
+void ck(cudaError_t e, const char* what);
+
+}  // namespace hios

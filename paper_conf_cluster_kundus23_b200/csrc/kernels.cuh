@@ -1,0 +1,100 @@
+// kernels.cuh -- device kernels of the HIOS executor (sm_100a) and their
+// host-side launch descriptors.  Activations are NHWC, batch 1, with a pixel
+// stride `ldc` (elements, multiple of 8) so producers can write straight into
+// a channel slice of a concat buffer (zero-copy concat) or of a peer GPU's
+// buffer (fused transfer).
+#pragma once
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <cstdint>
+
+namespace hios {
+
+typedef __nv_bfloat16 bf16;
+
+// ------------------------------------------------------------------ conv
+// Implicit-GEMM convolution on tcgen05 tensor cores (bf16 in, fp32 TMEM
+// accumulate, bf16 out).  GEMM view: M = output pixels (tile = th x tw = 128
+// pixels of one spatial block), N = out channels (BLOCK_N <= 256), K = R*S*C
+// walked as (r, s, 64-channel chunk).  Both operands arrive by TMA into
+// 128B-swizzled K-major smem tiles: A = a 3-D box of the NHWC input at the
+// (r, s)-shifted, stride-traversed window (OOB = zero padding), B = a box of
+// the [K][R*S][Cp] weights.
+struct ConvTcArgs {
+  int P, Q, K, C, R, S, sh, sw, ph, pw, dh, dw;
+  int th, tw, tiles_q, n_tile, c_chunks, stages, relu;
+  const float* scale;  // [K]
+  const float* shift;  // [K]
+  bf16* out;  int ldo; // primary output (channel offset applied)
+  bf16* out2; int ldo2;// optional second destination (peer replica), or null
+};
+
+// CUDA-core implicit GEMM (fp32) for the fp32 path (1e-4 parity).
+struct ConvSimtArgs {
+  const float* x; int H, W, C, ldx;
+  const float* w;      // [K][R][S][C]
+  int P, Q, K, R, S, sh, sw, ph, pw, dh, dw, relu;
+  const float* scale; const float* shift;
+  float* out; int ldo;
+  float* out2; int ldo2;
+};
+
+// Depthwise stage of a separable conv: a = sum_i agg_i x_i ; relu? ; depthwise.
+#define HIOS_MAX_IN 16
+template <typename T>
+struct DwArgs {
+  const T* x[HIOS_MAX_IN]; int ldx[HIOS_MAX_IN]; float agg[HIOS_MAX_IN]; int n_in;
+  int H, W, C, P, Q, R, S, sh, sw, ph, pw, pre_relu;
+  const float* w;  // [R*S][C]
+  T* out; int ldo;
+};
+
+template <typename T>
+struct PoolArgs {
+  const T* x; int H, W, C, ldx;
+  int P, Q, kh, kw, sh, sw, ph, pw, is_max, cip;
+  T* out; int ldo;
+  T* out2; int ldo2;
+};
+
+template <typename T>
+struct AddArgs {
+  const T* x[HIOS_MAX_IN]; int ldx[HIOS_MAX_IN]; float agg[HIOS_MAX_IN]; int n_in;
+  int HW, C, relu;
+  T* out; int ldo;
+  T* out2; int ldo2;
+};
+
+template <typename T>
+struct CopyArgs {
+  const T* x; int ldx; int HW, C; T* out; int ldo;
+};
+
+// launchers (stream-ordered, capture-safe)
+void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcArgs& a, int n_tiles_m,
+                    int n_tiles_n, size_t smem, cudaStream_t st);
+size_t conv_tc_smem_bytes(int n_tile, int stages);
+void launch_conv_simt(const ConvSimtArgs& a, cudaStream_t st);
+template <typename T> void launch_dw(const DwArgs<T>& a, cudaStream_t st);
+template <typename T> void launch_pool(const PoolArgs<T>& a, cudaStream_t st);
+template <typename T> void launch_add(const AddArgs<T>& a, cudaStream_t st);
+template <typename T> void launch_copy(const CopyArgs<T>& a, cudaStream_t st);
+template <typename T> void launch_gap(const T* x, int HW, int C, int ldx, T* out, cudaStream_t st);
+template <typename T> void launch_linear(const T* x, int Cin, const T* w, int ldw, const float* b, int K,
+                                         T* out, cudaStream_t st);
+template <typename T> void launch_input(const float* nchw, int C, int H, int W, T* out, int ldo,
+                                        cudaStream_t st);
+template <typename T> void launch_output(const T* x, int C, int H, int W, int ldx, float* nchw,
+                                         cudaStream_t st);
+void launch_epoch(unsigned* epoch, cudaStream_t st);
+void launch_signal(const unsigned* epoch, unsigned* flag, cudaStream_t st);
+void launch_wait(const unsigned* epoch, const unsigned* flag, unsigned lag, cudaStream_t st);
+void launch_fill(void* p, size_t bytes, cudaStream_t st);
+
+// tensor maps (driver entry point resolved at run time; no -lcuda)
+bool make_tmap_3d(CUtensorMap* m, const void* base, uint64_t d0, uint64_t d1, uint64_t d2,
+                  uint64_t stride1_bytes, uint64_t stride2_bytes, uint32_t b0, uint32_t b1, uint32_t b2,
+                  uint32_t e1, uint32_t e2);
+
+}  // namespace hios

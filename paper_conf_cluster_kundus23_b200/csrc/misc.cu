@@ -1,0 +1,347 @@
+// misc.cu -- HBM-bound operator kernels: pooling, depthwise
+// stage of separable convs, n-ary add, copy (concat fallback and peer pushes),
+// GAP, linear head, input/output layout conversion, and the epoch flags used
+// for cross-GPU edges (a10/a11).  NHWC with a pixel stride; each thread owns
+// one pixel x VEC channels (16-byte vectors: 8 bf16 or 4 fp32) so a warp reads
+// contiguous 512-byte runs.
+#include "kernels.cuh"
+
+namespace hios {
+
+template <typename T> struct Vec;
+template <> struct Vec<float> { static constexpr int N = 4; };
+template <> struct Vec<bf16> { static constexpr int N = 8; };
+
+__device__ __forceinline__ float to_f(float x) { return x; }
+__device__ __forceinline__ float to_f(bf16 x) { return __bfloat162float(x); }
+template <typename T> __device__ __forceinline__ T from_f(float x);
+template <> __device__ __forceinline__ float from_f<float>(float x) { return x; }
+template <> __device__ __forceinline__ bf16 from_f<bf16>(float x) { return __float2bfloat16_rn(x); }
+
+// load VEC channels starting at c (vector path when fully inside, else scalar)
+template <typename T>
+__device__ __forceinline__ void load_vec(const T* p, int c, int C, float* v) {
+  constexpr int N = Vec<T>::N;
+  if (c + N <= C) {
+    uint4 raw = *reinterpret_cast<const uint4*>(p);
+    const T* e = reinterpret_cast<const T*>(&raw);
+#pragma unroll
+    for (int j = 0; j < N; ++j) v[j] = to_f(e[j]);
+  } else {
+#pragma unroll
+    for (int j = 0; j < N; ++j) v[j] = (c + j < C) ? to_f(p[j]) : 0.f;
+  }
+}
+template <typename T>
+__device__ __forceinline__ void store_vec(T* p, int c, int C, const float* v) {
+  constexpr int N = Vec<T>::N;
+  if (c + N <= C) {
+    uint4 raw;
+    T* e = reinterpret_cast<T*>(&raw);
+#pragma unroll
+    for (int j = 0; j < N; ++j) e[j] = from_f<T>(v[j]);
+    *reinterpret_cast<uint4*>(p) = raw;
+  } else {
+    for (int j = 0; j < N && c + j < C; ++j) p[j] = from_f<T>(v[j]);
+  }
+}
+
+static inline unsigned grid_for(long long n, int block) {
+  long long g = (n + block - 1) / block;
+  return (unsigned)(g < 1 ? 1 : g);
+}
+
+// ---------------------------------------------------------------- pooling
+template <typename T>
+__global__ void pool_kernel(const PoolArgs<T> a) {
+  constexpr int N = Vec<T>::N;
+  const int CG = (a.C + N - 1) / N;
+  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= (long long)a.P * a.Q * CG) return;
+  const int cg = (int)(idx % CG);
+  const long long pix = idx / CG;
+  const int q = (int)(pix % a.Q), p = (int)(pix / a.Q);
+  const int c = cg * N;
+  const int h0 = p * a.sh - a.ph, w0 = q * a.sw - a.pw;
+  float acc[N], v[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) acc[j] = a.is_max ? -INFINITY : 0.f;
+  int cnt = 0;
+  for (int r = 0; r < a.kh; ++r) {
+    const int h = h0 + r;
+    if (h < 0 || h >= a.H) continue;
+    for (int s = 0; s < a.kw; ++s) {
+      const int w = w0 + s;
+      if (w < 0 || w >= a.W) continue;
+      load_vec(a.x + ((size_t)h * a.W + w) * a.ldx + c, c, a.C, v);
+      ++cnt;
+#pragma unroll
+      for (int j = 0; j < N; ++j) acc[j] = a.is_max ? fmaxf(acc[j], v[j]) : acc[j] + v[j];
+    }
+  }
+  if (!a.is_max) {
+    int div = cnt;
+    if (a.cip) div = (min(h0 + a.kh, a.H + a.ph) - h0) * (min(w0 + a.kw, a.W + a.pw) - w0);
+    const float inv = 1.f / (float)div;
+#pragma unroll
+    for (int j = 0; j < N; ++j) acc[j] *= inv;
+  }
+  store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
+  if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+}
+
+template <typename T>
+void launch_pool(const PoolArgs<T>& a, cudaStream_t st) {
+  constexpr int N = Vec<T>::N;
+  long long n = (long long)a.P * a.Q * ((a.C + N - 1) / N);
+  pool_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(a);
+}
+
+// ------------------------------------------- depthwise (+ aggregation, ReLU)
+template <typename T>
+__global__ void dw_kernel(const DwArgs<T> a) {
+  constexpr int N = Vec<T>::N;
+  const int CG = (a.C + N - 1) / N;
+  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= (long long)a.P * a.Q * CG) return;
+  const int cg = (int)(idx % CG);
+  const long long pix = idx / CG;
+  const int q = (int)(pix % a.Q), p = (int)(pix / a.Q);
+  const int c = cg * N;
+  float acc[N], v[N], u[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) acc[j] = 0.f;
+  for (int r = 0; r < a.R; ++r) {
+    const int h = p * a.sh - a.ph + r;
+    if (h < 0 || h >= a.H) continue;
+    for (int s = 0; s < a.S; ++s) {
+      const int w = q * a.sw - a.pw + s;
+      if (w < 0 || w >= a.W) continue;
+      const size_t off = (size_t)h * a.W + w;
+#pragma unroll
+      for (int j = 0; j < N; ++j) u[j] = 0.f;
+      for (int i = 0; i < a.n_in; ++i) {
+        load_vec(a.x[i] + off * a.ldx[i] + c, c, a.C, v);
+#pragma unroll
+        for (int j = 0; j < N; ++j) u[j] += a.agg[i] * v[j];
+      }
+      const float* wt = a.w + (size_t)(r * a.S + s) * a.C + c;
+#pragma unroll
+      for (int j = 0; j < N; ++j) {
+        float x = a.pre_relu ? fmaxf(u[j], 0.f) : u[j];
+        acc[j] += x * ((c + j < a.C) ? __ldg(wt + j) : 0.f);
+      }
+    }
+  }
+  store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
+}
+
+template <typename T>
+void launch_dw(const DwArgs<T>& a, cudaStream_t st) {
+  constexpr int N = Vec<T>::N;
+  long long n = (long long)a.P * a.Q * ((a.C + N - 1) / N);
+  dw_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(a);
+}
+
+// ------------------------------------------------------------------- add
+template <typename T>
+__global__ void add_kernel(const AddArgs<T> a) {
+  constexpr int N = Vec<T>::N;
+  const int CG = (a.C + N - 1) / N;
+  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= (long long)a.HW * CG) return;
+  const int c = (int)(idx % CG) * N;
+  const long long pix = idx / CG;
+  float acc[N], v[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) acc[j] = 0.f;
+  for (int i = 0; i < a.n_in; ++i) {
+    load_vec(a.x[i] + pix * a.ldx[i] + c, c, a.C, v);
+#pragma unroll
+    for (int j = 0; j < N; ++j) acc[j] += a.agg[i] * v[j];
+  }
+  if (a.relu) {
+#pragma unroll
+    for (int j = 0; j < N; ++j) acc[j] = fmaxf(acc[j], 0.f);
+  }
+  store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
+  if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+}
+
+template <typename T>
+void launch_add(const AddArgs<T>& a, cudaStream_t st) {
+  constexpr int N = Vec<T>::N;
+  long long n = (long long)a.HW * ((a.C + N - 1) / N);
+  add_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(a);
+}
+
+// ------------------------------------------------------------------ copy
+template <typename T>
+__global__ void copy_kernel(const CopyArgs<T> a) {
+  constexpr int N = Vec<T>::N;
+  const int CG = (a.C + N - 1) / N;
+  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= (long long)a.HW * CG) return;
+  const int c = (int)(idx % CG) * N;
+  const long long pix = idx / CG;
+  const T* src = a.x + pix * a.ldx + c;
+  T* dst = a.out + pix * a.ldo + c;
+  if (c + N <= a.C) {
+    *reinterpret_cast<uint4*>(dst) = *reinterpret_cast<const uint4*>(src);
+  } else {
+    for (int j = 0; c + j < a.C; ++j) dst[j] = src[j];
+  }
+}
+
+template <typename T>
+void launch_copy(const CopyArgs<T>& a, cudaStream_t st) {
+  constexpr int N = Vec<T>::N;
+  long long n = (long long)a.HW * ((a.C + N - 1) / N);
+  copy_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(a);
+}
+
+// ------------------------------------------------------------------- GAP
+// one block per 8/4-channel group; threads stride over pixels; smem reduce
+template <typename T>
+__global__ void gap_kernel(const T* x, int HW, int C, int ldx, T* out) {
+  constexpr int N = Vec<T>::N;
+  const int c = blockIdx.x * N;
+  float acc[N], v[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) acc[j] = 0.f;
+  for (int pix = threadIdx.x; pix < HW; pix += blockDim.x) {
+    load_vec(x + (size_t)pix * ldx + c, c, C, v);
+#pragma unroll
+    for (int j = 0; j < N; ++j) acc[j] += v[j];
+  }
+  __shared__ float red[N][32];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    float s = acc[j];
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) red[j][warp] = s;
+  }
+  __syncthreads();
+  if (warp == 0) {
+    const int nw = blockDim.x >> 5;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+      float s = lane < nw ? red[j][lane] : 0.f;
+      for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+      acc[j] = s / (float)HW;
+    }
+    if (lane == 0) store_vec(out + c, c, C, acc);
+  }
+}
+
+template <typename T>
+void launch_gap(const T* x, int HW, int C, int ldx, T* out, cudaStream_t st) {
+  constexpr int N = Vec<T>::N;
+  gap_kernel<T><<<(C + N - 1) / N, 512, 0, st>>>(x, HW, C, ldx, out);
+}
+
+// ---------------------------------------------------------------- linear
+// one warp per output: y[k] = sum_c W[k,c] x[c] + b[k]
+template <typename T>
+__global__ void linear_kernel(const T* x, int Cin, const T* w, int ldw, const float* b, int K, T* out) {
+  const int k = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (k >= K) return;
+  constexpr int N = Vec<T>::N;
+  float s = 0.f, xv[N], wv[N];
+  const T* wr = w + (size_t)k * ldw;
+  for (int c = lane * N; c < Cin; c += 32 * N) {
+    load_vec(x + c, c, Cin, xv);
+    load_vec(wr + c, c, Cin, wv);
+#pragma unroll
+    for (int j = 0; j < N; ++j) s += xv[j] * wv[j];
+  }
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if (lane == 0) out[k] = from_f<T>(s + b[k]);
+}
+
+template <typename T>
+void launch_linear(const T* x, int Cin, const T* w, int ldw, const float* b, int K, T* out, cudaStream_t st) {
+  linear_kernel<T><<<(K + 7) / 8, 256, 0, st>>>(x, Cin, w, ldw, b, K, out);
+}
+
+// ------------------------------------------------- layout conversion
+template <typename T>
+__global__ void input_kernel(const float* nchw, int C, int HW, T* out, int ldo) {
+  const long long pix = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (pix >= HW) return;
+  for (int c = 0; c < ldo; ++c)
+    out[pix * ldo + c] = from_f<T>(c < C ? nchw[(size_t)c * HW + pix] : 0.f);
+}
+template <typename T>
+void launch_input(const float* nchw, int C, int H, int W, T* out, int ldo, cudaStream_t st) {
+  input_kernel<T><<<grid_for((long long)H * W, 256), 256, 0, st>>>(nchw, C, H * W, out, ldo);
+}
+
+template <typename T>
+__global__ void output_kernel(const T* x, int C, int HW, int ldx, float* nchw) {
+  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= (long long)C * HW) return;
+  const int c = (int)(i / HW);
+  const long long pix = i % HW;
+  nchw[i] = to_f(x[pix * ldx + c]);
+}
+template <typename T>
+void launch_output(const T* x, int C, int H, int W, int ldx, float* nchw, cudaStream_t st) {
+  output_kernel<T><<<grid_for((long long)C * H * W, 256), 256, 0, st>>>(x, C, H * W, ldx, nchw);
+}
+
+// ----------------------------------------------- cross-GPU epoch flags
+// epoch: incremented by the first kernel of every per-GPU graph replay.
+// signal: after the producer's stores (kernel boundary + system fence), the
+// producer GPU writes its epoch into the consumer's flag with a release store.
+// wait: the consumer spins (acquire, system scope) until flag >= epoch - lag.
+__global__ void epoch_kernel(unsigned* epoch) { *epoch += 1u; }
+
+__global__ void signal_kernel(const unsigned* epoch, unsigned* flag) {
+  const unsigned e = *epoch;
+  __threadfence_system();
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(flag), "r"(e) : "memory");
+}
+
+__global__ void wait_kernel(const unsigned* epoch, const unsigned* flag, unsigned lag) {
+  const unsigned target = *epoch - lag;
+  unsigned v;
+  while (true) {
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
+    if ((int)(v - target) >= 0) break;
+    __nanosleep(64);
+  }
+}
+
+void launch_epoch(unsigned* epoch, cudaStream_t st) { epoch_kernel<<<1, 1, 0, st>>>(epoch); }
+void launch_signal(const unsigned* epoch, unsigned* flag, cudaStream_t st) {
+  signal_kernel<<<1, 1, 0, st>>>(epoch, flag);
+}
+void launch_wait(const unsigned* epoch, const unsigned* flag, unsigned lag, cudaStream_t st) {
+  wait_kernel<<<1, 1, 0, st>>>(epoch, flag, lag);
+}
+
+__global__ void fill_kernel(uint4* p, size_t n) {
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
+    p[i] = make_uint4(i, i ^ 0x9e3779b9u, 0, 1);
+}
+void launch_fill(void* p, size_t bytes, cudaStream_t st) {
+  fill_kernel<<<148 * 8, 512, 0, st>>>(reinterpret_cast<uint4*>(p), bytes / 16);
+}
+
+// explicit instantiations
+#define HIOS_INST(T)                                                                                   \
+  template void launch_pool<T>(const PoolArgs<T>&, cudaStream_t);                                      \
+  template void launch_dw<T>(const DwArgs<T>&, cudaStream_t);                                          \
+  template void launch_add<T>(const AddArgs<T>&, cudaStream_t);                                        \
+  template void launch_copy<T>(const CopyArgs<T>&, cudaStream_t);                                      \
+  template void launch_gap<T>(const T*, int, int, int, T*, cudaStream_t);                              \
+  template void launch_linear<T>(const T*, int, const T*, int, const float*, int, T*, cudaStream_t);        \
+  template void launch_input<T>(const float*, int, int, int, T*, int, cudaStream_t);                   \
+  template void launch_output<T>(const T*, int, int, int, int, float*, cudaStream_t);
+HIOS_INST(float)
+HIOS_INST(bf16)
+
+}  // namespace hios

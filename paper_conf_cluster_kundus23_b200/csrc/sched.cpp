@@ -1,0 +1,290 @@
+// sched.cpp -- host-side HIOS-LP scheduler (§IV).
+//
+//   priorities       p(v), §IV-A
+//   longest path     Alg. 1 line 5, readings C3/C4
+//   list schedule    Alg. 1 lines 10-13, readings C1/C5
+//   hios_lp          Alg. 1 lines 1-16
+//   parallelize      Alg. 2, readings C7-C11
+//   simulate         cost model of §III: stage start = max(prev
+//                    stage on the GPU, inputs' finish + t(u,v) across GPUs)
+//
+// Integer nanosecond costs; every tie rule is fixed so the
+// result is bit-identical to the step-by-step CPU oracle on the same costs.
+#include <algorithm>
+#include <limits>
+
+#include "internal.h"
+
+namespace hios {
+
+int64_t Graph::stage_cost(const std::vector<int>& S_in) {
+  if (S_in.size() == 1) return op_cost(S_in[0]);
+  std::vector<int> S = S_in;
+  std::sort(S.begin(), S.end());
+  auto it = group_cost.find(S);
+  if (it != group_cost.end()) return it->second;
+  if (prof) {
+    int64_t c = prof->measure_group(*this, S);
+    group_cost[S] = c;
+    return c;
+  }
+  if (gm_num > 0) {
+    int64_t mx = 0, sum = 0;
+    for (int v : S) { mx = std::max(mx, op_cost(v)); sum += op_cost(v); }
+    return std::max(mx, (sum * gm_num) / gm_den);
+  }
+  fail(HIOS_E_STATE, "t(S) unknown for a candidate group (profile, set_group_cost or set_group_model)");
+}
+
+std::vector<int64_t> priorities(const Graph& g) {
+  std::vector<int64_t> p(g.n, 0);
+  for (int k = g.n - 1; k >= 0; --k) {
+    int v = g.topo[k];
+    int64_t best = 0;
+    for (int e : g.ops[v].out_edges) best = std::max(best, g.edge_cost(e) + p[g.edges[e].dst]);
+    p[v] = g.op_cost(v) + best;
+  }
+  return p;
+}
+
+std::vector<int> priority_order(const Graph& g) {
+  auto p = priorities(g);
+  std::vector<int> order(g.n);
+  for (int i = 0; i < g.n; ++i) order[i] = i;
+  std::sort(order.begin(), order.end(), [&](int a, int b) {
+    if (p[a] != p[b]) return p[a] > p[b];
+    return g.topo_pos[a] < g.topo_pos[b];
+  });
+  return order;
+}
+
+// ------------------------------------------------ longest valid path (C3, C4)
+static std::vector<int> longest_valid_path(const Graph& g, const std::vector<char>& unsched,
+                                           const std::vector<int>& rank) {
+  const int n = g.n;
+  std::vector<int64_t> start(n, 0), end(n, 0);
+  std::vector<char> clean(n, 1);
+  // unique successor lists inside G' with max parallel-edge weight
+  std::vector<std::vector<std::pair<int, int64_t>>> succ(n);
+  for (int e = 0; e < (int)g.edges.size(); ++e) {
+    int u = g.edges[e].src, v = g.edges[e].dst;
+    int64_t c = g.edge_cost(e);
+    if (unsched[u] && unsched[v]) {
+      bool found = false;
+      for (auto& sc : succ[u]) if (sc.first == v) { sc.second = std::max(sc.second, c); found = true; }
+      if (!found) succ[u].push_back({v, c});
+    } else if (!unsched[u] && unsched[v]) {
+      start[v] = std::max(start[v], c); clean[v] = 0;
+    } else if (unsched[u] && !unsched[v]) {
+      end[u] = std::max(end[u], c); clean[u] = 0;
+    }
+  }
+  // tail(v): best path starting at v with v not the first vertex.  Among equal
+  // lengths the lexicographically smallest rank sequence wins; since every
+  // candidate starts with v, stopping ([v]) beats continuing ([v, u, ...]),
+  // and between continuations the smaller rank(u) wins.
+  std::vector<int64_t> tl(n, 0);
+  std::vector<int> tn(n, -1);
+  for (int k = n - 1; k >= 0; --k) {
+    int v = g.topo[k];
+    if (!unsched[v]) continue;
+    int64_t bl = g.op_cost(v) + end[v];
+    int bn = -1;
+    if (clean[v]) {
+      for (auto& sc : succ[v]) {
+        int64_t c = g.op_cost(v) + sc.second + tl[sc.first];
+        if (c > bl || (c == bl && bn >= 0 && rank[sc.first] < rank[bn])) { bl = c; bn = sc.first; }
+      }
+    }
+    tl[v] = bl;
+    tn[v] = bn;
+  }
+  int64_t best_len = std::numeric_limits<int64_t>::min();
+  int best_v = -1, best_next = -1;
+  for (int v = 0; v < n; ++v) {
+    if (!unsched[v]) continue;
+    int64_t bl = start[v] + g.op_cost(v) + end[v];
+    int bn = -1;
+    for (auto& sc : succ[v]) {
+      int64_t c = start[v] + g.op_cost(v) + sc.second + tl[sc.first];
+      if (c > bl || (c == bl && bn >= 0 && rank[sc.first] < rank[bn])) { bl = c; bn = sc.first; }
+    }
+    if (bl > best_len || (bl == best_len && rank[v] < rank[best_v])) {
+      best_len = bl; best_v = v; best_next = bn;
+    }
+  }
+  std::vector<int> P{best_v};
+  for (int u = best_next; u >= 0; u = tn[u]) P.push_back(u);
+  return P;
+}
+
+// ------------------------------------ list scheduling (Alg. 1 L10-13, C1, C5)
+static int64_t list_schedule(const Graph& g, const std::vector<int>& gpu, const std::vector<int>& order,
+                             int M, std::vector<std::vector<int>>* seq) {
+  std::vector<int64_t> ready(M, 0), F(g.n, 0);
+  int64_t L = 0;
+  if (seq) seq->assign(M, {});
+  for (int v : order) {
+    int gv = gpu[v];
+    if (gv < 0) continue;
+    int64_t st = ready[gv];
+    for (int e : g.ops[v].in_edges) {
+      int u = g.edges[e].src;
+      if (gpu[u] < 0) continue;
+      st = std::max(st, F[u] + (gpu[u] != gv ? g.edge_cost(e) : 0));
+    }
+    F[v] = st + g.op_cost(v);
+    ready[gv] = F[v];
+    L = std::max(L, F[v]);
+    if (seq) (*seq)[gv].push_back(v);
+  }
+  return L;
+}
+
+// ------------------------------------------------ cost-model simulator (§III)
+SimResult simulate(Graph& g, const std::vector<std::vector<std::vector<int>>>& Q) {
+  SimResult r{false, 0, {}, {}};
+  const int M = (int)Q.size();
+  std::vector<int> base(M + 1, 0);
+  for (int i = 0; i < M; ++i) base[i + 1] = base[i] + (int)Q[i].size();
+  const int NS = base[M];
+  std::vector<int> sid(g.n, -1), sgpu(NS);
+  for (int i = 0; i < M; ++i)
+    for (int j = 0; j < (int)Q[i].size(); ++j) {
+      sgpu[base[i] + j] = i;
+      for (int v : Q[i][j]) sid[v] = base[i] + j;
+    }
+  std::vector<std::vector<std::pair<int, int64_t>>> succ(NS);
+  std::vector<int> indeg(NS, 0);
+  for (int i = 0; i < M; ++i)
+    for (int j = 1; j < (int)Q[i].size(); ++j) {
+      succ[base[i] + j - 1].push_back({base[i] + j, 0});
+      indeg[base[i] + j]++;
+    }
+  for (int e = 0; e < (int)g.edges.size(); ++e) {
+    int su = sid[g.edges[e].src], sv = sid[g.edges[e].dst];
+    if (su < 0 || sv < 0) continue;
+    if (su == sv) return r;  // dependent ops in one stage
+    succ[su].push_back({sv, sgpu[su] != sgpu[sv] ? g.edge_cost(e) : 0});
+    indeg[sv]++;
+  }
+  std::vector<int64_t> start(NS, 0), finish(NS, 0);
+  std::vector<int> stack;
+  for (int s = 0; s < NS; ++s) if (!indeg[s]) stack.push_back(s);
+  int done = 0;
+  while (!stack.empty()) {
+    int s = stack.back(); stack.pop_back();
+    int i = sgpu[s];
+    finish[s] = start[s] + g.stage_cost(Q[i][s - base[i]]);
+    r.L = std::max(r.L, finish[s]);
+    ++done;
+    for (auto& x : succ[s]) {
+      start[x.first] = std::max(start[x.first], finish[s] + x.second);
+      if (--indeg[x.first] == 0) stack.push_back(x.first);
+    }
+  }
+  if (done != NS) return r;  // cycle: deadlock
+  r.ok = true;
+  r.start.resize(M); r.finish.resize(M);
+  for (int i = 0; i < M; ++i) {
+    r.start[i].assign(start.begin() + base[i], start.begin() + base[i + 1]);
+    r.finish[i].assign(finish.begin() + base[i], finish.begin() + base[i + 1]);
+  }
+  return r;
+}
+
+// ------------------------------------------------------ Alg. 2 (C7 - C11)
+static void parallelize(Graph& g, Schedule& s, const std::vector<int>& order) {
+  auto& Q = s.Q;
+  auto r0 = simulate(g, Q);
+  if (!r0.ok) fail(HIOS_E_CYCLE, "inter-GPU schedule deadlocks");
+  int64_t L = r0.L;
+  for (int i = 0; i + 1 < g.n; ++i) {
+    int v = order[i];
+    int gi = -1, j = -1;
+    for (int a = 0; a < (int)Q.size() && gi < 0; ++a)
+      for (int b = 0; b < (int)Q[a].size(); ++b)
+        if (std::find(Q[a][b].begin(), Q[a][b].end(), v) != Q[a][b].end()) { gi = a; j = b; break; }
+    if (Q[gi][j].size() > 1) continue;  // C10: already grouped
+    int64_t best_L = L;
+    std::vector<std::vector<std::vector<int>>> best_Q;
+    bool have = false;
+    std::vector<int> W{v};
+    for (int p = 1; p < s.w; ++p) {
+      if (j + p >= (int)Q[gi].size() || Q[gi][j + p].size() > 1) break;
+      int u = Q[gi][j + p][0];
+      bool ind = true;
+      for (int x : W) ind = ind && g.independent(u, x);
+      if (!ind) break;  // C8: stop growing at the first dependent pair
+      W.push_back(u);
+      auto Q2 = Q;
+      std::vector<std::vector<int>> row(Q2[gi].begin(), Q2[gi].begin() + j);
+      row.push_back(W);
+      row.insert(row.end(), Q2[gi].begin() + j + p + 1, Q2[gi].end());
+      Q2[gi] = std::move(row);
+      auto r2 = simulate(g, Q2);
+      if (!r2.ok) continue;  // C11: merging creates a cycle
+      if (r2.L < best_L) { best_L = r2.L; best_Q = std::move(Q2); have = true; }
+    }
+    if (have) { Q = std::move(best_Q); L = best_L; }  // C9: commit only if L' < L
+  }
+  s.L = L;
+}
+
+// ------------------------------------------------------------ Alg. 1
+void hios_lp(Graph& g, int M, int w, Schedule& s) {
+  s.M = M;
+  s.w = w;
+  auto order = priority_order(g);
+  std::vector<int> rank(g.n);
+  for (int i = 0; i < g.n; ++i) rank[order[i]] = i;
+  std::vector<char> unsched(g.n, 1);
+  int left = g.n;
+  std::vector<int> gpu(g.n, -1);
+  while (left > 0) {
+    auto P = longest_valid_path(g, unsched, rank);
+    for (int v : P) { unsched[v] = 0; --left; }
+    int64_t best_L = std::numeric_limits<int64_t>::max();
+    int best_i = 0;
+    for (int i = 0; i < M; ++i) {
+      for (int v : P) gpu[v] = i;
+      int64_t L2 = list_schedule(g, gpu, order, M, nullptr);
+      if (L2 < best_L) { best_L = L2; best_i = i; }  // Alg. 1 L14: first index wins ties
+    }
+    for (int v : P) gpu[v] = best_i;
+  }
+  std::vector<std::vector<int>> seq;
+  list_schedule(g, gpu, order, M, &seq);
+  s.Q.assign(M, {});
+  for (int i = 0; i < M; ++i)
+    for (int v : seq[i]) s.Q[i].push_back({v});
+  parallelize(g, s, order);  // Alg. 1 L17
+}
+
+void finalize_schedule(Schedule& s) {
+  Graph& g = *s.g;
+  s.gpu_of.assign(g.n, -1);
+  s.stage_of.assign(g.n, -1);
+  for (int i = 0; i < (int)s.Q.size(); ++i)
+    for (int j = 0; j < (int)s.Q[i].size(); ++j) {
+      auto& S = s.Q[i][j];
+      if (S.empty() || (int)S.size() > std::max(s.w, 1))
+        fail(HIOS_E_INVALID, "stage size out of [1, w]");
+      for (size_t a = 0; a < S.size(); ++a) {
+        int v = S[a];
+        if (v < 0 || v >= g.n) fail(HIOS_E_INVALID, "op id out of range");
+        if (s.gpu_of[v] >= 0) fail(HIOS_E_INVALID, "op " + std::to_string(v) + " scheduled twice");
+        s.gpu_of[v] = i;
+        s.stage_of[v] = j;
+        for (size_t b = a + 1; b < S.size(); ++b)
+          if (!g.independent(v, S[b])) fail(HIOS_E_INVALID, "dependent ops in one stage");
+      }
+    }
+  for (int v = 0; v < g.n; ++v)
+    if (s.gpu_of[v] < 0) fail(HIOS_E_INVALID, "op " + std::to_string(v) + " unscheduled");
+  auto r = simulate(g, s.Q);
+  if (!r.ok) fail(HIOS_E_CYCLE, "schedule deadlocks (cycle in the stage graph)");
+  s.L = r.L;
+}
+
+}  // namespace hios

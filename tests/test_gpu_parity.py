@@ -1,0 +1,180 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the CPU oracle on the
+same seeded inputs.  Tolerances (north star): normwise max relative error
+max|y - y_ref| / max|y_ref| <= 2e-2 for bf16, <= 1e-4 for fp32.
+
+Per-op checks feed each op the GPU's own inputs (read back through
+hios_read_op_output) so they isolate one kernel's error; end-to-end checks
+compare the network output with the oracle's sequential inference."""
+import numpy as np
+import pytest
+
+from oracle import infer
+from workloads import gen, graphs
+
+pytestmark = pytest.mark.gpu
+
+TOL = {"bf16": 2e-2, "f32": 1e-4}
+
+
+def hios():
+    from paper_conf_cluster_kundus23_b200 import hios as h
+    return h
+
+
+def nerr(y, ref):
+    den = float(np.abs(ref).max())
+    return float(np.abs(np.asarray(y, np.float64) - ref).max()) / (den if den > 0 else 1.0)
+
+
+def run_graph_gpu(g, W, x, dtype, M=1, w=1, profile=True, costs=None):
+    h = hios()
+    G = h.hios_graph_create(g.ops, g.edges, g.in_c, g.in_h, g.in_w, dtype, W)
+    if profile:
+        h.hios_profile(G, [0], 3)
+    else:
+        for op in g.ops:
+            h.hios_set_op_cost(G, op.id, 1000)
+        for e in range(g.n_edges):
+            h.hios_set_edge_cost(G, e, 1000)
+        h.hios_set_group_model(G, 7, 10)
+    S = h.hios_schedule_lp(G, M, w)
+    y = h.hios_run(S, x)
+    return G, S, y
+
+
+def per_op_check(g, W, S, dtype, skip_kinds=()):
+    """Each op's GPU output vs the oracle op evaluated on the GPU's inputs."""
+    h = hios()
+    outs = {}
+    shapes = {}
+    G = S.graph
+    for op in g.ops:
+        shapes[op.id] = h.hios_graph_shape(G, op.id)
+        outs[op.id] = h.hios_read_op_output(S, op.id, shapes[op.id]).astype(np.float64)
+    worst = {}
+    for op in g.ops:
+        if op.kind == "input" or op.kind in skip_kinds:
+            continue
+        ins = [outs[s] for s in g.preds(op.id)]
+        ref = infer.run_op(op, ins, W[op.id])
+        e = nerr(outs[op.id], ref)
+        worst[op.name] = e
+        assert e <= TOL[dtype], (op.name, op.kind, e)
+    return worst
+
+
+CONV_CASES = [
+    # (C, K, H, W, kh, kw, s, ph, pw)
+    (64, 64, 56, 56, 3, 3, 1, 1, 1),
+    (3, 32, 75, 75, 3, 3, 2, 0, 0),       # stem: C=3, stride 2, odd size
+    (96, 80, 17, 17, 1, 7, 1, 0, 3),      # 1x7
+    (80, 192, 17, 19, 7, 1, 1, 3, 0),     # 7x1, K not a power of 2
+    (288, 384, 35, 35, 3, 3, 2, 0, 0),    # C tail (288 = 4.5 x 64), stride 2
+    (42, 42, 21, 21, 1, 1, 1, 0, 0),      # C, K not multiples of 8
+    (192, 320, 9, 9, 3, 3, 2, 0, 0),
+    (512, 1000, 13, 13, 1, 1, 1, 0, 0),   # classifier-like, K tail over 256 tiles
+    (48, 64, 35, 35, 5, 5, 1, 2, 2),
+]
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+@pytest.mark.parametrize("case", CONV_CASES)
+def test_conv_parity(dtype, case):
+    C, K, H, Wd, kh, kw, s, ph, pw = case
+    g = graphs.GraphSpec("conv", C, H, Wd)
+    x0 = g.input()
+    g.conv(x0, K, (kh, kw), s=s, p=(ph, pw), relu=1)
+    W = gen.make_weights(g)
+    x = gen.make_input(g) - 0.5
+    _, S, y = run_graph_gpu(g, W, x, dtype, profile=False)
+    ref = infer.run_graph(g, W, x)[1]
+    assert nerr(y.reshape(ref.shape), ref) <= TOL[dtype] / (4 if dtype == "bf16" else 1)
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_small_op_zoo(dtype):
+    """pools (ceil / pad / count_include_pad), add (weighted, ReLU), concat
+    (in-place and copied slices), sepconv (aggregation, reps=2, stride 2),
+    gap, linear, identity."""
+    g = graphs.GraphSpec("zoo", 24, 23, 23)
+    x0 = g.input()
+    a = g.conv(x0, 40, 3, p=1)
+    b = g.maxpool(a, 3, 2, 1, ceil_mode=1)
+    c = g.avgpool(a, 3, 2, 1, count_include_pad=0)
+    d = g.avgpool(a, 3, 2, 1, count_include_pad=1)
+    e = g.add([b, c, d], relu=1, agg=1)
+    f = g.sepconv([b, c], 42, 5, s=1, pre_relu=1, relu=1, reps=2)
+    f2 = g.sepconv([e], 40, 3, s=2, pre_relu=1)
+    f3 = g.conv(f2, 40, 1, relu=0)
+    up = g.maxpool(e, 1, 1)
+    cc = g.concat([f, up, e])          # 42-channel slice first: later slices misaligned -> copies
+    cc2 = g.concat([g.identity(cc), f])
+    gp = g.concat([g.gap(cc2), g.gap(f3)])
+    g.linear(gp, 10)
+    W = gen.make_weights(g)
+    x = gen.make_input(g)
+    _, S, y = run_graph_gpu(g, W, x, dtype, profile=False)
+    per_op_check(g, W, S, dtype)
+    ref = infer.run_graph(g, W, x)[g.n_ops - 1].reshape(-1)
+    assert nerr(y, ref) <= TOL[dtype]
+
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+@pytest.mark.parametrize("M,w", [(1, 1), (2, 2), (4, 3)])
+def test_tiny_end_to_end(dtype, M, w):
+    """configs[0]: Fig.-4-topology conv DAG, 1x64x56x56; multi-GPU schedules run
+    on logical GPUs aliased onto cuda:0 (same flags / peer-store code path)."""
+    g = graphs.tiny()
+    W = gen.make_weights(g)
+    x = gen.make_input(g)
+    _, S, y = run_graph_gpu(g, W, x, dtype, M=M, w=w)
+    ref = infer.run_graph(g, W, x)[g.n_ops - 1].reshape(-1)
+    assert nerr(y, ref) <= TOL[dtype]
+    per_op_check(g, W, S, dtype)
+
+
+@pytest.mark.parametrize("name,size", [("inception_v3", 299), ("squeezenet", 224),
+                                       ("randwire_ws", 224), ("nasnet_a_large", 331)])
+def test_benchmark_end_to_end_bf16(name, size):
+    g = graphs.build(name, size)
+    W = gen.make_weights(g)
+    x = gen.make_input(g)
+    _, S, y = run_graph_gpu(g, W, x, "bf16", M=1, w=3)
+    per_op_check(g, W, S, "bf16")
+    ref = infer.run_graph(g, W, x, keep={g.n_ops - 1})[g.n_ops - 1].reshape(-1)
+    assert nerr(y, ref) <= TOL["bf16"]
+
+
+@pytest.mark.parametrize("name,size", [("inception_v3", 299), ("randwire_ws", 224)])
+def test_multi_gpu_schedules_bit_identical(name, size):
+    """Placement never changes arithmetic: M = 2, 4, 8 logical GPUs (aliased)
+    give bit-identical outputs to the single-GPU sequential schedule."""
+    g = graphs.build(name, size)
+    W = gen.make_weights(g)
+    x = gen.make_input(g)
+    _, _, y1 = run_graph_gpu(g, W, x, "bf16", M=1, w=1)
+    for M, w in [(2, 2), (4, 3), (8, 3)]:
+        _, S, yM = run_graph_gpu(g, W, x, "bf16", M=M, w=w)
+        assert np.array_equal(y1, yM), (M, w)
+
+
+def test_inception_fp32_end_to_end():
+    g = graphs.inception_v3(299)
+    W = gen.make_weights(g)
+    x = gen.make_input(g)
+    _, S, y = run_graph_gpu(g, W, x, "f32", M=2, w=2)
+    ref = infer.run_graph(g, W, x, keep={g.n_ops - 1})[g.n_ops - 1].reshape(-1)
+    assert nerr(y, ref) <= TOL["f32"]
+
+
+def test_inception_1024_bench_config():
+    """configs[1] at full size (1x3x1024x1024) in the bench's launch
+    configuration (profiled HIOS-LP, M=1, w=3): logits vs the oracle."""
+    g = graphs.inception_v3(1024)
+    W = gen.make_weights(g)
+    x = gen.make_input(g)
+    _, S, y = run_graph_gpu(g, W, x, "bf16", M=1, w=3)
+    ref = infer.run_graph(g, W, x, keep={g.n_ops - 1})[g.n_ops - 1].reshape(-1)
+    assert nerr(y, ref) <= TOL["bf16"]
+    # repeated runs are deterministic
+    assert np.array_equal(y, hios().hios_run(S, x))
