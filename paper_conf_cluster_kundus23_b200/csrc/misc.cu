@@ -186,10 +186,12 @@ __global__ void copy_kernel(const CopyArgs<T> a) {
   const long long pix = idx / CG;
   const T* src = a.x + pix * a.ldx + c;
   T* dst = a.out + pix * a.ldo + c;
-  if (c + N <= a.C) {
+  // concat slices at channel offsets that are not multiples of 8 are not
+  // 16-byte aligned: fall back to element copies there
+  if (c + N <= a.C && ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15) == 0) {
     *reinterpret_cast<uint4*>(dst) = *reinterpret_cast<const uint4*>(src);
   } else {
-    for (int j = 0; c + j < a.C; ++j) dst[j] = src[j];
+    for (int j = 0; j < N && c + j < a.C; ++j) dst[j] = src[j];
   }
 }
 
