@@ -1,20 +1,31 @@
-// conv_tc.cu -- implicit-GEMM convolution on Blackwell 5th-gen tensor cores.
+// conv_tc.cu -- implicit-GEMM convolution on Blackwell 5th-gen tensor cores
+// ("convolution ... operators" of G).
 //
-// One CTA = one 128-pixel x BLOCK_N output tile.  Warp roles (128 threads):
-//   warp 0 lane 0  TMA producer: per K-step (r, s, 64-channel chunk) one 3-D
-//                  box of the NHWC input at the (r,s)-shifted window with the
-//                  conv stride as the TMA traversal stride (OOB -> zero, i.e.
-//                  the conv padding) and one box of the [K][R*S][Cp] weights,
-//                  both 128B-swizzled K-major, into a `stages`-deep ring
-//   warp 1 lane 0  MMA issuer: 4 x tcgen05.mma.kind::f16 (M=128, N=BLOCK_N,
-//                  K=16) per K-step into the TMEM accumulator; tcgen05.commit
-//                  frees the smem slot
-//   warp 2         TMEM allocator (BLOCK_N fp32 columns)
-//   warps 0-3      epilogue: tcgen05.ld 32 lanes x 16 columns -> folded-BN
-//                  scale/shift -> ReLU -> bf16 -> 16-byte stores into the
-//                  destination (local buffer, concat slice, and optionally a
-//                  peer GPU's replica: the transfer fused into the epilogue)
-// SURVEY §8(a) a8; PAPER.md P:80 (conv operators of G).
+// GEMM view: M = output pixels, N = output channels, K = R*S*C.  bf16
+// operands, fp32 accumulation in TMEM, folded-BN scale/shift + ReLU + bf16
+// epilogue.  Persistent, warp-specialised CTA (192 threads):
+//   warp 0      TMA producer (one elected lane)
+//   warp 1      MMA issuer (one elected lane): 4 x tcgen05.mma.kind::f16
+//               (M=128, N=n_tile, K=16) per K-step
+//   warps 2-5   epilogue: tcgen05.ld -> scale/shift/ReLU -> bf16 -> stores
+//               to the local buffer / concat slice and, optionally, a peer
+//               GPU's replica (cross-GPU edge fused into the epilogue)
+// Two TMEM accumulators (2 x n_tile columns) let the epilogue of tile i run
+// under the main loop of tile i+1.  Tiles are walked N-fastest so CTAs that
+// share an input tile run together (L2 reuse).
+//
+// Operand staging (both 128B-swizzled, K-major, by TMA):
+//   halo mode  (stride 1 along W, one output row of 128 pixels per tile):
+//              per 64-channel chunk ONE box of R input rows x (128+(S-1)dw)
+//              pixels; the A operand of tap (r, s) is the row window starting
+//              at pixel r*Wh + s*dw of that box (descriptor start + base
+//              offset), so every input pixel crosses L2->SM once per tile
+//              instead of R*S times; B (weights of one tap) streams through
+//              a ring.
+//   tap mode   (generic: strides, narrow outputs): per K-step (r, s, chunk)
+//              one box of th x tw output positions of the (r,s)-shifted input
+//              with the conv stride as TMA traversal stride, plus B.
+// Out-of-bounds TMA reads return zero = the convolution's zero padding.
 #include <cstdio>
 
 #include "kernels.cuh"
@@ -29,6 +40,9 @@ __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
 }
 __device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   asm volatile(
@@ -52,14 +66,19 @@ __device__ __forceinline__ void tma_load_3d(uint32_t dst, const CUtensorMap* map
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 
-// UMMA shared-memory descriptor: K-major, 128B swizzle, 8-row atoms 1024 B apart.
-__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) {
+// UMMA shared-memory descriptor: K-major, 128B swizzle, 8-row atoms 1024 B
+// apart.  The swizzle phase follows the absolute smem address bits [7,10), so
+// a window starting at any 128-byte row of a TMA-written (same-swizzle) box is
+// addressed with base offset 0 (measured on B200: a non-zero base offset
+// breaks the shifted halo windows).
+__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr, int bo_mode = 0) {
   uint64_t d = 0;
-  d |= (uint64_t)((saddr & 0x3FFFFu) >> 4);  // start address  [0,14)
-  d |= (uint64_t)1 << 16;                    // LBO (unused for swizzled K-major) [16,30)
-  d |= (uint64_t)(1024 >> 4) << 32;          // SBO = 1024 B   [32,46)
-  d |= (uint64_t)1 << 46;                    // descriptor version (sm_100)
-  d |= (uint64_t)2 << 61;                    // SWIZZLE_128B
+  d |= (uint64_t)((saddr & 0x3FFFFu) >> 4);        // start address  [0,14)
+  d |= (uint64_t)1 << 16;                          // LBO (unused for swizzled K-major)
+  d |= (uint64_t)(1024 >> 4) << 32;                // SBO = 1024 B
+  d |= (uint64_t)1 << 46;                          // descriptor version (sm_100)
+  if (bo_mode) d |= (uint64_t)((saddr >> 7) & 7u) << 49;  // (measured: must stay 0)
+  d |= (uint64_t)2 << 61;                          // SWIZZLE_128B
   return d;
 }
 
@@ -87,13 +106,31 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
+// optional timeline instrumentation (HIOS_TRACE): globaltimer at checkpoints
+__device__ unsigned long long g_conv_trace[256 * 8];
+__device__ unsigned long long g_conv_trace2[32 * 48];  // per CTA: issue[16], full[16], empty_ok[16]
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#define TRACE2(slot, k)                                                   \
+  do {                                                                    \
+    if (a.trace && blockIdx.x < 32 && (k) < 16) g_conv_trace2[blockIdx.x * 48 + (slot) * 16 + (k)] = gtimer(); \
+  } while (0)
+#define TRACE(k)                                                          \
+  do {                                                                    \
+    if (a.trace && blockIdx.x < 256) g_conv_trace[blockIdx.x * 8 + (k)] = gtimer(); \
+  } while (0)
+
 static __host__ __device__ inline uint32_t tmem_cols(int n) {
   uint32_t c = 32;
   while ((int)c < n) c <<= 1;
   return c;
 }
 
-__global__ void __launch_bounds__(128, 1)
+
+__global__ void __launch_bounds__(192, 1)
     conv_tc_kernel(const __grid_constant__ CUtensorMap mx, const __grid_constant__ CUtensorMap mw,
                    const ConvTcArgs a) {
   extern __shared__ uint8_t smem_raw[];
@@ -101,28 +138,39 @@ __global__ void __launch_bounds__(128, 1)
   const int ST = a.stages;
   const uint32_t A_BYTES = 128 * 128;
   const uint32_t B_BYTES = (uint32_t)a.n_tile * 128;
-  uint8_t* sA = smem;
-  uint8_t* sB = smem + ST * A_BYTES;
+  const uint32_t H_BYTES = a.halo ? halo_bytes_of(a.R, a.halo_w) : 0u;
+  uint8_t* sA = smem;  // halo: a_bufs x H_BYTES ; tap: ST x A_BYTES
+  uint8_t* sB = smem + (a.halo ? a.a_bufs * H_BYTES : ST * A_BYTES);
   uint64_t* bars = reinterpret_cast<uint64_t*>(sB + ST * B_BYTES);
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * ST + 1);
-  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + ST), accum = smem_u32(bars + 2 * ST);
+  // barriers: full[ST] empty[ST] afull[2] aempty[2] tfull[2] tempty[2]
+  const uint32_t full0 = smem_u32(bars), empty0 = full0 + 8 * ST;
+  const uint32_t afull0 = empty0 + 8 * ST, aempty0 = afull0 + 16, tfull0 = aempty0 + 16, tempty0 = tfull0 + 16;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * ST + 8);
+  float* s_scale = reinterpret_cast<float*>(bars + 2 * ST + 10);  // [256]
+  float* s_shift = s_scale + 256;                                  // [256]
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int tp = blockIdx.x / a.tiles_q, tq = blockIdx.x % a.tiles_q;
-  const int p0 = tp * a.th, q0 = tq * a.tw, n0 = blockIdx.y * a.n_tile;
-  const uint32_t ncols = tmem_cols(a.n_tile);
+  const uint32_t ncols = tmem_cols(2 * a.n_tile);
+  const int RS = a.R * a.S;
+  const int tiles = a.tiles_m * a.tiles_n;
+  if (threadIdx.x == 0) TRACE(0);
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < ST; ++i) {
       mbar_init(full0 + 8 * i, 1);
       mbar_init(empty0 + 8 * i, 1);
     }
-    mbar_init(accum, 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(afull0 + 8 * i, 1);
+      mbar_init(aempty0 + 8 * i, 1);
+      mbar_init(tfull0 + 8 * i, 1);
+      mbar_init(tempty0 + 8 * i, 128);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mx)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mw)) : "memory");
   }
-  if (warp == 2) {
+  if (warp == 1) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                  "r"(ncols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -131,99 +179,189 @@ __global__ void __launch_bounds__(128, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  if (threadIdx.x == 0) TRACE(1);
 
-  const int KI = a.R * a.S * a.c_chunks;
-  if (warp == 0 && lane == 0) {
-    // ---------------- TMA producer
-    for (int ki = 0; ki < KI; ++ki) {
-      const int st = ki % ST;
-      const uint32_t ph = (uint32_t)(ki / ST) & 1u;
-      mbar_wait(empty0 + 8 * st, ph ^ 1u);
-      mbar_expect_tx(full0 + 8 * st, A_BYTES + B_BYTES);
-      const int rs = ki / a.c_chunks, cc = ki - rs * a.c_chunks;
-      const int r = rs / a.S, s = rs - r * a.S;
-      tma_load_3d(smem_u32(sA + st * A_BYTES), &mx, full0 + 8 * st, cc * 64, q0 * a.sw - a.pw + s * a.dw,
-                  p0 * a.sh - a.ph + r * a.dh);
-      tma_load_3d(smem_u32(sB + st * B_BYTES), &mw, full0 + 8 * st, cc * 64, rs, n0);
+  if (warp == 0) {
+    if (lane == 0) {
+      // ------------------------------------------------------ TMA producer
+      // (single thread: every division is hoisted out of the K loop; stage,
+      //  phase, tap and chunk advance incrementally)
+      uint32_t st = 0, ph = 0, ab = 0, aph = 0, ks = 0;
+      const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
+      for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+        const int m_blk = tile / a.tiles_n, n_blk = tile - m_blk * a.tiles_n;
+        const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
+        const int p0 = tp * a.th, q0 = tq * a.tw, n0 = n_blk * a.n_tile;
+        const int x0 = q0 * a.sw - a.pw, y0 = p0 * a.sh - a.ph;
+        for (int cc = 0; cc < a.c_chunks; ++cc) {
+          const int c0 = cc * 64;
+          if (a.halo) {
+            mbar_wait(aempty0 + 8 * ab, aph ^ 1u);
+            mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.R * a.halo_w * 128u);
+            tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, c0, x0, y0);
+            if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
+          }
+          int r = 0, s = 0;
+          for (int rs = 0; rs < RS; ++rs, ++ks) {
+            mbar_wait(empty0 + 8 * st, ph ^ 1u);
+            TRACE2(2, ks);
+            if (a.halo) {
+              mbar_expect_tx(full0 + 8 * st, B_BYTES);
+            } else {
+              mbar_expect_tx(full0 + 8 * st, A_BYTES + B_BYTES);
+              tma_load_3d(sA0 + st * A_BYTES, &mx, full0 + 8 * st, c0, x0 + s * a.dw, y0 + r * a.dh);
+            }
+            tma_load_3d(sB0 + st * B_BYTES, &mw, full0 + 8 * st, c0, rs, n0);
+            if (ks == 0) TRACE(2);
+            TRACE2(0, ks);
+            if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
+            if (++s == a.S) { s = 0; ++r; }
+          }
+        }
+      }
     }
-  } else if (warp == 1 && lane == 0) {
-    // ---------------- MMA issuer (single thread)
-    const uint32_t idesc = (1u << 4)                             // D format f32
-                           | (1u << 7)                           // A bf16
-                           | (1u << 10)                          // B bf16
-                           | ((uint32_t)(a.n_tile >> 3) << 17)   // N
-                           | ((uint32_t)(128 >> 4) << 24);       // M = 128
-    for (int ki = 0; ki < KI; ++ki) {
-      const int st = ki % ST;
-      const uint32_t ph = (uint32_t)(ki / ST) & 1u;
-      mbar_wait(full0 + 8 * st, ph);
+    __syncwarp();
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // ------------------------------------------------------ MMA issuer
+      const uint32_t idesc = (1u << 4)                            // D f32
+                             | (1u << 7)                          // A bf16
+                             | (1u << 10)                         // B bf16
+                             | ((uint32_t)(a.n_tile >> 3) << 17)  // N
+                             | ((uint32_t)(128 >> 4) << 24);      // M = 128
+      uint32_t st = 0, ph = 0, ab = 0, aph = 0, ks = 0, acc = 0, tph = 0;
+      const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
+      // halo mode: A window of tap (r, s) starts (r * halo_w + s * dw) rows in
+      const uint32_t row_r = (uint32_t)a.halo_w * 128u, row_s = (uint32_t)a.dw * 128u;
+      int tcount = 0;
+      for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
+        mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
+        tc_fence_after();
+        const uint32_t d = tmem + acc * (uint32_t)a.n_tile;
+        uint32_t accum = 0;
+        for (int cc = 0; cc < a.c_chunks; ++cc) {
+          const uint32_t abase = sA0 + ab * H_BYTES;
+          if (a.halo) {
+            mbar_wait(afull0 + 8 * ab, aph);
+            tc_fence_after();
+          }
+          uint32_t aoff_r = 0, aoff = 0;
+          int s = 0;
+          for (int rs = 0; rs < RS; ++rs, ++ks) {
+            mbar_wait(full0 + 8 * st, ph);
+            tc_fence_after();
+            if (ks == 0) TRACE(3);
+            TRACE2(1, ks);
+            const uint32_t a_addr = a.halo ? abase + aoff : sA0 + st * A_BYTES;
+            const uint64_t ad = umma_desc_sw128(a_addr, a.bo_mode);
+            const uint64_t bd = umma_desc_sw128(sB0 + st * B_BYTES);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {  // 4 x K=16 inside the 128-byte swizzle row
+              mma_bf16(d, ad + 2 * k, bd + 2 * k, idesc, accum | (uint32_t)k);
+            }
+            accum = 1;
+            mma_commit(empty0 + 8 * st);
+            if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
+            if (++s == a.S) { s = 0; aoff_r += row_r; aoff = aoff_r; } else { aoff += row_s; }
+          }
+          if (a.halo) {
+            mma_commit(aempty0 + 8 * ab);
+            if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
+          }
+        }
+        mma_commit(tfull0 + 8 * acc);
+        if (tcount == 0) TRACE(4);
+        acc ^= 1u;
+        if (acc == 0) tph ^= 1u;
+      }
+    }
+    __syncwarp();
+  } else {
+    // -------------------------------------------------------- epilogue
+    const int lw = warp & 3;  // TMEM lane quarter this warp may access
+    const int m = lw * 32 + lane;
+    uint32_t tcount = 0, acc = 0, tph = 0;
+    const int hh = m / a.tw, ww = m - hh * a.tw;
+    for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
+      const int m_blk = tile / a.tiles_n, n_blk = tile - m_blk * a.tiles_n;
+      const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
+      const int p0 = tp * a.th, q0 = tq * a.tw, n0 = n_blk * a.n_tile;
+      // stage this tile's folded-BN scale/shift in smem (overlaps the main loop)
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      for (int j = threadIdx.x - 64; j < a.n_tile; j += 128) {
+        const int nj = min(n0 + j, a.K - 1);
+        s_scale[j] = __ldg(a.scale + nj);
+        s_shift[j] = __ldg(a.shift + nj);
+      }
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      mbar_wait(tfull0 + 8 * acc, tph);
+      __syncwarp();
       tc_fence_after();
-      const uint64_t ad = umma_desc_sw128(smem_u32(sA + st * A_BYTES));
-      const uint64_t bd = umma_desc_sw128(smem_u32(sB + st * B_BYTES));
+      if (tcount == 0 && warp == 2 && lane == 0) TRACE(5);
+      const int p = p0 + hh, q = q0 + ww;
+      const bool valid = p < a.P && q < a.Q;
+      const size_t pix = (size_t)p * a.Q + q;
+      const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)a.n_tile;
+      for (int col = 0; col < a.n_tile; col += 16) {
+        uint32_t r[16];
+        tmem_ld16(tbase + (uint32_t)col, r);
+        const int n = n0 + col;
+        if (!valid || n >= a.K) continue;
+        float v[16];
 #pragma unroll
-      for (int k = 0; k < 4; ++k)  // 4 x K=16 inside the 128-byte swizzle row
-        mma_bf16(tmem, ad + 2 * k, bd + 2 * k, idesc, (ki | k) != 0);
-      mma_commit(empty0 + 8 * st);
-    }
-    mma_commit(accum);
-  }
-  // ---------------- epilogue (all 4 warps; warp w owns TMEM lanes 32w..32w+31)
-  mbar_wait(accum, 0);
-  __syncwarp();
-  tc_fence_after();
-  const int m = warp * 32 + lane;
-  const int hh = m / a.tw, ww = m - hh * a.tw;
-  const int p = p0 + hh, q = q0 + ww;
-  const bool valid = p < a.P && q < a.Q;
-  const size_t pix = (size_t)p * a.Q + q;
-  for (int col = 0; col < a.n_tile; col += 16) {
-    uint32_t r[16];
-    tmem_ld16(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)col, r);
-    const int n = n0 + col;
-    if (!valid || n >= a.K) continue;
-    float v[16];
+        for (int j = 0; j < 16; ++j) {
+          float y = __uint_as_float(r[j]) * s_scale[col + j] + s_shift[col + j];
+          v[j] = a.relu ? fmaxf(y, 0.f) : y;
+        }
+        if (n + 16 <= a.K) {
+          uint32_t pk[8];
 #pragma unroll
-    for (int j = 0; j < 16; ++j) {
-      const int nj = min(n + j, a.K - 1);
-      float y = __uint_as_float(r[j]) * __ldg(a.scale + nj) + __ldg(a.shift + nj);
-      v[j] = a.relu ? fmaxf(y, 0.f) : y;
-    }
-    if (n + 16 <= a.K) {
-      uint32_t pk[8];
+          for (int j = 0; j < 8; ++j) {
+            __nv_bfloat162 b2 = __floats2bfloat162_rn(v[2 * j], v[2 * j + 1]);
+            pk[j] = *reinterpret_cast<uint32_t*>(&b2);
+          }
+          uint4* dst = reinterpret_cast<uint4*>(a.out + pix * a.ldo + n);
+          dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+          dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+          if (a.out2) {
+            uint4* d2 = reinterpret_cast<uint4*>(a.out2 + pix * a.ldo2 + n);
+            d2[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+            d2[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+          }
+        } else {
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        __nv_bfloat162 b2 = __floats2bfloat162_rn(v[2 * j], v[2 * j + 1]);
-        pk[j] = *reinterpret_cast<uint32_t*>(&b2);
+          for (int j = 0; j < 16; ++j) {
+            if (n + j < a.K) {
+              a.out[pix * a.ldo + n + j] = __float2bfloat16_rn(v[j]);
+              if (a.out2) a.out2[pix * a.ldo2 + n + j] = __float2bfloat16_rn(v[j]);
+            }
+          }
+        }
       }
-      uint4* d = reinterpret_cast<uint4*>(a.out + pix * a.ldo + n);
-      d[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-      d[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
-      if (a.out2) {
-        uint4* d2 = reinterpret_cast<uint4*>(a.out2 + pix * a.ldo2 + n);
-        d2[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-        d2[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
-      }
-    } else {
-      for (int j = 0; j < 16 && n + j < a.K; ++j) {
-        a.out[pix * a.ldo + n + j] = __float2bfloat16_rn(v[j]);
-        if (a.out2) a.out2[pix * a.ldo2 + n + j] = __float2bfloat16_rn(v[j]);
-      }
+      tc_fence_before();
+      mbar_arrive(tempty0 + 8 * acc);
+      if (tcount == 0 && warp == 2 && lane == 0) TRACE(6);
+      acc ^= 1u;
+      if (acc == 0) tph ^= 1u;
     }
   }
   tc_fence_before();
   __syncthreads();
-  if (warp == 2) {
+  if (threadIdx.x == 0) TRACE(7);
+  if (warp == 1) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(ncols));
   }
 }
 
-size_t conv_tc_smem_bytes(int n_tile, int stages) {
-  return 1024 + (size_t)stages * (128 * 128 + (size_t)n_tile * 128) + (2 * stages + 1) * 8 + 16;
+size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
+  const size_t B = (size_t)a.n_tile * 128;
+  const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.R, a.halo_w) : (size_t)a.stages * 128 * 128;
+  return 1024 + A + (size_t)a.stages * B + (2 * a.stages + 10) * 8 + 2 * 256 * 4;
 }
 
-void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcArgs& a, int n_tiles_m,
-                    int n_tiles_n, size_t smem, cudaStream_t st) {
+void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcArgs& a, int grid, size_t smem,
+                    cudaStream_t st) {
   static bool attr_set[64] = {false};
   int dev = 0;
   cudaGetDevice(&dev);
@@ -231,9 +369,25 @@ void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcAr
     cudaFuncSetAttribute(conv_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr_set[dev] = true;
   }
-  conv_tc_kernel<<<dim3(n_tiles_m, n_tiles_n), 128, smem, st>>>(mx, mw, a);
+  conv_tc_kernel<<<grid, 192, smem, st>>>(mx, mw, a);
 }
 
+}  // namespace hios
+
+extern "C" int hios_debug_conv_trace_reset(void) {
+  static unsigned long long zero[2048];
+  return (int)cudaMemcpyToSymbol(hios::g_conv_trace, zero, sizeof(zero));
+}
+
+extern "C" int hios_debug_conv_trace2(unsigned long long* out) {
+  return (int)cudaMemcpyFromSymbol(out, hios::g_conv_trace2, sizeof(unsigned long long) * 32 * 48);
+}
+
+extern "C" int hios_debug_conv_trace(unsigned long long* out, int n) {
+  return (int)cudaMemcpyFromSymbol(out, hios::g_conv_trace, sizeof(unsigned long long) * (n < 2048 ? n : 2048));
+}
+
+namespace hios {
 // ------------------------------------------------------------ tensor maps
 typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                      const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,

@@ -13,6 +13,8 @@
 //     which is what the paper's MPI engine lacked
 //   * stages of different GPUs are not synchronised otherwise
 #include <algorithm>
+#include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <numeric>
 #include <set>
@@ -276,33 +278,58 @@ void Executor::allocate() {
 }
 
 // --------------------------------------------------------------- closures
-struct ConvPlan {
-  int th, tw, tiles_q, tiles_m, n_tile, tiles_n, stages;
-  size_t smem;
-};
-
-static ConvPlan plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh, int sw) {
-  ConvPlan c{};
-  int64_t best = -1;
-  for (int tw : {128, 64, 32, 16, 8}) {
-    const int th = 128 / tw;
-    if (tw * sw > 256 || th * sh > 256) continue;
-    const int64_t cost = (int64_t)((P + th - 1) / th) * th * ((Q + tw - 1) / tw) * tw;
-    if (best < 0 || cost < best) { best = cost; c.th = th; c.tw = tw; }
+// Tile plan of one tcgen05 conv (see conv_tc.cu): halo mode for stride-1-in-W
+// convs with wide outputs, tap mode otherwise; n_tile from a small cost model
+// (waves x per-K-step time, where a K-step costs max(MMA, L2->SM bytes)).
+static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh, int sw, int dh, int dw) {
+  ConvTcArgs c{};
+  const int hw = 128 + (S - 1) * dw;
+  c.halo = (sw == 1 && Q >= 96 && hw <= 256 && R * dh <= 256 && halo_bytes_of(R, hw) <= 100 * 1024) ? 1 : 0;
+  if (c.halo) {
+    c.th = 1;
+    c.tw = 128;
+    c.halo_w = hw;
+  } else {
+    int64_t best = -1;
+    for (int tw : {128, 64, 32, 16, 8}) {
+      const int th = 128 / tw;
+      if (tw * sw > 256 || th * sh > 256) continue;
+      const int64_t cost = (int64_t)((P + th - 1) / th) * th * ((Q + tw - 1) / tw) * tw;
+      if (best < 0 || cost < best) { best = cost; c.th = th; c.tw = tw; }
+    }
+    if (best < 0) fail(HIOS_E_UNSUPPORTED, "conv stride too large for the TMA box");
   }
-  if (best < 0) fail(HIOS_E_UNSUPPORTED, "conv stride too large for the TMA box");
   c.tiles_q = (Q + c.tw - 1) / c.tw;
   c.tiles_m = ((P + c.th - 1) / c.th) * c.tiles_q;
-  const int nb = (K + 255) / 256;
-  c.n_tile = rup((K + nb - 1) / nb, 16);
-  while ((int64_t)c.tiles_m * ((K + c.n_tile - 1) / c.n_tile) < 148 && c.n_tile > 32)
-    c.n_tile = rup(c.n_tile / 2, 16);
+  c.c_chunks = (C + 63) / 64;
+  const int KI = R * S * c.c_chunks;
+  const double a_bytes = c.halo ? (double)R * hw * 128.0 / (R * S) : 16384.0;
+  double best_cost = 1e300;
+  for (int nt = 16; nt <= 256; nt += 16) {
+    if (nt > rup(K, 16)) break;
+    const int tn = (K + nt - 1) / nt;
+    const double waves = std::ceil((double)c.tiles_m * tn / 148.0);
+    const double kstep = std::max(2.0 * nt, (a_bytes + nt * 128.0) / 128.0) + 40.0;
+    const double cost = waves * (KI * kstep + 600.0);
+    if (cost < best_cost * 0.999) { best_cost = cost; c.n_tile = nt; }
+  }
   c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
-  const int KI = R * S * ((C + 63) / 64);
-  const size_t stage_bytes = 16384 + (size_t)c.n_tile * 128;
-  c.stages = (int)std::min<size_t>(8, (200 * 1024 - 2048) / stage_bytes);
+  const size_t B = (size_t)c.n_tile * 128;
+  const size_t budget = 200 * 1024;
+  if (c.halo) {
+    const size_t H = halo_bytes_of(R, hw);
+    c.a_bufs = (2 * H + 2 * B <= budget) ? 2 : 1;
+    c.stages = (int)std::min<size_t>(8, (budget - c.a_bufs * H) / B);
+  } else {
+    c.stages = (int)std::min<size_t>(6, budget / (16384 + B));
+  }
   c.stages = std::max(2, std::min(c.stages, std::max(KI, 2)));
-  c.smem = conv_tc_smem_bytes(c.n_tile, c.stages);
+  // debug overrides for tuning experiments (tools/conv_micro.py)
+  if (getenv("HIOS_NTILE")) {
+    c.n_tile = std::min(256, rup(atoi(getenv("HIOS_NTILE")), 16));
+    c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
+  }
+  if (getenv("HIOS_STAGES")) c.stages = std::max(2, atoi(getenv("HIOS_STAGES")));
   return c;
 }
 
@@ -323,22 +350,33 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor&, const View& in, 
                                                      float* scale, float* shift, int K, int R, int S, int sh, int sw,
                                                      int ph, int pw, int dh, int dw, int P, int Q, int relu,
                                                      const View& out, const View* out2, int& nk) {
-  ConvPlan cp = plan_conv_tc(P, Q, K, C, R, S, sh, sw);
+  ConvTcArgs a = plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw);
+  if (getenv("HIOS_NOHALO") && a.halo) {  // debug: force tap mode on the same tiles
+    a.halo = 0;
+    a.stages = std::max(2, std::min(a.stages, (int)((200 * 1024) / (16384 + a.n_tile * 128))));
+  }
   CUtensorMap mx, mw;
-  if (!make_tmap_3d(&mx, in.p, C, W, H, (uint64_t)in.ldc * 2, (uint64_t)W * in.ldc * 2, 64, cp.tw * sw, cp.th * sh,
-                    sw, sh))
-    fail(HIOS_E_CUDA, "tensor map (activation)");
+  bool ok;
+  if (a.halo)  // R input rows (stride dh) x halo_w pixels per channel chunk
+    ok = make_tmap_3d(&mx, in.p, C, W, H, (uint64_t)in.ldc * 2, (uint64_t)W * in.ldc * 2, 64, a.halo_w, R * dh, 1,
+                      dh);
+  else         // th x tw output positions of one (r, s) tap, conv stride as traversal stride
+    ok = make_tmap_3d(&mx, in.p, C, W, H, (uint64_t)in.ldc * 2, (uint64_t)W * in.ldc * 2, 64, a.tw * sw, a.th * sh,
+                      sw, sh);
+  if (!ok) fail(HIOS_E_CUDA, "tensor map (activation)");
   const int Cp = rup(C, 8);
-  if (!make_tmap_3d(&mw, w, Cp, R * S, K, (uint64_t)Cp * 2, (uint64_t)R * S * Cp * 2, 64, 1, cp.n_tile, 1, 1))
+  if (!make_tmap_3d(&mw, w, Cp, R * S, K, (uint64_t)Cp * 2, (uint64_t)R * S * Cp * 2, 64, 1, a.n_tile, 1, 1))
     fail(HIOS_E_CUDA, "tensor map (weights)");
-  ConvTcArgs a{};
   a.P = P; a.Q = Q; a.K = K; a.C = C; a.R = R; a.S = S; a.sh = sh; a.sw = sw; a.ph = ph; a.pw = pw;
-  a.dh = dh; a.dw = dw; a.th = cp.th; a.tw = cp.tw; a.tiles_q = cp.tiles_q; a.n_tile = cp.n_tile;
-  a.c_chunks = (C + 63) / 64; a.stages = cp.stages; a.relu = relu; a.scale = scale; a.shift = shift;
+  a.dh = dh; a.dw = dw; a.relu = relu; a.scale = scale; a.shift = shift;
+  a.bo_mode = getenv("HIOS_BO") ? atoi(getenv("HIOS_BO")) : 0;
+  a.trace = getenv("HIOS_TRACE") ? 1 : 0;
   a.out = (bf16*)out.p; a.ldo = out.ldc;
   a.out2 = out2 ? (bf16*)out2->p : nullptr; a.ldo2 = out2 ? out2->ldc : 0;
+  const size_t smem = conv_tc_smem_bytes(a);
+  const int grid = std::min(a.tiles_m * a.tiles_n, 148);
   nk += 1;
-  return [mx, mw, a, cp](cudaStream_t st) { launch_conv_tc(mx, mw, a, cp.tiles_m, cp.tiles_n, cp.smem, st); };
+  return [mx, mw, a, smem, grid](cudaStream_t st) { launch_conv_tc(mx, mw, a, grid, smem, st); };
 }
 
 template <>

@@ -23,7 +23,10 @@ typedef __nv_bfloat16 bf16;
 // the [K][R*S][Cp] weights.
 struct ConvTcArgs {
   int P, Q, K, C, R, S, sh, sw, ph, pw, dh, dw;
-  int th, tw, tiles_q, n_tile, c_chunks, stages, relu;
+  int th, tw, tiles_q, tiles_m, tiles_n, n_tile, c_chunks, stages, relu;
+  int halo, halo_w, a_bufs;  // halo mode: one R x halo_w input box per channel chunk
+  int bo_mode;               // descriptor base-offset encoding (debug switch, 0)
+  int trace;                 // write a globaltimer timeline (debug)
   const float* scale;  // [K]
   const float* shift;  // [K]
   bf16* out;  int ldo; // primary output (channel offset applied)
@@ -72,9 +75,12 @@ struct CopyArgs {
 };
 
 // launchers (stream-ordered, capture-safe)
-void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcArgs& a, int n_tiles_m,
-                    int n_tiles_n, size_t smem, cudaStream_t st);
-size_t conv_tc_smem_bytes(int n_tile, int stages);
+void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcArgs& a, int grid, size_t smem,
+                    cudaStream_t st);
+size_t conv_tc_smem_bytes(const ConvTcArgs& a);
+__host__ __device__ inline uint32_t halo_bytes_of(int R, int halo_w) {
+  return ((uint32_t)R * halo_w * 128u + 1023u) & ~1023u;
+}
 void launch_conv_simt(const ConvSimtArgs& a, cudaStream_t st);
 template <typename T> void launch_dw(const DwArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_pool(const PoolArgs<T>& a, cudaStream_t st);

@@ -56,11 +56,11 @@ template <typename T>
 __global__ void pool_kernel(const PoolArgs<T> a) {
   constexpr int N = Vec<T>::N;
   const int CG = (a.C + N - 1) / N;
-  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= (long long)a.P * a.Q * CG) return;
-  const int cg = (int)(idx % CG);
-  const long long pix = idx / CG;
-  const int q = (int)(pix % a.Q), p = (int)(pix / a.Q);
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= a.P * a.Q * CG) return;
+  const int cg = idx % CG;
+  const int pix = idx / CG;
+  const int q = pix % a.Q, p = pix / a.Q;
   const int c = cg * N;
   const int h0 = p * a.sh - a.ph, w0 = q * a.sw - a.pw;
   float acc[N], v[N];
@@ -86,8 +86,8 @@ __global__ void pool_kernel(const PoolArgs<T> a) {
 #pragma unroll
     for (int j = 0; j < N; ++j) acc[j] *= inv;
   }
-  store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
-  if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+  store_vec(a.out + (size_t)pix * a.ldo + c, c, a.C, acc);
+  if (a.out2) store_vec(a.out2 + (size_t)pix * a.ldo2 + c, c, a.C, acc);
 }
 
 template <typename T>
@@ -102,11 +102,11 @@ template <typename T>
 __global__ void dw_kernel(const DwArgs<T> a) {
   constexpr int N = Vec<T>::N;
   const int CG = (a.C + N - 1) / N;
-  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= (long long)a.P * a.Q * CG) return;
-  const int cg = (int)(idx % CG);
-  const long long pix = idx / CG;
-  const int q = (int)(pix % a.Q), p = (int)(pix / a.Q);
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= a.P * a.Q * CG) return;
+  const int cg = idx % CG;
+  const int pix = idx / CG;
+  const int q = pix % a.Q, p = pix / a.Q;
   const int c = cg * N;
   float acc[N], v[N], u[N];
 #pragma unroll
@@ -133,7 +133,7 @@ __global__ void dw_kernel(const DwArgs<T> a) {
       }
     }
   }
-  store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
+  store_vec(a.out + (size_t)pix * a.ldo + c, c, a.C, acc);
 }
 
 template <typename T>
@@ -148,10 +148,10 @@ template <typename T>
 __global__ void add_kernel(const AddArgs<T> a) {
   constexpr int N = Vec<T>::N;
   const int CG = (a.C + N - 1) / N;
-  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= (long long)a.HW * CG) return;
-  const int c = (int)(idx % CG) * N;
-  const long long pix = idx / CG;
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= a.HW * CG) return;
+  const int c = (idx % CG) * N;
+  const size_t pix = idx / CG;
   float acc[N], v[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) acc[j] = 0.f;
@@ -180,10 +180,10 @@ template <typename T>
 __global__ void copy_kernel(const CopyArgs<T> a) {
   constexpr int N = Vec<T>::N;
   const int CG = (a.C + N - 1) / N;
-  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= (long long)a.HW * CG) return;
-  const int c = (int)(idx % CG) * N;
-  const long long pix = idx / CG;
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= a.HW * CG) return;
+  const int c = (idx % CG) * N;
+  const size_t pix = idx / CG;
   const T* src = a.x + pix * a.ldx + c;
   T* dst = a.out + pix * a.ldo + c;
   // concat slices at channel offsets that are not multiples of 8 are not
@@ -271,10 +271,15 @@ void launch_linear(const T* x, int Cin, const T* w, int ldw, const float* b, int
 // ------------------------------------------------- layout conversion
 template <typename T>
 __global__ void input_kernel(const float* nchw, int C, int HW, T* out, int ldo) {
-  const long long pix = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  constexpr int N = Vec<T>::N;
+  const int pix = blockIdx.x * blockDim.x + threadIdx.x;
   if (pix >= HW) return;
-  for (int c = 0; c < ldo; ++c)
-    out[pix * ldo + c] = from_f<T>(c < C ? nchw[(size_t)c * HW + pix] : 0.f);
+  for (int c0 = 0; c0 < ldo; c0 += N) {
+    float v[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) v[j] = (c0 + j < C) ? __ldg(nchw + (size_t)(c0 + j) * HW + pix) : 0.f;
+    store_vec(out + (size_t)pix * ldo + c0, c0, ldo, v);
+  }
 }
 template <typename T>
 void launch_input(const float* nchw, int C, int H, int W, T* out, int ldo, cudaStream_t st) {

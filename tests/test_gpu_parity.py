@@ -74,6 +74,12 @@ CONV_CASES = [
     (192, 320, 9, 9, 3, 3, 2, 0, 0),
     (512, 1000, 13, 13, 1, 1, 1, 0, 0),   # classifier-like, K tail over 256 tiles
     (48, 64, 35, 35, 5, 5, 1, 2, 2),
+    # halo mode (stride 1, output width >= 96): shifted-window A descriptors
+    (32, 64, 37, 130, 3, 3, 1, 1, 1),
+    (48, 64, 21, 125, 5, 5, 1, 2, 2),
+    (80, 192, 9, 252, 3, 3, 1, 0, 0),
+    (96, 96, 7, 300, 1, 7, 1, 0, 3),
+    (64, 80, 13, 100, 7, 1, 1, 3, 0),
 ]
 
 
