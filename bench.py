@@ -215,6 +215,59 @@ def _blas_threads():
     return len(os.sched_getaffinity(0))
 
 
+# ------------------------------------------------------------ N > 1 plumbing
+def owners(M, world):
+    """Logical GPU i of the schedule is executed by rank i % world (one
+    process per GPU; HIOS-LP may leave some GPUs idle, P:82 'm <= M')."""
+    return [i % world for i in range(M)]
+
+
+def share_schedule(h, dist, G, g, S, M, window, rank):
+    """Rank 0 profiled and scheduled; every other rank receives t(v), t(u,v)
+    and Q (per-op GPU + stage) and imports the identical schedule."""
+    if rank == 0:
+        opc, edc = h.hios_get_costs(G)
+        og, ost, _ = h.hios_schedule_stages(S)
+        obj = [opc.tolist(), edc.tolist(), og.tolist(), ost.tolist()]
+    else:
+        obj = [None, None, None, None]
+    dist.broadcast_object_list(obj, src=0)
+    opc, edc, og, ost = obj
+    if rank != 0:
+        for v in range(g.n_ops):
+            h.hios_set_op_cost(G, v, int(opc[v]))
+        for e in range(g.n_edges):
+            h.hios_set_edge_cost(G, e, int(edc[e]))
+        h.hios_set_group_model(G, 7, 10)  # t(S) of the imported groups (prediction only)
+        S = h.hios_schedule_import(G, M, window, og, ost)
+    return S
+
+
+def bind_and_exchange(h, dist, S, M, world, rank, dev):
+    """Each rank owns its logical GPUs; device buffers and flag words are
+    exported as CUDA IPC handles and mapped by every other rank, so producers
+    store straight into consumer buffers (peer memory over NVLink)."""
+    own = owners(M, world)
+    h.hios_schedule_place(S, [dev] * M)
+    h.hios_schedule_bind_rank(S, own, rank)
+    blob = h.hios_ipc_export(S)
+    blobs = [None] * world
+    dist.all_gather_object(blobs, blob)
+    for r in range(world):
+        if r != rank:
+            h.hios_ipc_import(S, r, blobs[r])
+    return own
+
+
+def max_over_ranks(dist, x, world):
+    if world <= 1:
+        return x
+    import torch
+    t = torch.tensor([float(x)], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 # ------------------------------------------------------------ main
 def main():
     ap = argparse.ArgumentParser()
@@ -269,10 +322,13 @@ def main():
     import torch.distributed as dist
     from paper_conf_cluster_kundus23_b200 import hios as h
 
+    ndev_vis = torch.cuda.device_count()
+    dev = local_rank % ndev_vis
+    torch.cuda.set_device(dev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
-    torch.cuda.set_device(local_rank)
-    dev = local_rank
+        # host-side plumbing only (costs, schedule, IPC handles, barriers,
+        # max-over-ranks timing): activations never go through a collective
+        dist.init_process_group(os.environ.get("HIOS_DIST_BACKEND", "gloo"))
     esz = 2 if args.dtype == "bf16" else 4
     pk = peaks()
     M = args.gpus if world > 1 else max(args.gpus, args.logical or 1)
@@ -282,36 +338,14 @@ def main():
     shapes = {o.id: h.hios_graph_shape(G, o.id) for o in g.ops}
     t0 = time.perf_counter()
     if rank == 0:
-        ndev = torch.cuda.device_count()
-        h.hios_profile(G, [dev] + ([1] if ndev > 1 and dev != 1 else []), 10)
+        h.hios_profile(G, [dev] + ([(dev + 1) % ndev_vis] if ndev_vis > 1 else []), 10)
     t_prof = time.perf_counter() - t0
     t0 = time.perf_counter()
-    sched = {}
-    if rank == 0:
-        S = h.hios_schedule_lp(G, M, args.window)
-        sched["main"] = h.hios_schedule_stages(S)
+    S = h.hios_schedule_lp(G, M, args.window) if rank == 0 else None
     t_sched = time.perf_counter() - t0
     if world > 1:
-        opc, edc = h.hios_get_costs(G) if rank == 0 else (None, None)
-        obj = [opc, edc, sched.get("main")]
-        dist.broadcast_object_list(obj, src=0)
-        opc, edc, main = obj
-        if rank != 0:
-            for v in range(g.n_ops):
-                h.hios_set_op_cost(G, v, int(opc[v]))
-            for e in range(g.n_edges):
-                h.hios_set_edge_cost(G, e, int(edc[e]))
-            h.hios_set_group_model(G, 7, 10)
-            S = h.hios_schedule_import(G, M, args.window, main[0], main[1])
-        owner = [i % world for i in range(M)]
-        h.hios_schedule_place(S, [dev if owner[i] == rank else 0 for i in range(M)])
-        h.hios_schedule_bind_rank(S, owner, rank)
-        blob = h.hios_ipc_export(S)
-        blobs = [None] * world
-        dist.all_gather_object(blobs, blob)
-        for r in range(world):
-            if r != rank:
-                h.hios_ipc_import(S, r, blobs[r])
+        S = share_schedule(h, dist, G, g, S, M, args.window, rank)
+        bind_and_exchange(h, dist, S, M, world, rank, dev)
     elif M > 1:
         ndev = torch.cuda.device_count()
         h.hios_schedule_place(S, [i % ndev for i in range(M)])
@@ -358,11 +392,7 @@ def main():
         torch.cuda.profiler.stop()
     wall = time.perf_counter() - wall0
     clocks = clk.stop()
-    total = float(np.sum(times))
-    if world > 1:
-        t = torch.tensor([total], device=f"cuda:{dev}")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total = float(t.item())
+    total = max_over_ranks(dist, float(np.sum(times)), world)
     ms = total / args.steps
 
     # ---------------- end-to-end through hios_run (pinned host buffers)
@@ -374,11 +404,7 @@ def main():
         t0 = time.perf_counter()
         y = h.hios_run(S, xin if (world == 1 or int(op_gpu[0]) % world == rank or True) else None)
         e2e.append((time.perf_counter() - t0) * 1e3)
-    e2e_ms = float(np.mean(e2e[args.warmup:]))
-    if world > 1:
-        t = torch.tensor([e2e_ms], device=f"cuda:{dev}")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_ms = float(t.item())
+    e2e_ms = max_over_ranks(dist, float(np.mean(e2e[args.warmup:])), world)
 
     # ---------------- per-op device times (instrumented graph) for the roofline
     op_ns_acc = np.zeros(g.n_ops)
