@@ -3,11 +3,13 @@
 //
 // GEMM view: M = output pixels, N = output channels, K = R*S*C.  bf16
 // operands, fp32 accumulation in TMEM, folded-BN scale/shift + ReLU + bf16
-// epilogue.  Persistent, warp-specialised CTA (192 threads):
-//   warp 0      TMA producer (one elected lane)
-//   warp 1      MMA issuer (one elected lane): 4 x tcgen05.mma.kind::f16
-//               (M=128, N=n_tile, K=16) per K-step
-//   warps 2-5   epilogue: tcgen05.ld -> scale/shift/ReLU -> bf16 -> stores
+// epilogue.  Persistent, warp-specialised CTA (384 threads):
+//   warps 0-3   TMA producers (one lane each, K-steps round-robin)
+//   warps 4-7   MMA issuers (one lane each, one N sub-tile each): 4 x
+//               tcgen05.mma.kind::f16 (M=128, N=n_tile/n_mma, K=16) per K-step;
+//               warp 4 allocates TMEM
+//   warps 8-11  epilogue: tcgen05.ld -> scale/shift/ReLU -> bf16 -> smem
+//               staging -> coalesced stores
 //               to the local buffer / concat slice and, optionally, a peer
 //               GPU's replica (cross-GPU edge fused into the epilogue)
 // Two TMEM accumulators (2 x n_tile columns) let the epilogue of tile i run
@@ -51,6 +53,34 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       "HIOS_WAIT_%=:\n"
       "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
       "@!p bra HIOS_WAIT_%=;\n"
+      "}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void sts128(uint32_t addr, uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3) {
+  asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a0), "r"(a1), "r"(a2), "r"(a3)
+               : "memory");
+}
+__device__ __forceinline__ uint4 lds128(uint32_t addr) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr)
+               : "memory");
+  return v;
+}
+__device__ __forceinline__ uint16_t lds16(uint32_t addr) {
+  uint16_t v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(addr) : "memory");
+  return v;
+}
+
+// non-blocking probe loop (no HW suspend between probes)
+__device__ __forceinline__ void mbar_spin(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "HIOS_SPIN_%=:\n"
+      "mbarrier.test_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra HIOS_SPIN_%=;\n"
       "}\n" ::"r"(bar),
       "r"(parity)
       : "memory");
@@ -109,6 +139,7 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
 // optional timeline instrumentation (HIOS_TRACE): globaltimer at checkpoints
 __device__ unsigned long long g_conv_trace[256 * 8];
 __device__ unsigned long long g_conv_trace2[32 * 48];  // per CTA: issue[16], full[16], empty_ok[16]
+__device__ unsigned long long g_conv_trace3[32 * 8];   // per CTA: epilogue checkpoints
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
@@ -117,6 +148,10 @@ __device__ __forceinline__ unsigned long long gtimer() {
 #define TRACE2(slot, k)                                                   \
   do {                                                                    \
     if (a.trace && blockIdx.x < 32 && (k) < 16) g_conv_trace2[blockIdx.x * 48 + (slot) * 16 + (k)] = gtimer(); \
+  } while (0)
+#define TRACE3(k)                                                         \
+  do {                                                                    \
+    if (a.trace && blockIdx.x < 32) g_conv_trace3[blockIdx.x * 8 + (k)] = gtimer(); \
   } while (0)
 #define TRACE(k)                                                          \
   do {                                                                    \
@@ -130,7 +165,15 @@ static __host__ __device__ inline uint32_t tmem_cols(int n) {
 }
 
 
-__global__ void __launch_bounds__(192, 1)
+constexpr int kProducers = 4;  // TMA issuing warps
+constexpr int kMma = 4;        // MMA issuing warps (one N sub-tile each)
+constexpr int kEpi = 4;        // epilogue warps (one TMEM lane quarter each)
+constexpr int kThreads = 32 * (kProducers + kMma + kEpi);
+constexpr int kEpiWarp0 = kProducers + kMma;
+
+__host__ __device__ inline uint32_t stage_pitch(int n_tile) { return (uint32_t)n_tile * 2u + 16u; }
+
+__global__ void __launch_bounds__(kThreads, 1)
     conv_tc_kernel(const __grid_constant__ CUtensorMap mx, const __grid_constant__ CUtensorMap mw,
                    const ConvTcArgs a) {
   extern __shared__ uint8_t smem_raw[];
@@ -139,9 +182,11 @@ __global__ void __launch_bounds__(192, 1)
   const uint32_t A_BYTES = 128 * 128;
   const uint32_t B_BYTES = (uint32_t)a.n_tile * 128;
   const uint32_t H_BYTES = a.halo ? halo_bytes_of(a.R, a.halo_w) : 0u;
+  const uint32_t PITCH = stage_pitch(a.n_tile);
   uint8_t* sA = smem;  // halo: a_bufs x H_BYTES ; tap: ST x A_BYTES
   uint8_t* sB = smem + (a.halo ? a.a_bufs * H_BYTES : ST * A_BYTES);
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sB + ST * B_BYTES);
+  uint8_t* sOut = sB + ST * B_BYTES;  // epilogue staging [128][PITCH]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sOut + 128 * PITCH);
   // barriers: full[ST] empty[ST] afull[2] aempty[2] tfull[2] tempty[2]
   const uint32_t full0 = smem_u32(bars), empty0 = full0 + 8 * ST;
   const uint32_t afull0 = empty0 + 8 * ST, aempty0 = afull0 + 16, tfull0 = aempty0 + 16, tempty0 = tfull0 + 16;
@@ -153,24 +198,26 @@ __global__ void __launch_bounds__(192, 1)
   const uint32_t ncols = tmem_cols(2 * a.n_tile);
   const int RS = a.R * a.S;
   const int tiles = a.tiles_m * a.tiles_n;
+  const int nmma = a.n_mma;  // active MMA warps; N sub-tile = n_tile / nmma
+  const int n_sub = a.n_tile / nmma;
   if (threadIdx.x == 0) TRACE(0);
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < ST; ++i) {
       mbar_init(full0 + 8 * i, 1);
-      mbar_init(empty0 + 8 * i, 1);
+      mbar_init(empty0 + 8 * i, nmma);
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(afull0 + 8 * i, 1);
-      mbar_init(aempty0 + 8 * i, 1);
-      mbar_init(tfull0 + 8 * i, 1);
-      mbar_init(tempty0 + 8 * i, 128);
+      mbar_init(aempty0 + 8 * i, nmma);
+      mbar_init(tfull0 + 8 * i, nmma);
+      mbar_init(tempty0 + 8 * i, 32 * kEpi);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mx)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mw)) : "memory");
   }
-  if (warp == 1) {
+  if (warp == kProducers) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                  "r"(ncols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -181,12 +228,20 @@ __global__ void __launch_bounds__(192, 1)
   const uint32_t tmem = *tmem_slot;
   if (threadIdx.x == 0) TRACE(1);
 
-  if (warp == 0) {
-    if (lane == 0) {
-      // ------------------------------------------------------ TMA producer
-      // (single thread: every division is hoisted out of the K loop; stage,
-      //  phase, tap and chunk advance incrementally)
+  // Each stage is owned by one producer warp (st = w mod n_prod, n_prod | ST),
+  // so a stage's empty barrier is never waited on two phases ahead (parity
+  // waits cannot tell phase u from u-2).
+  const int n_prod = (ST % 4 == 0) ? 4 : ((ST % 2 == 0) ? 2 : 1);
+  if (warp < kProducers) {
+    if (lane == 0 && (warp < n_prod || (a.halo && warp == 0))) {
+      // ------------------------------------------------------ TMA producers
+      // A cp.async.bulk.tensor keeps its issuing thread busy for hundreds of
+      // cycles (measured, tools/tma_bench.cu), so kProducers warps issue in
+      // parallel: warp w owns the K-steps ks = w (mod kProducers); warp 0
+      // also loads the halo boxes.  Every division is hoisted out of the K
+      // loop; stage, phase, tap and chunk advance incrementally.
       uint32_t st = 0, ph = 0, ab = 0, aph = 0, ks = 0;
+      int mine = warp < n_prod ? warp : 1 << 30;
       const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
       for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
         const int m_blk = tile / a.tiles_n, n_blk = tile - m_blk * a.tiles_n;
@@ -195,25 +250,31 @@ __global__ void __launch_bounds__(192, 1)
         const int x0 = q0 * a.sw - a.pw, y0 = p0 * a.sh - a.ph;
         for (int cc = 0; cc < a.c_chunks; ++cc) {
           const int c0 = cc * 64;
-          if (a.halo) {
+          if (a.halo && warp == 0) {
             mbar_wait(aempty0 + 8 * ab, aph ^ 1u);
             mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.R * a.halo_w * 128u);
             tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, c0, x0, y0);
+          }
+          if (a.halo) {
             if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
           }
           int r = 0, s = 0;
           for (int rs = 0; rs < RS; ++rs, ++ks) {
-            mbar_wait(empty0 + 8 * st, ph ^ 1u);
-            TRACE2(2, ks);
-            if (a.halo) {
-              mbar_expect_tx(full0 + 8 * st, B_BYTES);
-            } else {
-              mbar_expect_tx(full0 + 8 * st, A_BYTES + B_BYTES);
-              tma_load_3d(sA0 + st * A_BYTES, &mx, full0 + 8 * st, c0, x0 + s * a.dw, y0 + r * a.dh);
+            if (mine == 0) {
+              mbar_wait(empty0 + 8 * st, ph ^ 1u);
+              TRACE2(2, ks);
+              if (a.halo) {
+                mbar_expect_tx(full0 + 8 * st, B_BYTES);
+              } else {
+                mbar_expect_tx(full0 + 8 * st, A_BYTES + B_BYTES);
+                tma_load_3d(sA0 + st * A_BYTES, &mx, full0 + 8 * st, c0, x0 + s * a.dw, y0 + r * a.dh);
+              }
+              tma_load_3d(sB0 + st * B_BYTES, &mw, full0 + 8 * st, c0, rs, n0);
+              if (ks == 0) TRACE(2);
+              TRACE2(0, ks);
+              mine = n_prod;
             }
-            tma_load_3d(sB0 + st * B_BYTES, &mw, full0 + 8 * st, c0, rs, n0);
-            if (ks == 0) TRACE(2);
-            TRACE2(0, ks);
+            --mine;
             if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
             if (++s == a.S) { s = 0; ++r; }
           }
@@ -221,23 +282,25 @@ __global__ void __launch_bounds__(192, 1)
       }
     }
     __syncwarp();
-  } else if (warp == 1) {
-    if (lane == 0) {
-      // ------------------------------------------------------ MMA issuer
-      const uint32_t idesc = (1u << 4)                            // D f32
-                             | (1u << 7)                          // A bf16
-                             | (1u << 10)                         // B bf16
-                             | ((uint32_t)(a.n_tile >> 3) << 17)  // N
-                             | ((uint32_t)(128 >> 4) << 24);      // M = 128
+  } else if (warp < kProducers + kMma) {
+    const int j = warp - kProducers;  // N sub-tile of this MMA warp
+    if (lane == 0 && j < nmma) {
+      // ------------------------------------------------------ MMA issuers
+      // tcgen05.mma issue also occupies its thread for ~100 cycles, so the N
+      // tile is split across nmma warps (separate TMEM column ranges, same A)
+      const uint32_t idesc = (1u << 4)                          // D f32
+                             | (1u << 7)                        // A bf16
+                             | (1u << 10)                       // B bf16
+                             | ((uint32_t)(n_sub >> 3) << 17)   // N
+                             | ((uint32_t)(128 >> 4) << 24);    // M = 128
       uint32_t st = 0, ph = 0, ab = 0, aph = 0, ks = 0, acc = 0, tph = 0;
-      const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
-      // halo mode: A window of tap (r, s) starts (r * halo_w + s * dw) rows in
+      const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB) + (uint32_t)(j * n_sub) * 128u;
       const uint32_t row_r = (uint32_t)a.halo_w * 128u, row_s = (uint32_t)a.dw * 128u;
       int tcount = 0;
       for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
         mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
         tc_fence_after();
-        const uint32_t d = tmem + acc * (uint32_t)a.n_tile;
+        const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
         uint32_t accum = 0;
         for (int cc = 0; cc < a.c_chunks; ++cc) {
           const uint32_t abase = sA0 + ab * H_BYTES;
@@ -250,15 +313,14 @@ __global__ void __launch_bounds__(192, 1)
           for (int rs = 0; rs < RS; ++rs, ++ks) {
             mbar_wait(full0 + 8 * st, ph);
             tc_fence_after();
-            if (ks == 0) TRACE(3);
-            TRACE2(1, ks);
+            if (ks == 0 && j == 0) TRACE(3);
+            if (j == 0) TRACE2(1, ks);
             const uint32_t a_addr = a.halo ? abase + aoff : sA0 + st * A_BYTES;
             const uint64_t ad = umma_desc_sw128(a_addr, a.bo_mode);
             const uint64_t bd = umma_desc_sw128(sB0 + st * B_BYTES);
 #pragma unroll
-            for (int k = 0; k < 4; ++k) {  // 4 x K=16 inside the 128-byte swizzle row
+            for (int k = 0; k < 4; ++k)  // 4 x K=16 inside the 128-byte swizzle row
               mma_bf16(d, ad + 2 * k, bd + 2 * k, idesc, accum | (uint32_t)k);
-            }
             accum = 1;
             mma_commit(empty0 + 8 * st);
             if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
@@ -270,7 +332,7 @@ __global__ void __launch_bounds__(192, 1)
           }
         }
         mma_commit(tfull0 + 8 * acc);
-        if (tcount == 0) TRACE(4);
+        if (tcount == 0 && j == 0) TRACE(4);
         acc ^= 1u;
         if (acc == 0) tph ^= 1u;
       }
@@ -278,77 +340,107 @@ __global__ void __launch_bounds__(192, 1)
     __syncwarp();
   } else {
     // -------------------------------------------------------- epilogue
+    // TMEM -> registers -> folded BN + ReLU -> bf16 -> smem staging tile;
+    // the accumulator is released to the MMA warps as soon as it is read,
+    // then the tile leaves smem in coalesced 16-byte row segments (to the
+    // local destination and, fused, to the peer GPU's replica).
+    const int ew = warp - kEpiWarp0;
     const int lw = warp & 3;  // TMEM lane quarter this warp may access
     const int m = lw * 32 + lane;
+    const int et = threadIdx.x - 32 * kEpiWarp0;  // 0..127
     uint32_t tcount = 0, acc = 0, tph = 0;
-    const int hh = m / a.tw, ww = m - hh * a.tw;
     for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
       const int m_blk = tile / a.tiles_n, n_blk = tile - m_blk * a.tiles_n;
       const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
       const int p0 = tp * a.th, q0 = tq * a.tw, n0 = n_blk * a.n_tile;
-      // stage this tile's folded-BN scale/shift in smem (overlaps the main loop)
+      const int n_valid = min(a.n_tile, a.K - n0);
+      // previous tile fully copied out of sOut / s_scale (all 128 threads)
       asm volatile("bar.sync 1, 128;" ::: "memory");
-      for (int j = threadIdx.x - 64; j < a.n_tile; j += 128) {
-        const int nj = min(n0 + j, a.K - 1);
-        s_scale[j] = __ldg(a.scale + nj);
-        s_shift[j] = __ldg(a.shift + nj);
+      for (int jj = et; jj < a.n_tile; jj += 128) {
+        const int nj = min(n0 + jj, a.K - 1);
+        s_scale[jj] = __ldg(a.scale + nj);
+        s_shift[jj] = __ldg(a.shift + nj);
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
       mbar_wait(tfull0 + 8 * acc, tph);
       __syncwarp();
       tc_fence_after();
-      if (tcount == 0 && warp == 2 && lane == 0) TRACE(5);
-      const int p = p0 + hh, q = q0 + ww;
-      const bool valid = p < a.P && q < a.Q;
-      const size_t pix = (size_t)p * a.Q + q;
+      if (tcount == 0 && warp == kEpiWarp0 && lane == 0) TRACE(5);
       const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)a.n_tile;
+      const uint32_t srow = smem_u32(sOut) + (uint32_t)m * PITCH;
       for (int col = 0; col < a.n_tile; col += 16) {
         uint32_t r[16];
         tmem_ld16(tbase + (uint32_t)col, r);
-        const int n = n0 + col;
-        if (!valid || n >= a.K) continue;
-        float v[16];
+        uint32_t pk[8];
 #pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          float y = __uint_as_float(r[j]) * s_scale[col + j] + s_shift[col + j];
-          v[j] = a.relu ? fmaxf(y, 0.f) : y;
+        for (int q = 0; q < 8; ++q) {
+          float y0 = __uint_as_float(r[2 * q]) * s_scale[col + 2 * q] + s_shift[col + 2 * q];
+          float y1 = __uint_as_float(r[2 * q + 1]) * s_scale[col + 2 * q + 1] + s_shift[col + 2 * q + 1];
+          if (a.relu) { y0 = fmaxf(y0, 0.f); y1 = fmaxf(y1, 0.f); }
+          __nv_bfloat162 b2 = __floats2bfloat162_rn(y0, y1);
+          pk[q] = *reinterpret_cast<uint32_t*>(&b2);
         }
-        if (n + 16 <= a.K) {
-          uint32_t pk[8];
-#pragma unroll
-          for (int j = 0; j < 8; ++j) {
-            __nv_bfloat162 b2 = __floats2bfloat162_rn(v[2 * j], v[2 * j + 1]);
-            pk[j] = *reinterpret_cast<uint32_t*>(&b2);
-          }
-          uint4* dst = reinterpret_cast<uint4*>(a.out + pix * a.ldo + n);
-          dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-          dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
-          if (a.out2) {
-            uint4* d2 = reinterpret_cast<uint4*>(a.out2 + pix * a.ldo2 + n);
-            d2[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-            d2[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
-          }
-        } else {
-#pragma unroll
-          for (int j = 0; j < 16; ++j) {
-            if (n + j < a.K) {
-              a.out[pix * a.ldo + n + j] = __float2bfloat16_rn(v[j]);
-              if (a.out2) a.out2[pix * a.ldo2 + n + j] = __float2bfloat16_rn(v[j]);
-            }
-          }
-        }
+        sts128(srow + col * 2, pk[0], pk[1], pk[2], pk[3]);
+        sts128(srow + col * 2 + 16, pk[4], pk[5], pk[6], pk[7]);
       }
       tc_fence_before();
-      mbar_arrive(tempty0 + 8 * acc);
-      if (tcount == 0 && warp == 2 && lane == 0) TRACE(6);
+      mbar_arrive(tempty0 + 8 * acc);  // TMEM accumulator free for the next tile
+      if (tcount == 0 && warp == kEpiWarp0 && lane == 0) TRACE(6);
       acc ^= 1u;
       if (acc == 0) tph ^= 1u;
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (tcount == 0 && et == 0) TRACE3(0);
+      // coalesced copy-out: the 128 epilogue threads walk (row, 16-byte
+      // chunk) pairs row-major, so consecutive lanes store consecutive 16 B of
+      // one output pixel row (loads issued ahead of the dependent stores)
+      const int row_bytes = n_valid * 2;
+      const int chunks = row_bytes >> 4;
+      const uint32_t sbase = smem_u32(sOut);
+      const int total = 128 * chunks;
+      for (int i0 = et; i0 < total; i0 += 128 * 4) {
+        uint4 v[4];
+        int rr[4], cc4[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int i = i0 + u * 128;
+          rr[u] = i / chunks;
+          cc4[u] = i - rr[u] * chunks;
+          if (i < total) v[u] = lds128(sbase + (uint32_t)rr[u] * PITCH + (uint32_t)cc4[u] * 16u);
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int i = i0 + u * 128;
+          if (i >= total) break;
+          const int hh = rr[u] / a.tw, ww = rr[u] - hh * a.tw;
+          const int p = p0 + hh, q = q0 + ww;
+          if (p >= a.P || q >= a.Q) continue;
+          const size_t pix = (size_t)p * a.Q + q;
+          *reinterpret_cast<uint4*>(a.out + pix * a.ldo + n0 + cc4[u] * 8) = v[u];
+          if (a.out2) *reinterpret_cast<uint4*>(a.out2 + pix * a.ldo2 + n0 + cc4[u] * 8) = v[u];
+        }
+      }
+      if (n_valid & 7) {  // channel tail (K % 8 != 0): element copies
+        const int tail0 = chunks * 8, nt = n_valid - tail0;
+        for (int i = et; i < 128 * nt; i += 128) {
+          const int rr1 = i / nt, e = tail0 + (i - rr1 * nt);
+          const int hh = rr1 / a.tw, ww = rr1 - hh * a.tw;
+          const int p = p0 + hh, q = q0 + ww;
+          if (p >= a.P || q >= a.Q) continue;
+          const size_t pix = (size_t)p * a.Q + q;
+          const uint16_t v = lds16(sbase + (uint32_t)rr1 * PITCH + (uint32_t)e * 2u);
+          reinterpret_cast<uint16_t*>(a.out + pix * a.ldo + n0)[e] = v;
+          if (a.out2) reinterpret_cast<uint16_t*>(a.out2 + pix * a.ldo2 + n0)[e] = v;
+        }
+      }
+      if (tcount == 0 && et == 0) TRACE3(1);
     }
+    if (et == 0) TRACE3(2);
   }
+  if (lane == 0 && warp < 8) TRACE3(3 + (warp >> 1));
   tc_fence_before();
   __syncthreads();
   if (threadIdx.x == 0) TRACE(7);
-  if (warp == 1) {
+  if (warp == kProducers) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(ncols));
   }
@@ -357,7 +449,8 @@ __global__ void __launch_bounds__(192, 1)
 size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
   const size_t B = (size_t)a.n_tile * 128;
   const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.R, a.halo_w) : (size_t)a.stages * 128 * 128;
-  return 1024 + A + (size_t)a.stages * B + (2 * a.stages + 10) * 8 + 2 * 256 * 4;
+  return 1024 + A + (size_t)a.stages * B + 128 * (size_t)stage_pitch(a.n_tile) + (2 * a.stages + 10) * 8 +
+         2 * 256 * 4;
 }
 
 void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcArgs& a, int grid, size_t smem,
@@ -369,7 +462,7 @@ void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcAr
     cudaFuncSetAttribute(conv_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr_set[dev] = true;
   }
-  conv_tc_kernel<<<grid, 192, smem, st>>>(mx, mw, a);
+  conv_tc_kernel<<<grid, kThreads, smem, st>>>(mx, mw, a);
 }
 
 }  // namespace hios
@@ -377,6 +470,10 @@ void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcAr
 extern "C" int hios_debug_conv_trace_reset(void) {
   static unsigned long long zero[2048];
   return (int)cudaMemcpyToSymbol(hios::g_conv_trace, zero, sizeof(zero));
+}
+
+extern "C" int hios_debug_conv_trace3(unsigned long long* out) {
+  return (int)cudaMemcpyFromSymbol(out, hios::g_conv_trace3, sizeof(unsigned long long) * 32 * 8);
 }
 
 extern "C" int hios_debug_conv_trace2(unsigned long long* out) {

@@ -303,32 +303,51 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   c.tiles_m = ((P + c.th - 1) / c.th) * c.tiles_q;
   c.c_chunks = (C + 63) / 64;
   const int KI = R * S * c.c_chunks;
-  const double a_bytes = c.halo ? (double)R * hw * 128.0 / (R * S) : 16384.0;
+  // cost model (cycles), from the measured issue costs on B200
+  // (tools/mma_bench.cu, tools/tma_bench.cu): ~100 cycles per tcgen05.mma and
+  // ~500 per TMA instruction per issuing thread; MMA M=128 x N x K=16 takes
+  // N/2 cycles; ~64 B/cycle/SM of TMA bandwidth.
+  auto n_mma_of = [](int nt) { return nt % 64 == 0 ? 4 : (nt % 32 == 0 ? 2 : 1); };
   double best_cost = 1e300;
   for (int nt = 16; nt <= 256; nt += 16) {
     if (nt > rup(K, 16)) break;
     const int tn = (K + nt - 1) / nt;
+    const int nm = n_mma_of(nt);
+    const double mma = std::max(4.0 * nt / 2.0, 4.0 * 100.0 / nm);
+    const double a_bytes = c.halo ? (double)R * (128 + (S - 1) * dw) * 128.0 / (R * S) : 16384.0;
+    const double tma = std::max((c.halo ? 1.0 : 2.0) * 500.0 / 4.0, (a_bytes + nt * 128.0) / 64.0);
+    const double epi = nt / 16.0 * 80.0 + 128.0 * nt * 2.0 / 64.0;
+    const double tile = std::max(KI * std::max(mma, tma), epi) + 300.0;
     const double waves = std::ceil((double)c.tiles_m * tn / 148.0);
-    const double kstep = std::max(2.0 * nt, (a_bytes + nt * 128.0) / 128.0) + 40.0;
-    const double cost = waves * (KI * kstep + 600.0);
-    if (cost < best_cost * 0.999) { best_cost = cost; c.n_tile = nt; }
+    const double cost = waves * tile + 1500.0;
+    if (cost < best_cost * 0.98) { best_cost = cost; c.n_tile = nt; }
   }
   c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
-  const size_t B = (size_t)c.n_tile * 128;
-  const size_t budget = 200 * 1024;
-  if (c.halo) {
-    const size_t H = halo_bytes_of(R, hw);
-    c.a_bufs = (2 * H + 2 * B <= budget) ? 2 : 1;
-    c.stages = (int)std::min<size_t>(8, (budget - c.a_bufs * H) / B);
-  } else {
-    c.stages = (int)std::min<size_t>(6, budget / (16384 + B));
-  }
-  c.stages = std::max(2, std::min(c.stages, std::max(KI, 2)));
+  c.n_mma = n_mma_of(c.n_tile);
   // debug overrides for tuning experiments (tools/conv_micro.py)
   if (getenv("HIOS_NTILE")) {
     c.n_tile = std::min(256, rup(atoi(getenv("HIOS_NTILE")), 16));
     c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
+    c.n_mma = n_mma_of(c.n_tile);
   }
+  if (getenv("HIOS_NMMA")) {
+    const int want = atoi(getenv("HIOS_NMMA"));
+    c.n_mma = 1;
+    for (int m2 : {4, 2}) if (m2 <= want && c.n_tile % (16 * m2) == 0) { c.n_mma = m2; break; }
+  }
+  const size_t B = (size_t)c.n_tile * 128;
+  const size_t stage_out = 128 * ((size_t)c.n_tile * 2 + 16);
+  const size_t budget = 212 * 1024 - stage_out;
+  if (c.halo) {
+    const size_t H = halo_bytes_of(R, hw);
+    c.a_bufs = (2 * H + 2 * B <= budget) ? 2 : 1;
+    if (H + 2 * B > budget) c.halo = 0;  // does not fit: fall back to tap mode
+    else c.stages = (int)std::min<size_t>(8, (budget - c.a_bufs * H) / B);
+  }
+  if (!c.halo) {
+    c.stages = (int)std::min<size_t>(8, budget / (16384 + B));
+  }
+  c.stages = std::max(2, std::min(c.stages, std::max(KI, 2)));
   if (getenv("HIOS_STAGES")) c.stages = std::max(2, atoi(getenv("HIOS_STAGES")));
   return c;
 }
@@ -353,7 +372,7 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor&, const View& in, 
   ConvTcArgs a = plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw);
   if (getenv("HIOS_NOHALO") && a.halo) {  // debug: force tap mode on the same tiles
     a.halo = 0;
-    a.stages = std::max(2, std::min(a.stages, (int)((200 * 1024) / (16384 + a.n_tile * 128))));
+    a.stages = std::max(2, std::min(8, (int)((212 * 1024 - 128 * (a.n_tile * 2 + 16)) / (16384 + a.n_tile * 128))));
   }
   CUtensorMap mx, mw;
   bool ok;
@@ -371,6 +390,7 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor&, const View& in, 
   a.dh = dh; a.dw = dw; a.relu = relu; a.scale = scale; a.shift = shift;
   a.bo_mode = getenv("HIOS_BO") ? atoi(getenv("HIOS_BO")) : 0;
   a.trace = getenv("HIOS_TRACE") ? 1 : 0;
+  a.spin = getenv("HIOS_SPIN") ? atoi(getenv("HIOS_SPIN")) : 0;
   a.out = (bf16*)out.p; a.ldo = out.ldc;
   a.out2 = out2 ? (bf16*)out2->p : nullptr; a.ldo2 = out2 ? out2->ldc : 0;
   const size_t smem = conv_tc_smem_bytes(a);

@@ -27,6 +27,8 @@ struct ConvTcArgs {
   int halo, halo_w, a_bufs;  // halo mode: one R x halo_w input box per channel chunk
   int bo_mode;               // descriptor base-offset encoding (debug switch, 0)
   int trace;                 // write a globaltimer timeline (debug)
+  int spin;                  // unused (kept for ABI of the debug switches)
+  int n_mma;                 // MMA warps splitting the N tile (n_tile % (16 * n_mma) == 0)
   const float* scale;  // [K]
   const float* shift;  // [K]
   bf16* out;  int ldo; // primary output (channel offset applied)

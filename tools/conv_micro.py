@@ -26,7 +26,10 @@ SHAPES = [  # name, C, K, H, W, kh, kw, s, ph, pw
 
 def main():
     check = "--check" in sys.argv
+    only = [a for a in sys.argv[1:] if not a.startswith("--")]
     for (name, C, K, H, W, kh, kw, s, ph, pw) in SHAPES:
+        if only and name not in only:
+            continue
         g = graphs.GraphSpec("c", C, H, W)
         x0 = g.input()
         g.conv(x0, K, (kh, kw), s=s, p=(ph, pw), relu=1)

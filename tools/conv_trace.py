@@ -13,7 +13,10 @@ sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 from conv_micro import SHAPES  # noqa: E402
 
 lib = h.load()
+only = sys.argv[1:]
 for (name, C, K, H, W, kh, kw, s, ph, pw) in SHAPES:
+    if only and name not in only:
+        continue
     g = graphs.GraphSpec("c", C, H, W)
     x0 = g.input()
     g.conv(x0, K, (kh, kw), s=s, p=(ph, pw), relu=1)
@@ -40,6 +43,10 @@ for (name, C, K, H, W, kh, kw, s, ph, pw) in SHAPES:
     b2 = (ctypes.c_ulonglong * (32 * 48))()
     lib.hios_debug_conv_trace2(b2)
     t2 = (np.array(b2, dtype=np.int64).reshape(32, 3, 16)[0] - t0) / 1e3
+    b3 = (ctypes.c_ulonglong * (32 * 8))()
+    lib.hios_debug_conv_trace3(b3)
+    t3 = (np.array(b3, dtype=np.int64).reshape(32, 8)[0] - t0) / 1e3
+    print("   cta0 epi: staged-sync %.2f copied %.2f loop-done %.2f | warps0-1 %.2f 2-3 %.2f 4-5 %.2f 6-7 %.2f" % tuple(t3[:7]))
     print("   cta0 issue   ", " ".join(f"{v:6.2f}" for v in t2[0]))
     print("   cta0 full    ", " ".join(f"{v:6.2f}" for v in t2[1]))
     print("   cta0 emptyok ", " ".join(f"{v:6.2f}" for v in t2[2]))
