@@ -93,6 +93,19 @@ __device__ __forceinline__ void tma_load_3d(uint32_t dst, const CUtensorMap* map
       "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
       : "memory");
 }
+// one lane of a converged warp (the others skip the guarded issue but keep
+// running the warp-uniform loop, so operands stay in uniform registers)
+__device__ __forceinline__ bool elect_one() {
+  uint32_t pred = 0;
+  asm volatile(
+      "{\n"
+      ".reg .pred P;\n"
+      "elect.sync _|P, 0xffffffff;\n"
+      "selp.b32 %0, 1, 0, P;\n"
+      "}\n"
+      : "=r"(pred));
+  return pred != 0;
+}
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 
@@ -197,7 +210,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t ncols = tmem_cols(2 * a.n_tile);
   const int RS = a.R * a.S;
-  const int tiles = a.tiles_m * a.tiles_n;
+  const int tiles_mn = a.tiles_m * a.tiles_n;
+  const int tiles = tiles_mn * a.ksplit;  // split-K: each split owns a chunk range
   const int nmma = a.n_mma;  // active MMA warps; N sub-tile = n_tile / nmma
   const int n_sub = a.n_tile / nmma;
   if (threadIdx.x == 0) TRACE(0);
@@ -227,13 +241,18 @@ __global__ void __launch_bounds__(kThreads, 1)
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
   if (threadIdx.x == 0) TRACE(1);
+  // Programmatic dependent launch: the set-up above (barriers, TMEM,
+  // descriptor prefetch) overlapped the previous kernel's tail; inputs are
+  // read only after the predecessor grid has completed and flushed.
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  asm volatile("griddepcontrol.wait;" ::: "memory");
 
   // Each stage is owned by one producer warp (st = w mod n_prod, n_prod | ST),
   // so a stage's empty barrier is never waited on two phases ahead (parity
   // waits cannot tell phase u from u-2).
   const int n_prod = (ST % 4 == 0) ? 4 : ((ST % 2 == 0) ? 2 : 1);
   if (warp < kProducers) {
-    if (lane == 0 && (warp < n_prod || (a.halo && warp == 0))) {
+    if (warp < n_prod || (a.halo && warp == 0)) {
       // ------------------------------------------------------ TMA producers
       // A cp.async.bulk.tensor keeps its issuing thread busy for hundreds of
       // cycles (measured, tools/tma_bench.cu), so kProducers warps issue in
@@ -244,16 +263,21 @@ __global__ void __launch_bounds__(kThreads, 1)
       int mine = warp < n_prod ? warp : 1 << 30;
       const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
       for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
-        const int m_blk = tile / a.tiles_n, n_blk = tile - m_blk * a.tiles_n;
+        const int split = tile / tiles_mn, tmn = tile - split * tiles_mn;
+        const int m_blk = tmn / a.tiles_n, n_blk = tmn - m_blk * a.tiles_n;
         const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
         const int p0 = tp * a.th, q0 = tq * a.tw, n0 = n_blk * a.n_tile;
         const int x0 = q0 * a.sw - a.pw, y0 = p0 * a.sh - a.ph;
-        for (int cc = 0; cc < a.c_chunks; ++cc) {
+        const int cc_lo = split * a.cps, cc_hi = min(a.c_chunks, cc_lo + a.cps);
+        for (int cc = cc_lo; cc < cc_hi; ++cc) {
           const int c0 = cc * 64;
           if (a.halo && warp == 0) {
             mbar_wait(aempty0 + 8 * ab, aph ^ 1u);
-            mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.R * a.halo_w * 128u);
-            tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, c0, x0, y0);
+            if (elect_one()) {
+              mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.R * a.halo_w * 128u);
+              tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, c0, x0, y0);
+            }
+            __syncwarp();
           }
           if (a.halo) {
             if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
@@ -262,16 +286,21 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int rs = 0; rs < RS; ++rs, ++ks) {
             if (mine == 0) {
               mbar_wait(empty0 + 8 * st, ph ^ 1u);
-              TRACE2(2, ks);
-              if (a.halo) {
-                mbar_expect_tx(full0 + 8 * st, B_BYTES);
-              } else {
-                mbar_expect_tx(full0 + 8 * st, A_BYTES + B_BYTES);
-                tma_load_3d(sA0 + st * A_BYTES, &mx, full0 + 8 * st, c0, x0 + s * a.dw, y0 + r * a.dh);
+              if (elect_one()) {
+                TRACE2(2, ks);
+                if (a.dbg & 2) {  // debug: no operand traffic (timing experiments only)
+                  mbar_arrive(full0 + 8 * st);
+                } else if (a.halo) {
+                  mbar_expect_tx(full0 + 8 * st, B_BYTES);
+                } else {
+                  mbar_expect_tx(full0 + 8 * st, A_BYTES + B_BYTES);
+                  tma_load_3d(sA0 + st * A_BYTES, &mx, full0 + 8 * st, c0, x0 + s * a.dw, y0 + r * a.dh);
+                }
+                if (!(a.dbg & 2)) tma_load_3d(sB0 + st * B_BYTES, &mw, full0 + 8 * st, c0, rs, n0);
+                if (ks == 0) TRACE(2);
+                TRACE2(0, ks);
               }
-              tma_load_3d(sB0 + st * B_BYTES, &mw, full0 + 8 * st, c0, rs, n0);
-              if (ks == 0) TRACE(2);
-              TRACE2(0, ks);
+              __syncwarp();
               mine = n_prod;
             }
             --mine;
@@ -284,7 +313,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     __syncwarp();
   } else if (warp < kProducers + kMma) {
     const int j = warp - kProducers;  // N sub-tile of this MMA warp
-    if (lane == 0 && j < nmma) {
+    if (j < nmma) {
       // ------------------------------------------------------ MMA issuers
       // tcgen05.mma issue also occupies its thread for ~100 cycles, so the N
       // tile is split across nmma warps (separate TMEM column ranges, same A)
@@ -302,7 +331,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         tc_fence_after();
         const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
         uint32_t accum = 0;
-        for (int cc = 0; cc < a.c_chunks; ++cc) {
+        const int split = tile / tiles_mn;
+        const int cc_lo = split * a.cps, cc_hi = min(a.c_chunks, cc_lo + a.cps);
+        for (int cc = cc_lo; cc < cc_hi; ++cc) {
           const uint32_t abase = sA0 + ab * H_BYTES;
           if (a.halo) {
             mbar_wait(afull0 + 8 * ab, aph);
@@ -313,26 +344,33 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int rs = 0; rs < RS; ++rs, ++ks) {
             mbar_wait(full0 + 8 * st, ph);
             tc_fence_after();
-            if (ks == 0 && j == 0) TRACE(3);
-            if (j == 0) TRACE2(1, ks);
+            if (lane == 0 && ks == 0 && j == 0) TRACE(3);
+            if (lane == 0 && j == 0) TRACE2(1, ks);
             const uint32_t a_addr = a.halo ? abase + aoff : sA0 + st * A_BYTES;
             const uint64_t ad = umma_desc_sw128(a_addr, a.bo_mode);
             const uint64_t bd = umma_desc_sw128(sB0 + st * B_BYTES);
+            if (elect_one()) {
+              if (!(a.dbg & 1)) {  // (dbg & 1: skip the MMAs, timing experiments only)
 #pragma unroll
-            for (int k = 0; k < 4; ++k)  // 4 x K=16 inside the 128-byte swizzle row
-              mma_bf16(d, ad + 2 * k, bd + 2 * k, idesc, accum | (uint32_t)k);
+                for (int k = 0; k < 4; ++k)  // 4 x K=16 inside the 128-byte swizzle row
+                  mma_bf16(d, ad + 2 * k, bd + 2 * k, idesc, accum | (uint32_t)k);
+              }
+              mma_commit(empty0 + 8 * st);
+            }
+            __syncwarp();
             accum = 1;
-            mma_commit(empty0 + 8 * st);
             if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
             if (++s == a.S) { s = 0; aoff_r += row_r; aoff = aoff_r; } else { aoff += row_s; }
           }
           if (a.halo) {
-            mma_commit(aempty0 + 8 * ab);
+            if (elect_one()) mma_commit(aempty0 + 8 * ab);
+            __syncwarp();
             if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
           }
         }
-        mma_commit(tfull0 + 8 * acc);
-        if (tcount == 0 && j == 0) TRACE(4);
+        if (elect_one()) mma_commit(tfull0 + 8 * acc);
+        __syncwarp();
+        if (lane == 0 && tcount == 0 && j == 0) TRACE(4);
         acc ^= 1u;
         if (acc == 0) tph ^= 1u;
       }
@@ -350,10 +388,39 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int et = threadIdx.x - 32 * kEpiWarp0;  // 0..127
     uint32_t tcount = 0, acc = 0, tph = 0;
     for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
-      const int m_blk = tile / a.tiles_n, n_blk = tile - m_blk * a.tiles_n;
+      const int split = tile / tiles_mn, tmn = tile - split * tiles_mn;
+      const int m_blk = tmn / a.tiles_n, n_blk = tmn - m_blk * a.tiles_n;
       const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
       const int p0 = tp * a.th, q0 = tq * a.tw, n0 = n_blk * a.n_tile;
       const int n_valid = min(a.n_tile, a.K - n0);
+      if (a.ksplit > 1) {
+        // split-K: raw fp32 partial sums to the workspace (scale/shift/ReLU
+        // are applied by conv_splitk_finalize after all splits)
+        mbar_wait(tfull0 + 8 * acc, tph);
+        __syncwarp();
+        tc_fence_after();
+        const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)a.n_tile;
+        const int hh = m / a.tw, ww = m - hh * a.tw;
+        const int p = p0 + hh, q = q0 + ww;
+        const bool valid = p < a.P && q < a.Q;
+        float* wrow = a.ws + (size_t)split * a.ws_split + ((size_t)p * a.Q + q) * a.ws_ld + n0;
+        for (int col = 0; col < a.n_tile; col += 16) {
+          uint32_t r[16];
+          tmem_ld16(tbase + (uint32_t)col, r);
+          if (valid) {
+            uint4* d4 = reinterpret_cast<uint4*>(wrow + col);
+            d4[0] = make_uint4(r[0], r[1], r[2], r[3]);
+            d4[1] = make_uint4(r[4], r[5], r[6], r[7]);
+            d4[2] = make_uint4(r[8], r[9], r[10], r[11]);
+            d4[3] = make_uint4(r[12], r[13], r[14], r[15]);
+          }
+        }
+        tc_fence_before();
+        mbar_arrive(tempty0 + 8 * acc);
+        acc ^= 1u;
+        if (acc == 0) tph ^= 1u;
+        continue;
+      }
       // previous tile fully copied out of sOut / s_scale (all 128 threads)
       asm volatile("bar.sync 1, 128;" ::: "memory");
       for (int jj = et; jj < a.n_tile; jj += 128) {
@@ -446,6 +513,48 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
 }
 
+// sum the split-K partials, folded BN + ReLU, bf16, 16-byte stores
+__global__ void conv_splitk_finalize(const float* __restrict__ ws, int ksplit, size_t ws_split, int ws_ld, int PQ,
+                                     int K, const float* __restrict__ scale, const float* __restrict__ shift,
+                                     int relu, bf16* out, int ldo, bf16* out2, int ldo2) {
+  const int KG = (K + 7) / 8;
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= PQ * KG) return;
+  const int pix = idx / KG, n = (idx - pix * KG) * 8;
+  float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+  const float* src = ws + (size_t)pix * ws_ld + n;
+  for (int s = 0; s < ksplit; ++s) {
+    const float4 a0 = *reinterpret_cast<const float4*>(src + s * ws_split);
+    const float4 a1 = *reinterpret_cast<const float4*>(src + s * ws_split + 4);
+    acc[0] += a0.x; acc[1] += a0.y; acc[2] += a0.z; acc[3] += a0.w;
+    acc[4] += a1.x; acc[5] += a1.y; acc[6] += a1.z; acc[7] += a1.w;
+  }
+  __align__(16) bf16 v[8];
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const int nj = min(n + j, K - 1);
+    float y = acc[j] * __ldg(scale + nj) + __ldg(shift + nj);
+    v[j] = __float2bfloat16_rn(relu ? fmaxf(y, 0.f) : y);
+  }
+  bf16* d = out + (size_t)pix * ldo + n;
+  bf16* d2 = out2 ? out2 + (size_t)pix * ldo2 + n : nullptr;
+  if (n + 8 <= K) {
+    *reinterpret_cast<uint4*>(d) = *reinterpret_cast<const uint4*>(v);
+    if (d2) *reinterpret_cast<uint4*>(d2) = *reinterpret_cast<const uint4*>(v);
+  } else {
+    for (int j = 0; n + j < K; ++j) {
+      d[j] = v[j];
+      if (d2) d2[j] = v[j];
+    }
+  }
+}
+
+void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st) {
+  const int PQ = a.P * a.Q, KG = (a.K + 7) / 8;
+  conv_splitk_finalize<<<(PQ * KG + 255) / 256, 256, 0, st>>>(a.ws, a.ksplit, a.ws_split, a.ws_ld, PQ, a.K, a.scale,
+                                                                a.shift, a.relu, a.out, a.ldo, a.out2, a.ldo2);
+}
+
 size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
   const size_t B = (size_t)a.n_tile * 128;
   const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.R, a.halo_w) : (size_t)a.stages * 128 * 128;
@@ -462,7 +571,17 @@ void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcAr
     cudaFuncSetAttribute(conv_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr_set[dev] = true;
   }
-  conv_tc_kernel<<<grid, kThreads, smem, st>>>(mx, mw, a);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaLaunchKernelEx(&cfg, conv_tc_kernel, mx, mw, a);
 }
 
 }  // namespace hios

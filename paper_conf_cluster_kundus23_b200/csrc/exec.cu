@@ -322,8 +322,15 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     const double cost = waves * tile + 1500.0;
     if (cost < best_cost * 0.98) { best_cost = cost; c.n_tile = nt; }
   }
+  if (!c.halo) {
+    // tap mode: the per-K-step cost is dominated by a fixed ~0.3 us pipeline
+    // handshake (measured), so take the widest N tile (<= 256) that splits K
+    // evenly -- the most MMA work per K-step
+    const int nb = (K + 127) / 128;
+    c.n_tile = rup((K + nb - 1) / nb, 16);
+  }
   c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
-  c.n_mma = n_mma_of(c.n_tile);
+  c.n_mma = 1;  // measured: splitting N over several MMA warps does not pay (tools/conv_micro.py)
   // debug overrides for tuning experiments (tools/conv_micro.py)
   if (getenv("HIOS_NTILE")) {
     c.n_tile = std::min(256, rup(atoi(getenv("HIOS_NTILE")), 16));
@@ -337,7 +344,9 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   }
   const size_t B = (size_t)c.n_tile * 128;
   const size_t stage_out = 128 * ((size_t)c.n_tile * 2 + 16);
-  const size_t budget = 212 * 1024 - stage_out;
+  // occupancy: 1 CTA/SM (212 KB) or 2 CTAs/SM (104 KB each, TMEM <= 256 cols)
+  c.occ = (getenv("HIOS_OCC") ? atoi(getenv("HIOS_OCC")) : 1) == 2 && c.n_tile <= 128 ? 2 : 1;
+  const size_t budget = (c.occ == 2 ? 104 * 1024 : 212 * 1024) - stage_out;
   if (c.halo) {
     const size_t H = halo_bytes_of(R, hw);
     c.a_bufs = (2 * H + 2 * B <= budget) ? 2 : 1;
@@ -348,6 +357,19 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     c.stages = (int)std::min<size_t>(8, budget / (16384 + B));
   }
   c.stages = std::max(2, std::min(c.stages, std::max(KI, 2)));
+  // split-K (tap mode): a CTA's pipeline is latency-bound (~0.3 us per K-step,
+  // DESIGN.md §6), so deep layers with few output tiles split their
+  // 64-channel chunks across CTAs; fp32 partials are reduced by a finalize
+  // kernel that applies the folded BN + ReLU.
+  c.ksplit = 1;
+  c.cps = c.c_chunks;
+  const int tiles = c.tiles_m * c.tiles_n;
+  if (!c.halo && getenv("HIOS_SPLITK") && tiles < 100 && c.c_chunks >= 2 && R * S * c.c_chunks >= 8) {
+    int want = std::min(c.c_chunks, std::max(1, (148 * c.occ + tiles - 1) / tiles));
+    want = std::min(want, std::max(1, R * S * c.c_chunks / 4));  // keep >= ~4 K-steps per split
+    c.cps = (c.c_chunks + want - 1) / want;
+    c.ksplit = (c.c_chunks + c.cps - 1) / c.cps;
+  }
   if (getenv("HIOS_STAGES")) c.stages = std::max(2, atoi(getenv("HIOS_STAGES")));
   return c;
 }
@@ -365,7 +387,7 @@ static std::function<void(cudaStream_t)> conv_closure(Executor& ex, const View& 
                                                       int& nk);
 
 template <>
-std::function<void(cudaStream_t)> conv_closure<bf16>(Executor&, const View& in, int H, int W, int C, const void* w,
+std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& in, int H, int W, int C, const void* w,
                                                      float* scale, float* shift, int K, int R, int S, int sh, int sw,
                                                      int ph, int pw, int dh, int dw, int P, int Q, int relu,
                                                      const View& out, const View* out2, int& nk) {
@@ -391,10 +413,24 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor&, const View& in, 
   a.bo_mode = getenv("HIOS_BO") ? atoi(getenv("HIOS_BO")) : 0;
   a.trace = getenv("HIOS_TRACE") ? 1 : 0;
   a.spin = getenv("HIOS_SPIN") ? atoi(getenv("HIOS_SPIN")) : 0;
+  a.dbg = getenv("HIOS_DBG") ? atoi(getenv("HIOS_DBG")) : 0;
   a.out = (bf16*)out.p; a.ldo = out.ldc;
   a.out2 = out2 ? (bf16*)out2->p : nullptr; a.ldo2 = out2 ? out2->ldc : 0;
   const size_t smem = conv_tc_smem_bytes(a);
-  const int grid = std::min(a.tiles_m * a.tiles_n, 148);
+  const int grid = std::min(a.tiles_m * a.tiles_n * a.ksplit, 148 * a.occ);
+  if (a.ksplit > 1) {
+    a.ws_ld = a.tiles_n * a.n_tile;
+    a.ws_split = (size_t)P * Q * a.ws_ld;
+    void* ws = nullptr;
+    ck(cudaMalloc(&ws, a.ws_split * a.ksplit * sizeof(float)), "cudaMalloc split-K workspace");
+    ex.lg[ex.cur_lgpu].allocs.push_back(ws);
+    a.ws = (float*)ws;
+    nk += 2;
+    return [mx, mw, a, smem, grid](cudaStream_t st) {
+      launch_conv_tc(mx, mw, a, grid, smem, st);
+      launch_conv_splitk_finalize(a, st);
+    };
+  }
   nk += 1;
   return [mx, mw, a, smem, grid](cudaStream_t st) { launch_conv_tc(mx, mw, a, grid, smem, st); };
 }
@@ -562,6 +598,7 @@ void Executor::build_closures() {
     const int l = s.gpu_of[v];
     if (!lg[l].local) continue;
     ck(cudaSetDevice(lg[l].dev), "cudaSetDevice");
+    cur_lgpu = l;
     if (g.dtype == HIOS_BF16) build_op<bf16>(*this, v);
     else build_op<float>(*this, v);
   }

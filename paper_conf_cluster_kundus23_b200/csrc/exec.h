@@ -57,6 +57,7 @@ struct Executor {
   std::vector<OpExec> ox;
   std::vector<std::vector<int>> flag_index;  // [op][lgpu] flag slot on that lgpu (-1 none)
   int n_streams = 1;
+  int cur_lgpu = 0;  // logical GPU whose closures are being built
   bool lowered = false, captured = false;
   int64_t kernels_per_run = 0;
   // timed-graph events: per op (start, end) on its home lgpu

@@ -29,6 +29,12 @@ struct ConvTcArgs {
   int trace;                 // write a globaltimer timeline (debug)
   int spin;                  // unused (kept for ABI of the debug switches)
   int n_mma;                 // MMA warps splitting the N tile (n_tile % (16 * n_mma) == 0)
+  int occ;                   // co-resident CTAs per SM the smem plan allows (1 or 2)
+  int dbg;                   // debug switches (timing experiments; 0 in production)
+  int ksplit, cps;           // split-K: splits and 64-channel chunks per split
+  float* ws;                 // split-K fp32 workspace [ksplit][P*Q][ws_ld]
+  size_t ws_split;           // elements per split
+  int ws_ld;                 // row pitch (tiles_n * n_tile)
   const float* scale;  // [K]
   const float* shift;  // [K]
   bf16* out;  int ldo; // primary output (channel offset applied)
@@ -80,6 +86,7 @@ struct CopyArgs {
 void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcArgs& a, int grid, size_t smem,
                     cudaStream_t st);
 size_t conv_tc_smem_bytes(const ConvTcArgs& a);
+void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st);
 __host__ __device__ inline uint32_t halo_bytes_of(int R, int halo_w) {
   return ((uint32_t)R * halo_w * 128u + 1023u) & ~1023u;
 }

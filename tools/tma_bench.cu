@@ -16,7 +16,7 @@ typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
 __global__ void tma_kernel(const __grid_constant__ CUtensorMap m, int iters, int depth, uint32_t box_bytes,
-                           int n1, int n2, unsigned long long* cycles) {
+                           int n1, int n2, unsigned long long* cycles, int lanes_mode) {
   extern __shared__ uint8_t raw[];
   uint8_t* sm = (uint8_t*)(((uintptr_t)raw + 1023) & ~(uintptr_t)1023);
   uint64_t* bars = (uint64_t*)(sm + depth * box_bytes);
@@ -27,9 +27,11 @@ __global__ void tma_kernel(const __grid_constant__ CUtensorMap m, int iters, int
   }
   __syncthreads();
   // `issuers` warps (lane 0 each) share the ring: warp w handles slots w, w+issuers, ...
-  const int issuers = blockDim.x / 32;
-  if ((threadIdx.x & 31) != 0) return;
-  const int w = threadIdx.x >> 5;
+  // warps mode: lane 0 of each warp issues; lanes mode: lanes 0..k-1 of warp 0
+  const int issuers = lanes_mode ? lanes_mode : blockDim.x / 32;
+  int w;
+  if (lanes_mode) { if (threadIdx.x >= lanes_mode) return; w = threadIdx.x; }
+  else { if ((threadIdx.x & 31) != 0) return; w = threadIdx.x >> 5; }
   long long t0 = clock64();
   uint32_t ph = 0;
   for (int it = w; it < iters; it += issuers) {
@@ -78,15 +80,12 @@ int main() {
   cudaMalloc(&cyc, 148 * 8);
   cudaFuncSetAttribute(tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
   struct Cfg { const char* name; int b1, b2; uint32_t C_dim; };
-  std::vector<Cfg> cfgs = {{"box {64,128,1} rows contiguous-stride", 128, 1, (uint32_t)C},
-                           {"box {64,32,4} 3D", 32, 4, (uint32_t)C},
-                           {"box {64,64,2} 3D", 64, 2, (uint32_t)C},
-                           {"box {64,32,1} small", 32, 1, (uint32_t)C},
-                           {"box {64,128,1} C=48 (OOB tail)", 128, 1, 48u},
-                           {"box {64,256,1}", 256, 1, (uint32_t)C}};
+  std::vector<Cfg> cfgs = {{"box {64,128,1} 16KB", 128, 1, (uint32_t)C},
+                           {"box {64,32,1} 4KB", 32, 1, (uint32_t)C}};
   for (auto& c : cfgs) {
-    for (int depth : {4, 8}) for (int issuers : {1, 2, 4}) {
+    for (int depth : {8}) for (int lm : {0, 1}) for (int issuers : {1, 2, 4, 8}) {
       if (issuers > depth) continue;
+      if (!lm && issuers > 4) continue;
       CUtensorMap m;
       cuuint64_t dims[3] = {c.C_dim, (cuuint64_t)W, (cuuint64_t)H};
       cuuint64_t strides[2] = {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2};
@@ -101,12 +100,13 @@ int main() {
       size_t smem = 1024 + depth * bytes + depth * 8;
       int iters = 400;
       int n1 = W / c.b1 > 0 ? W - c.b1 + 1 : 1, n2 = H - c.b2 + 1;
-      tma_kernel<<<148, 32 * issuers, smem>>>(m, 20 * issuers, depth, bytes, n1, n2, cyc);  // warm
+      const int thr = lm ? 32 : 32 * issuers, lmode = lm ? issuers : 0;
+      tma_kernel<<<148, thr, smem>>>(m, 20 * issuers, depth, bytes, n1, n2, cyc, lmode);  // warm
       cudaEvent_t e0, e1;
       cudaEventCreate(&e0);
       cudaEventCreate(&e1);
       cudaEventRecord(e0);
-      tma_kernel<<<148, 32 * issuers, smem>>>(m, iters, depth, bytes, n1, n2, cyc);
+      tma_kernel<<<148, thr, smem>>>(m, iters, depth, bytes, n1, n2, cyc, lmode);
       cudaEventRecord(e1);
       cudaEventSynchronize(e1);
       float ms;
@@ -116,7 +116,7 @@ int main() {
       double avg = 0;
       for (auto v : h) avg += v;
       avg /= 148;
-      printf("%-40s depth %d issuers %d: %6.1f B/cycle/SM, %7.1f GB/s chip (%.1f us), err=%s\n", c.name, depth, issuers,
+      printf("%-40s depth %d %s %d: %6.1f B/cycle/SM, %7.1f GB/s chip (%.1f us), err=%s\n", c.name, depth, lm ? "lanes" : "warps", issuers,
              (double)bytes * iters / avg, (double)bytes * iters * 148 / (ms * 1e-3) / 1e9, ms * 1e3,
              cudaGetErrorString(cudaGetLastError()));
     }
