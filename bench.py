@@ -281,6 +281,8 @@ def main():
     ap.add_argument("--impl", default="hios", choices=["hios", "reference"])
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--sweep", default="2048,4096",
+                    help="extra input sizes timed on 1 GPU (HIOS-LP / sequential / IOS-style), '' to skip")
     ap.add_argument("--logical", type=int, default=0,
                     help="single process: schedule over this many logical GPUs (aliased on visible devices)")
     args = ap.parse_args()
@@ -406,12 +408,19 @@ def main():
         e2e.append((time.perf_counter() - t0) * 1e3)
     e2e_ms = max_over_ranks(dist, float(np.mean(e2e[args.warmup:])), world)
 
-    # ---------------- per-op device times (instrumented graph) for the roofline
+    # ---------------- dominant-kernel roofline: per-op device times from the
+    # instrumented graph (CUDA events recorded as graph nodes on the launching
+    # streams), over K steps with the L2 flushed between steps.  On one GPU the
+    # sequential schedule is instrumented so that no two ops overlap (the
+    # kernels and their launch order are those of the timed schedule).
+    Sr = h.hios_schedule_lp(G, 1, 1) if world == 1 else S
     op_ns_acc = np.zeros(g.n_ops)
     nt = max(3, min(args.steps, 10))
-    for i in range(nt):
+    for i in range(nt + 1):
         flush.fill_(float(i))
-        op_ns_acc += h.hios_run_timed(S, d_in.data_ptr(), d_out.data_ptr(), stream.cuda_stream)
+        t_ = h.hios_run_timed(Sr, d_in.data_ptr(), d_out.data_ptr(), stream.cuda_stream)
+        if i > 0:
+            op_ns_acc += t_
     torch.cuda.synchronize()
     op_ms = op_ns_acc / nt / 1e6
     F, B = op_work(g, shapes, esz)
@@ -424,6 +433,7 @@ def main():
     conv_ids = [o.id for o in g.ops if o.kind == "conv" and op_ms[o.id] > 0]
     conv_flops = float(F[conv_ids].sum())
     conv_s = float(op_ms[conv_ids].sum()) / 1e3
+    step_r = float(op_ms[op_ms > 0].sum())
     peak_t = pk["bf16_tflops_sustained"]
     achieved = conv_flops / conv_s / 1e12 if conv_s > 0 else 0.0
     traffic = None
@@ -433,13 +443,18 @@ def main():
             traffic = json.load(open(tp)).get("bytes_per_launch")
         except Exception:
             traffic = None
+    best = max(conv_ids, key=lambda v: F[v] / max(op_ms[v], 1e-9)) if conv_ids else None
     roof = {"bound": "tensor", "kernel": "conv_tc_kernel (tcgen05 implicit GEMM)",
             "achieved": achieved, "peak": peak_t, "unit": "TFLOP/s",
             "frac": achieved / peak_t if peak_t else None, "traffic": traffic,
             "launches_per_step": len(conv_ids),
             "flops_per_launch": conv_flops / max(len(conv_ids), 1),
             "avg_launch_us": conv_s / max(len(conv_ids), 1) * 1e6,
-            "share_of_step": conv_s * 1e3 / ms if ms > 0 else None,
+            "share_of_step": conv_s * 1e3 / step_r if step_r > 0 else None,
+            "best_launch": None if best is None else {
+                "op": g.ops[best].name, "us": float(op_ms[best] * 1e3),
+                "tflops": float(F[best] / (op_ms[best] * 1e-3) / 1e12)},
+            "measured_on": "sequential schedule, instrumented CUDA graph" if world == 1 else "timed schedule",
             "peak_src": f"{pk['src']} bf16 sustained (kernel inside a long step)"}
 
     cp_s = critical_path_bound(g, F, B, op_gpu, op_stage, M, pk, esz, shapes)
@@ -461,6 +476,43 @@ def main():
                            "predicted_ms": h.hios_schedule_latency_ns(Sx) / 1e6,
                            "gpus_used": int(len(set(h.hios_schedule_stages(Sx)[0].tolist())))}
             del Sx
+
+    sweep = {}
+    if world == 1 and args.sweep and not os.environ.get("HIOS_NCU"):
+        for sz in [int(v) for v in args.sweep.split(",") if v]:
+            gs = graphs.build(args.model, sz)
+            Ws = gen.make_weights(gs)
+            xs = gen.make_input(gs)
+            Gs = h.hios_graph_create(gs.ops, gs.edges, gs.in_c, gs.in_h, gs.in_w, args.dtype, Ws)
+            shp = {o.id: h.hios_graph_shape(Gs, o.id) for o in gs.ops}
+            h.hios_profile(Gs, [dev], 5)
+            din = torch.from_numpy(xs).to(f"cuda:{dev}")
+            dout = torch.empty(h.hios_output_numel(h.hios_schedule_lp(Gs, 1, 1)), dtype=torch.float32,
+                               device=f"cuda:{dev}")
+            row = {"input": f"1x{gs.in_c}x{sz}x{sz}"}
+            for name, (m_, w_) in {"hios_lp": (M, args.window), "sequential": (1, 1),
+                                   "ios_style": (1, args.window)}.items():
+                Sx = h.hios_schedule_lp(Gs, m_, w_)
+                for _ in range(3):
+                    h.hios_run_device(Sx, din.data_ptr(), dout.data_ptr(), stream.cuda_stream)
+                ev = []
+                for i in range(max(5, args.steps // 3)):
+                    flush.fill_(float(i))
+                    a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a_.record(stream)
+                    h.hios_run_device(Sx, din.data_ptr(), dout.data_ptr(), stream.cuda_stream)
+                    b_.record(stream)
+                    ev.append((a_, b_))
+                torch.cuda.synchronize()
+                row[name + "_ms"] = float(np.mean([a_.elapsed_time(b_) for a_, b_ in ev]))
+                if name == "hios_lp":
+                    og, ost, _ = h.hios_schedule_stages(Sx)
+                    Fs, Bs = op_work(gs, shp, esz)
+                    row["cp_bound_ms"] = critical_path_bound(gs, Fs, Bs, og, ost, M, pk, esz, shp) * 1e3
+                del Sx
+            row["cp_frac"] = row["cp_bound_ms"] / row["hios_lp_ms"]
+            sweep[str(sz)] = row
+            del Gs
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -485,6 +537,7 @@ def main():
                          "stages_per_gpu": [int(a) for a in n_stages], "predicted_ms": predicted_ms,
                          "profile_s": t_prof, "schedule_s": t_sched},
             "single_gpu_refs": extra,
+            "size_sweep": sweep,
             "wall_s_timed_region": wall,
         }
         if "sequential" in extra:

@@ -196,9 +196,9 @@ __global__ void __launch_bounds__(kThreads, 1)
   const uint32_t B_BYTES = (uint32_t)a.n_tile * 128;
   const uint32_t H_BYTES = a.halo ? halo_bytes_of(a.R, a.halo_w) : 0u;
   const uint32_t PITCH = stage_pitch(a.n_tile);
-  uint8_t* sA = smem;  // halo: a_bufs x H_BYTES ; tap: ST x A_BYTES
-  uint8_t* sB = smem + (a.halo ? a.a_bufs * H_BYTES : ST * A_BYTES);
-  uint8_t* sOut = sB + ST * B_BYTES;  // epilogue staging [128][PITCH]
+  uint8_t* sA = smem;  // halo: a_bufs x H_BYTES ; tap: ST x kps x A_BYTES
+  uint8_t* sB = smem + (a.halo ? a.a_bufs * H_BYTES : ST * a.kps * A_BYTES);
+  uint8_t* sOut = sB + ST * a.kps * B_BYTES;  // epilogue staging [128][PITCH]
   uint64_t* bars = reinterpret_cast<uint64_t*>(sOut + 128 * PITCH);
   // barriers: full[ST] empty[ST] afull[2] aempty[2] tfull[2] tempty[2]
   const uint32_t full0 = smem_u32(bars), empty0 = full0 + 8 * ST;
@@ -249,16 +249,16 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   // Each stage is owned by one producer warp (st = w mod n_prod, n_prod | ST),
   // so a stage's empty barrier is never waited on two phases ahead (parity
-  // waits cannot tell phase u from u-2).
+  // waits cannot tell phase u from u-2).  A stage carries up to `kps`
+  // consecutive K-steps: one full/empty handshake (~0.3 us of fixed latency,
+  // measured) is amortised over kps x 4 MMAs.
   const int n_prod = (ST % 4 == 0) ? 4 : ((ST % 2 == 0) ? 2 : 1);
+  const int KPS = a.kps;
+  const uint32_t A_STAGE = a.halo ? 0u : (uint32_t)KPS * A_BYTES;
+  const uint32_t B_STAGE = (uint32_t)KPS * B_BYTES;
   if (warp < kProducers) {
     if (warp < n_prod || (a.halo && warp == 0)) {
       // ------------------------------------------------------ TMA producers
-      // A cp.async.bulk.tensor keeps its issuing thread busy for hundreds of
-      // cycles (measured, tools/tma_bench.cu), so kProducers warps issue in
-      // parallel: warp w owns the K-steps ks = w (mod kProducers); warp 0
-      // also loads the halo boxes.  Every division is hoisted out of the K
-      // loop; stage, phase, tap and chunk advance incrementally.
       uint32_t st = 0, ph = 0, ab = 0, aph = 0, ks = 0;
       int mine = warp < n_prod ? warp : 1 << 30;
       const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
@@ -269,43 +269,58 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int p0 = tp * a.th, q0 = tq * a.tw, n0 = n_blk * a.n_tile;
         const int x0 = q0 * a.sw - a.pw, y0 = p0 * a.sh - a.ph;
         const int cc_lo = split * a.cps, cc_hi = min(a.c_chunks, cc_lo + a.cps);
-        for (int cc = cc_lo; cc < cc_hi; ++cc) {
-          const int c0 = cc * 64;
-          if (a.halo && warp == 0) {
+        int cc = cc_lo, rs = 0, r = 0, s = 0;
+        while (cc < cc_hi) {
+          if (a.halo && rs == 0 && warp == 0) {
             mbar_wait(aempty0 + 8 * ab, aph ^ 1u);
             if (elect_one()) {
               mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.R * a.halo_w * 128u);
-              tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, c0, x0, y0);
+              tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, cc * 64, x0, y0);
             }
             __syncwarp();
           }
-          if (a.halo) {
+          if (a.halo && rs == 0) {
             if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
           }
-          int r = 0, s = 0;
-          for (int rs = 0; rs < RS; ++rs, ++ks) {
-            if (mine == 0) {
-              mbar_wait(empty0 + 8 * st, ph ^ 1u);
-              if (elect_one()) {
-                TRACE2(2, ks);
-                if (a.dbg & 2) {  // debug: no operand traffic (timing experiments only)
-                  mbar_arrive(full0 + 8 * st);
-                } else if (a.halo) {
-                  mbar_expect_tx(full0 + 8 * st, B_BYTES);
-                } else {
-                  mbar_expect_tx(full0 + 8 * st, A_BYTES + B_BYTES);
-                  tma_load_3d(sA0 + st * A_BYTES, &mx, full0 + 8 * st, c0, x0 + s * a.dw, y0 + r * a.dh);
-                }
-                if (!(a.dbg & 2)) tma_load_3d(sB0 + st * B_BYTES, &mw, full0 + 8 * st, c0, rs, n0);
-                if (ks == 0) TRACE(2);
-                TRACE2(0, ks);
+          // K-steps of this stage: up to KPS, never crossing a chunk in halo mode
+          int nk = KPS;
+          if (a.halo) nk = min(nk, RS - rs);
+          if (mine == 0) {
+            mbar_wait(empty0 + 8 * st, ph ^ 1u);
+            if (elect_one()) {
+              TRACE2(2, ks);
+              // count this stage's K-steps (tap mode may cross chunks)
+              int c2 = cc, rs2 = rs, r2 = r, s2 = s, cnt = 0;
+              for (int j = 0; j < nk && c2 < cc_hi; ++j) {
+                ++cnt;
+                if (++rs2 == RS) { rs2 = 0; ++c2; }
               }
-              __syncwarp();
-              mine = n_prod;
+              if (a.dbg & 2) {
+                mbar_arrive(full0 + 8 * st);
+              } else {
+                mbar_expect_tx(full0 + 8 * st, (uint32_t)cnt * ((a.halo ? 0u : A_BYTES) + B_BYTES));
+                c2 = cc; rs2 = rs; r2 = r; s2 = s;
+                for (int j = 0; j < cnt; ++j) {
+                  if (!a.halo)
+                    tma_load_3d(sA0 + st * A_STAGE + j * A_BYTES, &mx, full0 + 8 * st, c2 * 64, x0 + s2 * a.dw,
+                                y0 + r2 * a.dh);
+                  tma_load_3d(sB0 + st * B_STAGE + j * B_BYTES, &mw, full0 + 8 * st, c2 * 64, rs2, n0);
+                  if (++s2 == a.S) { s2 = 0; ++r2; }
+                  if (++rs2 == RS) { rs2 = 0; r2 = 0; s2 = 0; ++c2; }
+                }
+              }
+              if (ks == 0) TRACE(2);
+              TRACE2(0, ks);
             }
-            --mine;
-            if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
+            __syncwarp();
+            mine = n_prod;
+          }
+          --mine;
+          if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
+          // advance by nk K-steps
+          for (int j = 0; j < nk && cc < cc_hi; ++j, ++ks) {
             if (++s == a.S) { s = 0; ++r; }
+            if (++rs == RS) { rs = 0; r = 0; s = 0; ++cc; }
           }
         }
       }
@@ -315,8 +330,6 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int j = warp - kProducers;  // N sub-tile of this MMA warp
     if (j < nmma) {
       // ------------------------------------------------------ MMA issuers
-      // tcgen05.mma issue also occupies its thread for ~100 cycles, so the N
-      // tile is split across nmma warps (separate TMEM column ranges, same A)
       const uint32_t idesc = (1u << 4)                          // D f32
                              | (1u << 7)                        // A bf16
                              | (1u << 10)                       // B bf16
@@ -333,40 +346,47 @@ __global__ void __launch_bounds__(kThreads, 1)
         uint32_t accum = 0;
         const int split = tile / tiles_mn;
         const int cc_lo = split * a.cps, cc_hi = min(a.c_chunks, cc_lo + a.cps);
-        for (int cc = cc_lo; cc < cc_hi; ++cc) {
-          const uint32_t abase = sA0 + ab * H_BYTES;
-          if (a.halo) {
+        int cc = cc_lo, rs = 0;
+        uint32_t aoff_r = 0, aoff = 0;
+        int s = 0;
+        uint32_t abase = sA0 + ab * H_BYTES;
+        while (cc < cc_hi) {
+          if (a.halo && rs == 0) {
+            abase = sA0 + ab * H_BYTES;
             mbar_wait(afull0 + 8 * ab, aph);
             tc_fence_after();
           }
-          uint32_t aoff_r = 0, aoff = 0;
-          int s = 0;
-          for (int rs = 0; rs < RS; ++rs, ++ks) {
-            mbar_wait(full0 + 8 * st, ph);
-            tc_fence_after();
-            if (lane == 0 && ks == 0 && j == 0) TRACE(3);
-            if (lane == 0 && j == 0) TRACE2(1, ks);
-            const uint32_t a_addr = a.halo ? abase + aoff : sA0 + st * A_BYTES;
+          int nk = KPS;
+          if (a.halo) nk = min(nk, RS - rs);
+          mbar_wait(full0 + 8 * st, ph);
+          tc_fence_after();
+          if (lane == 0 && ks == 0 && j == 0) TRACE(3);
+          if (lane == 0 && j == 0) TRACE2(1, ks);
+          const bool el = elect_one();
+          for (int jj = 0; jj < nk && cc < cc_hi; ++jj, ++ks) {
+            const uint32_t a_addr = a.halo ? abase + aoff : sA0 + st * A_STAGE + jj * A_BYTES;
             const uint64_t ad = umma_desc_sw128(a_addr, a.bo_mode);
-            const uint64_t bd = umma_desc_sw128(sB0 + st * B_BYTES);
-            if (elect_one()) {
-              if (!(a.dbg & 1)) {  // (dbg & 1: skip the MMAs, timing experiments only)
+            const uint64_t bd = umma_desc_sw128(sB0 + st * B_STAGE + jj * B_BYTES);
+            if (el && !(a.dbg & 1)) {
 #pragma unroll
-                for (int k = 0; k < 4; ++k)  // 4 x K=16 inside the 128-byte swizzle row
-                  mma_bf16(d, ad + 2 * k, bd + 2 * k, idesc, accum | (uint32_t)k);
-              }
-              mma_commit(empty0 + 8 * st);
+              for (int k = 0; k < 4; ++k)  // 4 x K=16 inside the 128-byte swizzle row
+                mma_bf16(d, ad + 2 * k, bd + 2 * k, idesc, accum | (uint32_t)k);
             }
-            __syncwarp();
             accum = 1;
-            if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
             if (++s == a.S) { s = 0; aoff_r += row_r; aoff = aoff_r; } else { aoff += row_s; }
+            if (++rs == RS) {
+              rs = 0; s = 0; aoff_r = 0; aoff = 0;
+              ++cc;
+              if (a.halo) {
+                if (el) mma_commit(aempty0 + 8 * ab);
+                if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
+                break;  // a halo stage never crosses a chunk
+              }
+            }
           }
-          if (a.halo) {
-            if (elect_one()) mma_commit(aempty0 + 8 * ab);
-            __syncwarp();
-            if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
-          }
+          if (el) mma_commit(empty0 + 8 * st);
+          __syncwarp();
+          if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
         }
         if (elect_one()) mma_commit(tfull0 + 8 * acc);
         __syncwarp();
@@ -556,8 +576,8 @@ void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st) {
 }
 
 size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
-  const size_t B = (size_t)a.n_tile * 128;
-  const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.R, a.halo_w) : (size_t)a.stages * 128 * 128;
+  const size_t B = (size_t)a.n_tile * 128 * a.kps;
+  const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.R, a.halo_w) : (size_t)a.stages * a.kps * 128 * 128;
   return 1024 + A + (size_t)a.stages * B + 128 * (size_t)stage_pitch(a.n_tile) + (2 * a.stages + 10) * 8 +
          2 * 256 * 4;
 }

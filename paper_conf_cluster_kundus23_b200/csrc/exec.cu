@@ -181,6 +181,12 @@ static std::vector<T> conv_layout(const float* W, int K, int C, int R, int S, in
   return out;
 }
 
+// stems (C <= 8, receptive field <= 49 taps, weights fit in smem): direct CUDA-core kernel
+static bool small_c_conv(const Op& o) {
+  return o.in_c <= 8 && o.kh * o.kw <= 49 && (size_t)o.out_c * o.kh * o.kw * o.in_c * 4 <= 96 * 1024 && o.dh == 1 &&
+         o.dw == 1;
+}
+
 template <typename T>
 static void upload_weights_T(Executor& ex, int v) {
   const Op& o = ex.g.ops[v];
@@ -191,6 +197,7 @@ static void upload_weights_T(Executor& ex, int v) {
     case HIOS_OP_CONV: {
       const int Cp = tc ? rup(o.in_c, 8) : o.in_c;
       x.w = upload(L, conv_layout<T>(o.weight.data(), o.out_c, o.in_c, o.kh, o.kw, Cp));
+      if (small_c_conv(o)) x.w_small = (float*)upload(L, conv_layout<float>(o.weight.data(), o.out_c, o.in_c, o.kh, o.kw, o.in_c));
       x.scale.push_back((float*)upload(L, o.scale));
       x.shift.push_back((float*)upload(L, o.shift));
       break;
@@ -347,16 +354,23 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   // occupancy: 1 CTA/SM (212 KB) or 2 CTAs/SM (104 KB each, TMEM <= 256 cols)
   c.occ = (getenv("HIOS_OCC") ? atoi(getenv("HIOS_OCC")) : 1) == 2 && c.n_tile <= 128 ? 2 : 1;
   const size_t budget = (c.occ == 2 ? 104 * 1024 : 212 * 1024) - stage_out;
+  // K-steps per stage: amortise the ~0.3 us full/empty handshake (measured)
+  c.kps = getenv("HIOS_KPS") ? std::max(1, atoi(getenv("HIOS_KPS"))) : 0;
   if (c.halo) {
     const size_t H = halo_bytes_of(R, hw);
-    c.a_bufs = (2 * H + 2 * B <= budget) ? 2 : 1;
-    if (H + 2 * B > budget) c.halo = 0;  // does not fit: fall back to tap mode
-    else c.stages = (int)std::min<size_t>(8, (budget - c.a_bufs * H) / B);
+    if (!c.kps) c.kps = std::min(4, R * S);
+    while (c.kps > 1 && H + 2 * c.kps * B > budget) --c.kps;
+    c.a_bufs = (2 * H + 2 * c.kps * B <= budget) ? 2 : 1;
+    if (H + 2 * c.kps * B > budget) c.halo = 0;  // does not fit: fall back to tap mode
+    else c.stages = (int)std::min<size_t>(8, (budget - c.a_bufs * H) / (c.kps * B));
   }
   if (!c.halo) {
-    c.stages = (int)std::min<size_t>(8, budget / (16384 + B));
+    if (!c.kps) c.kps = 4;
+    while (c.kps > 1 && 2 * c.kps * (16384 + B) > budget) --c.kps;
+    c.stages = (int)std::min<size_t>(8, budget / (c.kps * (16384 + B)));
   }
-  c.stages = std::max(2, std::min(c.stages, std::max(KI, 2)));
+  const int n_stage_steps = (KI + c.kps - 1) / c.kps;
+  c.stages = std::max(2, std::min(c.stages, std::max(n_stage_steps, 2)));
   // split-K (tap mode): a CTA's pipeline is latency-bound (~0.3 us per K-step,
   // DESIGN.md §6), so deep layers with few output tiles split their
   // 64-channel chunks across CTAs; fp32 partials are reduced by a finalize
@@ -364,9 +378,9 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   c.ksplit = 1;
   c.cps = c.c_chunks;
   const int tiles = c.tiles_m * c.tiles_n;
-  if (!c.halo && getenv("HIOS_SPLITK") && tiles < 100 && c.c_chunks >= 2 && R * S * c.c_chunks >= 8) {
+  if (!c.halo && !getenv("HIOS_NOSPLIT") && tiles < 48 && c.c_chunks >= 2 && R * S * c.c_chunks >= 24) {
     int want = std::min(c.c_chunks, std::max(1, (148 * c.occ + tiles - 1) / tiles));
-    want = std::min(want, std::max(1, R * S * c.c_chunks / 4));  // keep >= ~4 K-steps per split
+    want = std::min(want, std::max(1, R * S * c.c_chunks / 8));  // keep >= ~8 K-steps per split
     c.cps = (c.c_chunks + want - 1) / want;
     c.ksplit = (c.c_chunks + c.cps - 1) / c.cps;
   }
@@ -394,6 +408,7 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   ConvTcArgs a = plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw);
   if (getenv("HIOS_NOHALO") && a.halo) {  // debug: force tap mode on the same tiles
     a.halo = 0;
+    a.kps = 1;
     a.stages = std::max(2, std::min(8, (int)((212 * 1024 - 128 * (a.n_tile * 2 + 16)) / (16384 + a.n_tile * 128))));
   }
   CUtensorMap mx, mw;
@@ -475,6 +490,19 @@ static void build_op(Executor& ex, int v) {
     case HIOS_OP_CONV: {
       const int u = in_op(0);
       const Op& xi = g.ops[u];
+      if (small_c_conv(o)) {
+        View iv = view_of(u, l);
+        ConvSmallArgs<T> c{};
+        c.x = (const T*)iv.p; c.H = xi.H; c.W = xi.W; c.C = xi.C; c.ldx = iv.ldc;
+        c.w = x.w_small; c.scale = x.scale[0]; c.shift = x.shift[0];
+        c.P = o.H; c.Q = o.W; c.K = o.out_c; c.R = o.kh; c.S = o.kw; c.sh = o.sh; c.sw = o.sw;
+        c.ph = o.ph; c.pw = o.pw; c.relu = o.relu;
+        c.out = (T*)out.p; c.ldo = out.ldc;
+        c.out2 = out2 ? (T*)out2->p : nullptr; c.ldo2 = out2 ? out2->ldc : 0;
+        fns.push_back([c](cudaStream_t st) { launch_conv_small_c<T>(c, st); });
+        ++nk;
+        break;
+      }
       fns.push_back(conv_closure<T>(ex, view_of(u, l), xi.H, xi.W, xi.C, x.w, x.scale[0], x.shift[0], o.out_c, o.kh,
                                     o.kw, o.sh, o.sw, o.ph, o.pw, o.dh, o.dw, o.H, o.W, o.relu, out, out2, nk));
       break;

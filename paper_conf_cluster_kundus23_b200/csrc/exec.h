@@ -19,6 +19,7 @@ struct OpExec {
   std::vector<void*> pw;   // sepconv: per-rep pointwise weights
   std::vector<float*> dw;  // sepconv: per-rep depthwise weights [RS][C] fp32
   std::vector<float*> scale, shift;
+  float* w_small = nullptr;  // direct small-C conv weights [K][R][S][C] fp32
   float* bias = nullptr;
   int ldw = 0;
   // sepconv scratch (arena offsets)

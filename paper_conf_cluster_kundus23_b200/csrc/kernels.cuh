@@ -32,6 +32,7 @@ struct ConvTcArgs {
   int occ;                   // co-resident CTAs per SM the smem plan allows (1 or 2)
   int dbg;                   // debug switches (timing experiments; 0 in production)
   int ksplit, cps;           // split-K: splits and 64-channel chunks per split
+  int kps;                   // K-steps (64-channel x tap) per pipeline stage
   float* ws;                 // split-K fp32 workspace [ksplit][P*Q][ws_ld]
   size_t ws_split;           // elements per split
   int ws_ld;                 // row pitch (tiles_n * n_tile)
@@ -77,6 +78,15 @@ struct AddArgs {
   T* out2; int ldo2;
 };
 
+// direct conv for C <= 8 input channels (stems): fp32 weights [K][R][S][C]
+template <typename T>
+struct ConvSmallArgs {
+  const T* x; int H, W, C, ldx;
+  const float* w; const float* scale; const float* shift;
+  int P, Q, K, R, S, sh, sw, ph, pw, relu;
+  T* out; int ldo; T* out2; int ldo2;
+};
+
 template <typename T>
 struct CopyArgs {
   const T* x; int ldx; int HW, C; T* out; int ldo;
@@ -91,6 +101,7 @@ __host__ __device__ inline uint32_t halo_bytes_of(int R, int halo_w) {
   return ((uint32_t)R * halo_w * 128u + 1023u) & ~1023u;
 }
 void launch_conv_simt(const ConvSimtArgs& a, cudaStream_t st);
+template <typename T> void launch_conv_small_c(const ConvSmallArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_dw(const DwArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_pool(const PoolArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_add(const AddArgs<T>& a, cudaStream_t st);

@@ -352,3 +352,77 @@ HIOS_INST(float)
 HIOS_INST(bf16)
 
 }  // namespace hios
+
+namespace hios {
+// ------------------------------------------------- direct small-C conv
+// Stem convolutions with C <= 8 input channels (Inception's 3->32 3x3 s2,
+// SqueezeNet's 3->96 7x7 s2): K = C*R*S is tiny, so the tensor-core path
+// would waste >90 % of every 64-channel K-step.  One thread computes one
+// output pixel x 16 output channels on CUDA cores (fp32 FMA); the C x R x S
+// receptive field is read once into registers, weights come from smem.
+template <typename T>
+__global__ void conv_small_c_kernel(const ConvSmallArgs<T> a) {
+  extern __shared__ float sw[];  // [K][R*S*C] then scale[K], shift[K]
+  const int RSC = a.R * a.S * a.C;
+  for (int i = threadIdx.x; i < a.K * RSC; i += blockDim.x) sw[i] = a.w[i];
+  for (int i = threadIdx.x; i < a.K; i += blockDim.x) {
+    sw[a.K * RSC + i] = a.scale[i];
+    sw[a.K * RSC + a.K + i] = a.shift[i];
+  }
+  __syncthreads();
+  const int KG = (a.K + 15) / 16;
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= a.P * a.Q * KG) return;
+  const int kg = idx % KG, pix = idx / KG;
+  const int q = pix % a.Q, p = pix / a.Q;
+  const int h0 = p * a.sh - a.ph, w0 = q * a.sw - a.pw;
+  float x[8 * 49];  // C <= 8, R*S <= 49
+  int t = 0;
+  for (int r = 0; r < a.R; ++r)
+    for (int s = 0; s < a.S; ++s) {
+      const int h = h0 + r, w = w0 + s;
+      const bool ok = h >= 0 && h < a.H && w >= 0 && w < a.W;
+      const T* src = a.x + ((size_t)h * a.W + w) * a.ldx;
+      for (int c = 0; c < a.C; ++c) x[t++] = ok ? to_f(src[c]) : 0.f;
+    }
+  float acc[16];
+#pragma unroll
+  for (int j = 0; j < 16; ++j) acc[j] = 0.f;
+  const int k0 = kg * 16;
+  for (int i = 0; i < RSC; ++i) {
+    const float xv = x[i];
+#pragma unroll
+    for (int j = 0; j < 16; ++j) acc[j] = fmaf(xv, sw[min(k0 + j, a.K - 1) * RSC + i], acc[j]);
+  }
+  const float* ssc = sw + a.K * RSC;
+  const float* ssh = ssc + a.K;
+#pragma unroll
+  for (int j = 0; j < 16; ++j) {
+    const int k = min(k0 + j, a.K - 1);
+    float y = acc[j] * ssc[k] + ssh[k];
+    acc[j] = a.relu ? fmaxf(y, 0.f) : y;
+  }
+  for (int half = 0; half < 16; half += Vec<T>::N) {
+    const int k = k0 + half;
+    if (k >= a.K) break;
+    store_vec(a.out + (size_t)pix * a.ldo + k, k, a.K, acc + half);
+    if (a.out2) store_vec(a.out2 + (size_t)pix * a.ldo2 + k, k, a.K, acc + half);
+  }
+}
+
+template <typename T>
+void launch_conv_small_c(const ConvSmallArgs<T>& a, cudaStream_t st) {
+  const int KG = (a.K + 15) / 16;
+  const size_t smem = ((size_t)a.K * a.R * a.S * a.C + 2 * a.K) * sizeof(float);
+  static bool attr_set[64] = {false};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 64 && !attr_set[dev]) {
+    cudaFuncSetAttribute(conv_small_c_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    attr_set[dev] = true;
+  }
+  conv_small_c_kernel<T><<<grid_for((long long)a.P * a.Q * KG, 128), 128, smem, st>>>(a);
+}
+template void launch_conv_small_c<float>(const ConvSmallArgs<float>&, cudaStream_t);
+template void launch_conv_small_c<bf16>(const ConvSmallArgs<bf16>&, cudaStream_t);
+}  // namespace hios

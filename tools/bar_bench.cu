@@ -23,13 +23,14 @@ __device__ __forceinline__ void arrive(uint32_t bar) {
 }
 
 __global__ void ring_kernel(int iters, int ST, int mode, int use_commit, unsigned long long* out) {
-  __shared__ __align__(8) uint64_t full[16], empty[16];
+  __shared__ __align__(8) uint64_t full[16], empty[16], never;
   __shared__ uint32_t tslot;
   if (threadIdx.x == 0) {
     for (int i = 0; i < ST; ++i) {
       asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&full[i])));
       asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&empty[i])));
     }
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&never)));
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (threadIdx.x >= 32 && threadIdx.x < 64 && use_commit) {
@@ -42,14 +43,14 @@ __global__ void ring_kernel(int iters, int ST, int mode, int use_commit, unsigne
   if (warp == 0 && lane == 0) {
     uint32_t st = 0, ph = 0;
     for (int i = 0; i < iters; ++i) {
-      if (mode) wait_test(smem_u32(&empty[st]), ph ^ 1); else wait_try(smem_u32(&empty[st]), ph ^ 1);
+      if (mode == 1) wait_test(smem_u32(&empty[st]), ph ^ 1); else wait_try(smem_u32(&empty[st]), ph ^ 1);
       arrive(smem_u32(&full[st]));
       if (++st == (uint32_t)ST) { st = 0; ph ^= 1; }
     }
   } else if (warp == 1 && lane == 0) {
     uint32_t st = 0, ph = 0;
     for (int i = 0; i < iters; ++i) {
-      if (mode) wait_test(smem_u32(&full[st]), ph); else wait_try(smem_u32(&full[st]), ph);
+      if (mode == 1) wait_test(smem_u32(&full[st]), ph); else wait_try(smem_u32(&full[st]), ph);
       if (use_commit)
         asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
                          smem_u32(&empty[st]))
@@ -59,6 +60,11 @@ __global__ void ring_kernel(int iters, int ST, int mode, int use_commit, unsigne
       if (++st == (uint32_t)ST) { st = 0; ph ^= 1; }
     }
     if (blockIdx.x == 0) out[0] = clock64() - t0;
+    arrive(smem_u32(&never));  // release the spinning warps
+  } else if (warp >= 2) {
+    // extra warps spinning on a barrier (like epilogue warps waiting for an accumulator)
+    if (mode == 2) { uint32_t ok = 0; while (!ok) { asm volatile("{\n.reg .pred p;\nmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\nselp.b32 %0, 1, 0, p;\n}\n" : "=r"(ok) : "r"(smem_u32(&never)) : "memory"); if (!ok) __nanosleep(200); } }
+    else wait_try(smem_u32(&never), 0);
   }
   __syncthreads();
   if (threadIdx.x >= 32 && threadIdx.x < 64 && use_commit)
@@ -68,17 +74,18 @@ __global__ void ring_kernel(int iters, int ST, int mode, int use_commit, unsigne
 int main() {
   unsigned long long* d;
   cudaMalloc(&d, 8);
-  for (int commit : {0, 1})
-    for (int mode : {0, 1})
-      for (int ST : {2, 4, 8}) {
+  for (int extra : {0, 4, 10})
+  for (int commit : {1})
+    for (int mode : {0, 2})
+      for (int ST : {4}) {
         int iters = 4096;
-        ring_kernel<<<148, 64>>>(iters, ST, mode, commit, d);
-        ring_kernel<<<148, 64>>>(iters, ST, mode, commit, d);
+        ring_kernel<<<148, 64 + 32 * extra>>>(iters, ST, mode, commit, d);
+        ring_kernel<<<148, 64 + 32 * extra>>>(iters, ST, mode, commit, d);
         cudaDeviceSynchronize();
         unsigned long long h;
         cudaMemcpy(&h, d, 8, cudaMemcpyDeviceToHost);
-        printf("%s %s ST=%d: %.1f cycles / iteration  %s\n", commit ? "tcgen05.commit" : "arrive        ",
-               mode ? "test_wait" : "try_wait ", ST, (double)h / iters, cudaGetErrorString(cudaGetLastError()));
+        printf("extra spinning warps %2d, spin %s ST=%d: %.1f cycles / iteration  %s\n", extra,
+               mode == 2 ? "try+nanosleep" : "try_wait     ", ST, (double)h / iters, cudaGetErrorString(cudaGetLastError()));
       }
   return 0;
 }
