@@ -462,10 +462,10 @@ def main():
     extra = {}
     if world == 1:
         for name, (m_, w_) in {"sequential": (1, 1), "ios_style": (1, args.window),
-                               "lp_inter_only": (M, 1)}.items():
-            if name == "lp_inter_only" and M == 1:
+                               "lp_inter_only": (M, 1), "hios_mr": (M, args.window)}.items():
+            if name in ("lp_inter_only", "hios_mr") and M == 1:
                 continue
-            Sx = h.hios_schedule_lp(G, m_, w_)
+            Sx = h.hios_schedule_mr(G, m_, w_) if name == "hios_mr" else h.hios_schedule_lp(G, m_, w_)
             if m_ > 1:
                 ndev = torch.cuda.device_count()
                 h.hios_schedule_place(Sx, [i % ndev for i in range(m_)])

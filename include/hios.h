@@ -155,6 +155,15 @@ hios_status hios_profile(hios_graph g, const int32_t* devices, int32_t n_devices
  * measures t(S). */
 hios_status hios_schedule_lp(hios_graph g, int32_t n_gpus, int32_t window, hios_schedule* out);
 
+/* HIOS-MR, the paper's second scheduler (Alg. 3):
+ * mapping-recording DP over the ops in priority order (an n x M table of
+ * earliest finish times with back-pointers to the GPU of the previous op),
+ * back-tracked from the best GPU of the last op, then Alg. 2.  The extracted
+ * pseudo-code is garbled; the reconstruction is SURVEY C17 / DESIGN.md §3.
+ * Same arguments, costs and errors as hios_schedule_lp; window = 1 gives
+ * "MR-based inter-GPU" only. */
+hios_status hios_schedule_mr(hios_graph g, int32_t n_gpus, int32_t window, hios_schedule* out);
+
 /* Import a schedule: op_gpu[v] in [0, n_gpus), op_stage[v] = stage index on
  * that GPU (stages numbered 0..K_i-1; ops sharing an index form one stage).
  * Checked for feasibility (C6): HIOS_E_INVALID (dependent ops in a stage,

@@ -496,3 +496,53 @@ def random_dag(n_ops=200, n_layers=14, n_deps=None, p=0.8, seed=0, unit=1000):
             es.add((u, v))
     edges = [(u, v, max(int(0.1 * unit), int(round(p * t[u])))) for (u, v) in sorted(es)]
     return n_ops, t, edges
+
+
+# ------------------------------------------------ Alg. 3 (HIOS-MR)
+def hios_mr(n, t, edges, M, w, gcost):
+    """Alg. 3 (the extracted pseudo-code is garbled, reconstruction
+    C17): an n x M table (t_{i,j}, g_{i,j}) over the ops in priority order;
+    t_{i,j} = earliest finish of v_i on GPU j given the recorded schedule of
+    v_1..v_{i-1} that ends with v_{i-1} on GPU k (k chosen to minimise it,
+    first k wins ties: `if t_{i,j} > t_k + t(v_i)`); v_1 on GPU 1; back-track
+    from J = argmin_j t_{n,j}; then Alg. 2.  Returns (Q, L, gpu_of)."""
+    order = priority_order(n, t, edges)
+    pos = {v: i for i, v in enumerate(order)}
+    _, preds = succ_lists(n, edges)
+    INFV = float("inf")
+    T = [[INFV] * M for _ in range(n)]
+    Gb = [[0] * M for _ in range(n)]
+    T[0][0] = t[order[0]]
+    for i in range(1, n):
+        vi = order[i]
+        for j in range(min(M, i + 1)):
+            for k in range(min(M, i)):
+                if T[i - 1][k] == INFV:
+                    continue
+                # schedule of v_1..v_{i-1} recorded with v_{i-1} on GPU k (L10-12)
+                tF, gp = {}, {}
+                m = k
+                for l in range(i - 1, -1, -1):
+                    tF[order[l]] = T[l][m]
+                    gp[order[l]] = m
+                    m = Gb[l][m]
+                # L14: GPU j becomes free after the last op recorded on it
+                tk = max([tF[order[l]] for l in range(i) if gp[order[l]] == j] or [0])
+                # L15-19: inputs of v_i
+                for (u, c) in preds[vi]:
+                    if pos[u] >= i:
+                        continue
+                    tk = max(tk, tF[u] if gp[u] == j else tF[u] + c)
+                if T[i][j] > tk + t[vi]:  # L20-21
+                    T[i][j] = tk + t[vi]
+                    Gb[i][j] = k
+    J = min(range(M), key=lambda j: (T[n - 1][j], j))  # L22
+    gpu = {}
+    m = J
+    for i in range(n - 1, -1, -1):  # L24-25
+        gpu[order[i]] = m
+        m = Gb[i][m]
+    Q = [[(v,) for v in order if gpu[v] == g] for g in range(M)]
+    reach = reachability(n, edges)
+    Q, L = parallelize(n, t, edges, Q, w, gcost, order, reach)  # L27
+    return Q, L, gpu

@@ -142,6 +142,22 @@ hios_status hios_schedule_lp(hios_graph g, int32_t n_gpus, int32_t window, hios_
   });
 }
 
+hios_status hios_schedule_mr(hios_graph g, int32_t n_gpus, int32_t window, hios_schedule* out) {
+  if (out) *out = nullptr;
+  return guard([&] {
+    NEED(g && out, HIOS_E_INVALID, "NULL argument");
+    NEED(n_gpus >= 1 && n_gpus <= 64, HIOS_E_INVALID, "n_gpus out of [1, 64]");
+    NEED(window >= 1 && window <= 8, HIOS_E_INVALID, "window out of [1, 8]");
+    std::unique_ptr<hios::Schedule> s(new hios::Schedule);
+    s->g = g->g;
+    hios::hios_mr(*g->g, n_gpus, window, *s);
+    hios::finalize_schedule(*s);
+    auto* h = new hios_schedule_s;
+    h->s = std::move(s);
+    *out = h;
+  });
+}
+
 hios_status hios_schedule_import(hios_graph g, int32_t n_gpus, int32_t window, const int32_t* op_gpu,
                                  const int32_t* op_stage, hios_schedule* out) {
   if (out) *out = nullptr;

@@ -360,68 +360,105 @@ namespace hios {
 // would waste >90 % of every 64-channel K-step.  One thread computes one
 // output pixel x 16 output channels on CUDA cores (fp32 FMA); the C x R x S
 // receptive field is read once into registers, weights come from smem.
-template <typename T>
+template <typename T, int CC, int RR, int SS, int KT>
 __global__ void conv_small_c_kernel(const ConvSmallArgs<T> a) {
+  // CC/RR/SS > 0: compile-time receptive field (registers only); KT output
+  // channels per thread
   extern __shared__ float sw[];  // [K][R*S*C] then scale[K], shift[K]
-  const int RSC = a.R * a.S * a.C;
+  const int C = CC > 0 ? CC : a.C, R = RR > 0 ? RR : a.R, S = SS > 0 ? SS : a.S;
+  const int RSC = R * S * C;
   for (int i = threadIdx.x; i < a.K * RSC; i += blockDim.x) sw[i] = a.w[i];
   for (int i = threadIdx.x; i < a.K; i += blockDim.x) {
     sw[a.K * RSC + i] = a.scale[i];
     sw[a.K * RSC + a.K + i] = a.shift[i];
   }
   __syncthreads();
-  const int KG = (a.K + 15) / 16;
+  const int KG = (a.K + KT - 1) / KT;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= a.P * a.Q * KG) return;
   const int kg = idx % KG, pix = idx / KG;
   const int q = pix % a.Q, p = pix / a.Q;
   const int h0 = p * a.sh - a.ph, w0 = q * a.sw - a.pw;
-  float x[8 * 49];  // C <= 8, R*S <= 49
-  int t = 0;
-  for (int r = 0; r < a.R; ++r)
-    for (int s = 0; s < a.S; ++s) {
-      const int h = h0 + r, w = w0 + s;
-      const bool ok = h >= 0 && h < a.H && w >= 0 && w < a.W;
-      const T* src = a.x + ((size_t)h * a.W + w) * a.ldx;
-      for (int c = 0; c < a.C; ++c) x[t++] = ok ? to_f(src[c]) : 0.f;
-    }
-  float acc[16];
+  constexpr int XN = (CC > 0 && RR > 0 && SS > 0) ? CC * RR * SS : 8 * 49;
+  float x[XN];
+  if (CC > 0 && RR > 0 && SS > 0) {
 #pragma unroll
-  for (int j = 0; j < 16; ++j) acc[j] = 0.f;
-  const int k0 = kg * 16;
-  for (int i = 0; i < RSC; ++i) {
-    const float xv = x[i];
+    for (int r = 0; r < RR; ++r)
 #pragma unroll
-    for (int j = 0; j < 16; ++j) acc[j] = fmaf(xv, sw[min(k0 + j, a.K - 1) * RSC + i], acc[j]);
+      for (int s2 = 0; s2 < SS; ++s2) {
+        const int h = h0 + r, w = w0 + s2;
+        const bool ok = h >= 0 && h < a.H && w >= 0 && w < a.W;
+        const T* src = a.x + ((size_t)h * a.W + w) * a.ldx;
+#pragma unroll
+        for (int c = 0; c < CC; ++c) x[(r * SS + s2) * CC + c] = ok ? to_f(src[c]) : 0.f;
+      }
+  } else {
+    int t = 0;
+    for (int r = 0; r < R; ++r)
+      for (int s2 = 0; s2 < S; ++s2) {
+        const int h = h0 + r, w = w0 + s2;
+        const bool ok = h >= 0 && h < a.H && w >= 0 && w < a.W;
+        const T* src = a.x + ((size_t)h * a.W + w) * a.ldx;
+        for (int c = 0; c < C; ++c) x[t++] = ok ? to_f(src[c]) : 0.f;
+      }
   }
+  const int k0 = kg * KT;
   const float* ssc = sw + a.K * RSC;
   const float* ssh = ssc + a.K;
+  for (int kb = 0; kb < KT; kb += 16) {
+    float acc[16];
 #pragma unroll
-  for (int j = 0; j < 16; ++j) {
-    const int k = min(k0 + j, a.K - 1);
-    float y = acc[j] * ssc[k] + ssh[k];
-    acc[j] = a.relu ? fmaxf(y, 0.f) : y;
-  }
-  for (int half = 0; half < 16; half += Vec<T>::N) {
-    const int k = k0 + half;
-    if (k >= a.K) break;
-    store_vec(a.out + (size_t)pix * a.ldo + k, k, a.K, acc + half);
-    if (a.out2) store_vec(a.out2 + (size_t)pix * a.ldo2 + k, k, a.K, acc + half);
+    for (int j = 0; j < 16; ++j) acc[j] = 0.f;
+    if (CC > 0 && RR > 0 && SS > 0) {
+#pragma unroll
+      for (int i = 0; i < XN; ++i) {
+#pragma unroll
+        for (int j = 0; j < 16; ++j) acc[j] = fmaf(x[i], sw[min(k0 + kb + j, a.K - 1) * RSC + i], acc[j]);
+      }
+    } else {
+      for (int i = 0; i < RSC; ++i) {
+#pragma unroll
+        for (int j = 0; j < 16; ++j) acc[j] = fmaf(x[i], sw[min(k0 + kb + j, a.K - 1) * RSC + i], acc[j]);
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+      const int k = min(k0 + kb + j, a.K - 1);
+      float y = acc[j] * ssc[k] + ssh[k];
+      acc[j] = a.relu ? fmaxf(y, 0.f) : y;
+    }
+    for (int half = 0; half < 16; half += Vec<T>::N) {
+      const int k = k0 + kb + half;
+      if (k >= a.K) break;
+      store_vec(a.out + (size_t)pix * a.ldo + k, k, a.K, acc + half);
+      if (a.out2) store_vec(a.out2 + (size_t)pix * a.ldo2 + k, k, a.K, acc + half);
+    }
   }
 }
 
-template <typename T>
-void launch_conv_small_c(const ConvSmallArgs<T>& a, cudaStream_t st) {
-  const int KG = (a.K + 15) / 16;
+template <typename T, int CC, int RR, int SS, int KT>
+static void launch_small(const ConvSmallArgs<T>& a, cudaStream_t st) {
+  const int KG = (a.K + KT - 1) / KT;
   const size_t smem = ((size_t)a.K * a.R * a.S * a.C + 2 * a.K) * sizeof(float);
   static bool attr_set[64] = {false};
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev < 64 && !attr_set[dev]) {
-    cudaFuncSetAttribute(conv_small_c_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    cudaFuncSetAttribute(conv_small_c_kernel<T, CC, RR, SS, KT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         200 * 1024);
     attr_set[dev] = true;
   }
-  conv_small_c_kernel<T><<<grid_for((long long)a.P * a.Q * KG, 128), 128, smem, st>>>(a);
+  conv_small_c_kernel<T, CC, RR, SS, KT><<<grid_for((long long)a.P * a.Q * KG, 128), 128, smem, st>>>(a);
+}
+
+template <typename T>
+void launch_conv_small_c(const ConvSmallArgs<T>& a, cudaStream_t st) {
+  if (a.C == 3 && a.R == 3 && a.S == 3 && a.K % 32 == 0)
+    launch_small<T, 3, 3, 3, 32>(a, st);           // Inception / RandWire stems
+  else if (a.C == 3 && a.R == 7 && a.S == 7)
+    launch_small<T, 3, 7, 7, 16>(a, st);           // SqueezeNet conv1
+  else
+    launch_small<T, 0, 0, 0, 16>(a, st);
 }
 template void launch_conv_small_c<float>(const ConvSmallArgs<float>&, cudaStream_t);
 template void launch_conv_small_c<bf16>(const ConvSmallArgs<bf16>&, cudaStream_t);

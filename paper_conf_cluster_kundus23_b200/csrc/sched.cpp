@@ -261,6 +261,69 @@ void hios_lp(Graph& g, int M, int w, Schedule& s) {
   parallelize(g, s, order);  // Alg. 1 L17
 }
 
+// ------------------------------------------------------------ Alg. 3
+// HIOS-MR (garbled pseudo-code reconstructed per C17):
+// n x M table of (earliest finish t_{i,j} of v_i on GPU j, GPU g_{i,j} of
+// v_{i-1} in that recorded schedule), then back-track and Alg. 2.
+void hios_mr(Graph& g, int M, int w, Schedule& s) {
+  s.M = M;
+  s.w = w;
+  auto order = priority_order(g);
+  const int n = g.n;
+  std::vector<int> pos(n);
+  for (int i = 0; i < n; ++i) pos[order[i]] = i;
+  const int64_t INF = std::numeric_limits<int64_t>::max();
+  std::vector<int64_t> T((size_t)n * M, INF);
+  std::vector<int> Gb((size_t)n * M, 0);
+  T[0] = g.op_cost(order[0]);  // v_1 on GPU 1 (L5)
+  std::vector<int64_t> tF(n, 0);
+  std::vector<int> gp(n, -1);
+  std::vector<int64_t> ready(M, 0);
+  for (int i = 1; i < n; ++i) {
+    const int vi = order[i];
+    const int kmax = std::min(M, i);
+    for (int k = 0; k < kmax; ++k) {
+      if (T[(size_t)(i - 1) * M + k] == INF) continue;
+      // recorded schedule of v_1..v_{i-1} with v_{i-1} on GPU k (L9-12)
+      int m = k;
+      std::fill(ready.begin(), ready.end(), 0);
+      for (int l = i - 1; l >= 0; --l) {
+        const int vl = order[l];
+        tF[vl] = T[(size_t)l * M + m];
+        gp[vl] = m;
+        ready[m] = std::max(ready[m], tF[vl]);
+        m = Gb[(size_t)l * M + m];
+      }
+      const int jmax = std::min(M, i + 1);
+      for (int j = 0; j < jmax; ++j) {
+        int64_t tk = ready[j];  // L14
+        for (int e : g.ops[vi].in_edges) {  // L15-19
+          const int u = g.edges[e].src;
+          if (pos[u] >= i) continue;
+          tk = std::max(tk, gp[u] == j ? tF[u] : tF[u] + g.edge_cost(e));
+        }
+        const int64_t f = tk + g.op_cost(vi);
+        if (T[(size_t)i * M + j] > f) {  // L20-21 (first k wins ties)
+          T[(size_t)i * M + j] = f;
+          Gb[(size_t)i * M + j] = k;
+        }
+      }
+    }
+  }
+  int J = 0;  // L22
+  for (int j = 1; j < M; ++j)
+    if (T[(size_t)(n - 1) * M + j] < T[(size_t)(n - 1) * M + J]) J = j;
+  std::vector<int> gpu(n, 0);
+  int m = J;
+  for (int i = n - 1; i >= 0; --i) {  // L24-25
+    gpu[order[i]] = m;
+    m = Gb[(size_t)i * M + m];
+  }
+  s.Q.assign(M, {});
+  for (int v : order) s.Q[gpu[v]].push_back({v});
+  parallelize(g, s, order);  // L27
+}
+
 void finalize_schedule(Schedule& s) {
   Graph& g = *s.g;
   s.gpu_of.assign(g.n, -1);

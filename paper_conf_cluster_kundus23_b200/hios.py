@@ -64,6 +64,7 @@ def load() -> C.CDLL:
         "hios_profile": [VP, P(I32), I32, I32],
         "hios_schedule_lp": [VP, I32, I32, P(VP)],
         "hios_schedule_import": [VP, I32, I32, P(I32), P(I32), P(VP)],
+        "hios_schedule_mr": [VP, I32, I32, P(VP)],
         "hios_schedule_latency_ns": [VP, P(I64)],
         "hios_schedule_stages": [VP, P(I32), P(I32), P(I32)],
         "hios_schedule_place": [VP, P(I32), I32],
@@ -232,6 +233,12 @@ def hios_profile(g: Graph, devices: Sequence[int] = (0,), reps: int = 10):
 def hios_schedule_lp(g: Graph, n_gpus: int, window: int) -> Schedule:
     h = C.c_void_p()
     _ck(load().hios_schedule_lp(g.h, n_gpus, window, C.byref(h)))
+    return Schedule(h, g, n_gpus)
+
+
+def hios_schedule_mr(g: Graph, n_gpus: int, window: int) -> Schedule:
+    h = C.c_void_p()
+    _ck(load().hios_schedule_mr(g.h, n_gpus, window, C.byref(h)))
     return Schedule(h, g, n_gpus)
 
 
