@@ -52,49 +52,62 @@ static inline unsigned grid_for(long long n, int block) {
 }
 
 // ---------------------------------------------------------------- pooling
-template <typename T>
+// grid = (ceil(Q * CG / 256), P): one output row per blockIdx.y; KH/KW > 0
+// unroll the window (loads hoisted, accumulated immediately).
+template <typename T, int KH, int KW>
 __global__ void pool_kernel(const PoolArgs<T> a) {
   constexpr int N = Vec<T>::N;
+  const int kh = KH > 0 ? KH : a.kh, kw = KW > 0 ? KW : a.kw;
   const int CG = (a.C + N - 1) / N;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= a.P * a.Q * CG) return;
-  const int cg = idx % CG;
-  const int pix = idx / CG;
-  const int q = pix % a.Q, p = pix / a.Q;
+  if (idx >= a.Q * CG) return;
+  const int p = blockIdx.y;
+  const int q = idx / CG, cg = idx - q * CG;
   const int c = cg * N;
   const int h0 = p * a.sh - a.ph, w0 = q * a.sw - a.pw;
   float acc[N], v[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) acc[j] = a.is_max ? -INFINITY : 0.f;
   int cnt = 0;
-  for (int r = 0; r < a.kh; ++r) {
-    const int h = h0 + r;
-    if (h < 0 || h >= a.H) continue;
-    for (int s = 0; s < a.kw; ++s) {
-      const int w = w0 + s;
-      if (w < 0 || w >= a.W) continue;
-      load_vec(a.x + ((size_t)h * a.W + w) * a.ldx + c, c, a.C, v);
-      ++cnt;
 #pragma unroll
-      for (int j = 0; j < N; ++j) acc[j] = a.is_max ? fmaxf(acc[j], v[j]) : acc[j] + v[j];
+  for (int r = 0; r < (KH > 0 ? KH : 1); ++r) {
+    for (int r2 = 0; r2 < (KH > 0 ? 1 : kh); ++r2) {
+      const int h = h0 + (KH > 0 ? r : r2);
+      if (h < 0 || h >= a.H) continue;
+#pragma unroll
+      for (int s2 = 0; s2 < (KW > 0 ? KW : 1); ++s2) {
+        for (int s3 = 0; s3 < (KW > 0 ? 1 : kw); ++s3) {
+          const int w = w0 + (KW > 0 ? s2 : s3);
+          if (w < 0 || w >= a.W) continue;
+          load_vec(a.x + ((size_t)h * a.W + w) * a.ldx + c, c, a.C, v);
+          ++cnt;
+#pragma unroll
+          for (int j = 0; j < N; ++j) acc[j] = a.is_max ? fmaxf(acc[j], v[j]) : acc[j] + v[j];
+        }
+      }
     }
   }
   if (!a.is_max) {
     int div = cnt;
-    if (a.cip) div = (min(h0 + a.kh, a.H + a.ph) - h0) * (min(w0 + a.kw, a.W + a.pw) - w0);
+    if (a.cip) div = (min(h0 + kh, a.H + a.ph) - h0) * (min(w0 + kw, a.W + a.pw) - w0);
     const float inv = 1.f / (float)div;
 #pragma unroll
     for (int j = 0; j < N; ++j) acc[j] *= inv;
   }
-  store_vec(a.out + (size_t)pix * a.ldo + c, c, a.C, acc);
-  if (a.out2) store_vec(a.out2 + (size_t)pix * a.ldo2 + c, c, a.C, acc);
+  const size_t pix = (size_t)p * a.Q + q;
+  store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
+  if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
 }
 
 template <typename T>
 void launch_pool(const PoolArgs<T>& a, cudaStream_t st) {
   constexpr int N = Vec<T>::N;
-  long long n = (long long)a.P * a.Q * ((a.C + N - 1) / N);
-  pool_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(a);
+  const int per_row = a.Q * ((a.C + N - 1) / N);
+  dim3 grid((per_row + 255) / 256, a.P);
+  if (a.kh == 3 && a.kw == 3)
+    pool_kernel<T, 3, 3><<<grid, 256, 0, st>>>(a);
+  else
+    pool_kernel<T, 0, 0><<<grid, 256, 0, st>>>(a);
 }
 
 // ------------------------------------------- depthwise (+ aggregation, ReLU)
@@ -361,9 +374,11 @@ namespace hios {
 // output pixel x 16 output channels on CUDA cores (fp32 FMA); the C x R x S
 // receptive field is read once into registers, weights come from smem.
 template <typename T, int CC, int RR, int SS, int KT>
-__global__ void conv_small_c_kernel(const ConvSmallArgs<T> a) {
-  // CC/RR/SS > 0: compile-time receptive field (registers only); KT output
-  // channels per thread
+__global__ void __launch_bounds__(128) conv_small_c_kernel(const ConvSmallArgs<T> a) {
+  // CC/RR/SS > 0: compile-time receptive field kept in registers; KT output
+  // channels x PX=2 neighbouring output pixels (along W) per thread, so each
+  // weight read from smem feeds two FMAs
+  constexpr int PX = (CC > 0 && CC * RR * SS <= 64) ? 2 : 1;
   extern __shared__ float sw[];  // [K][R*S*C] then scale[K], shift[K]
   const int C = CC > 0 ? CC : a.C, R = RR > 0 ? RR : a.R, S = SS > 0 ? SS : a.S;
   const int RSC = R * S * C;
@@ -374,64 +389,87 @@ __global__ void conv_small_c_kernel(const ConvSmallArgs<T> a) {
   }
   __syncthreads();
   const int KG = (a.K + KT - 1) / KT;
+  const int QP = (a.Q + PX - 1) / PX;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= a.P * a.Q * KG) return;
-  const int kg = idx % KG, pix = idx / KG;
-  const int q = pix % a.Q, p = pix / a.Q;
-  const int h0 = p * a.sh - a.ph, w0 = q * a.sw - a.pw;
+  if (idx >= a.P * QP * KG) return;
+  const int kg = idx % KG, pq = idx / KG;
+  const int qp = pq % QP, p = pq / QP;
+  const int q0 = qp * PX;
   constexpr int XN = (CC > 0 && RR > 0 && SS > 0) ? CC * RR * SS : 8 * 49;
-  float x[XN];
-  if (CC > 0 && RR > 0 && SS > 0) {
+  float x[PX][XN];
 #pragma unroll
-    for (int r = 0; r < RR; ++r)
+  for (int u = 0; u < PX; ++u) {
+    const int h0 = p * a.sh - a.ph, w0 = (q0 + u) * a.sw - a.pw;
+    if (CC > 0 && RR > 0 && SS > 0) {
 #pragma unroll
-      for (int s2 = 0; s2 < SS; ++s2) {
-        const int h = h0 + r, w = w0 + s2;
-        const bool ok = h >= 0 && h < a.H && w >= 0 && w < a.W;
-        const T* src = a.x + ((size_t)h * a.W + w) * a.ldx;
+      for (int r = 0; r < RR; ++r)
 #pragma unroll
-        for (int c = 0; c < CC; ++c) x[(r * SS + s2) * CC + c] = ok ? to_f(src[c]) : 0.f;
-      }
-  } else {
-    int t = 0;
-    for (int r = 0; r < R; ++r)
-      for (int s2 = 0; s2 < S; ++s2) {
-        const int h = h0 + r, w = w0 + s2;
-        const bool ok = h >= 0 && h < a.H && w >= 0 && w < a.W;
-        const T* src = a.x + ((size_t)h * a.W + w) * a.ldx;
-        for (int c = 0; c < C; ++c) x[t++] = ok ? to_f(src[c]) : 0.f;
-      }
+        for (int s2 = 0; s2 < SS; ++s2) {
+          const int h = h0 + r, w = w0 + s2;
+          const bool ok = h >= 0 && h < a.H && w >= 0 && w < a.W && q0 + u < a.Q;
+          const T* src = a.x + ((size_t)h * a.W + w) * a.ldx;
+          float v8[Vec<T>::N];
+          // one 16-byte load per tap (pixel stride >= 8 channels, padding is zero)
+          if (ok) load_vec(src, 0, Vec<T>::N, v8);
+#pragma unroll
+          for (int c = 0; c < CC; ++c) x[u][(r * SS + s2) * CC + c] = ok ? v8[c] : 0.f;
+        }
+    } else {
+      int t = 0;
+      for (int r = 0; r < R; ++r)
+        for (int s2 = 0; s2 < S; ++s2) {
+          const int h = h0 + r, w = w0 + s2;
+          const bool ok = h >= 0 && h < a.H && w >= 0 && w < a.W && q0 + u < a.Q;
+          const T* src = a.x + ((size_t)h * a.W + w) * a.ldx;
+          for (int c = 0; c < C; ++c) x[u][t++] = ok ? to_f(src[c]) : 0.f;
+        }
+    }
   }
   const int k0 = kg * KT;
   const float* ssc = sw + a.K * RSC;
   const float* ssh = ssc + a.K;
   for (int kb = 0; kb < KT; kb += 16) {
-    float acc[16];
+    float acc[PX][16];
 #pragma unroll
-    for (int j = 0; j < 16; ++j) acc[j] = 0.f;
+    for (int u = 0; u < PX; ++u)
+#pragma unroll
+      for (int j = 0; j < 16; ++j) acc[u][j] = 0.f;
     if (CC > 0 && RR > 0 && SS > 0) {
 #pragma unroll
       for (int i = 0; i < XN; ++i) {
 #pragma unroll
-        for (int j = 0; j < 16; ++j) acc[j] = fmaf(x[i], sw[min(k0 + kb + j, a.K - 1) * RSC + i], acc[j]);
+        for (int j = 0; j < 16; ++j) {
+          const float wv = sw[min(k0 + kb + j, a.K - 1) * RSC + i];
+#pragma unroll
+          for (int u = 0; u < PX; ++u) acc[u][j] = fmaf(x[u][i], wv, acc[u][j]);
+        }
       }
     } else {
       for (int i = 0; i < RSC; ++i) {
 #pragma unroll
-        for (int j = 0; j < 16; ++j) acc[j] = fmaf(x[i], sw[min(k0 + kb + j, a.K - 1) * RSC + i], acc[j]);
+        for (int j = 0; j < 16; ++j) {
+          const float wv = sw[min(k0 + kb + j, a.K - 1) * RSC + i];
+#pragma unroll
+          for (int u = 0; u < PX; ++u) acc[u][j] = fmaf(x[u][i], wv, acc[u][j]);
+        }
       }
     }
 #pragma unroll
-    for (int j = 0; j < 16; ++j) {
-      const int k = min(k0 + kb + j, a.K - 1);
-      float y = acc[j] * ssc[k] + ssh[k];
-      acc[j] = a.relu ? fmaxf(y, 0.f) : y;
-    }
-    for (int half = 0; half < 16; half += Vec<T>::N) {
-      const int k = k0 + kb + half;
-      if (k >= a.K) break;
-      store_vec(a.out + (size_t)pix * a.ldo + k, k, a.K, acc + half);
-      if (a.out2) store_vec(a.out2 + (size_t)pix * a.ldo2 + k, k, a.K, acc + half);
+    for (int u = 0; u < PX; ++u) {
+      if (q0 + u >= a.Q) break;
+#pragma unroll
+      for (int j = 0; j < 16; ++j) {
+        const int k = min(k0 + kb + j, a.K - 1);
+        float y = acc[u][j] * ssc[k] + ssh[k];
+        acc[u][j] = a.relu ? fmaxf(y, 0.f) : y;
+      }
+      const size_t pix = (size_t)p * a.Q + q0 + u;
+      for (int half = 0; half < 16; half += Vec<T>::N) {
+        const int k = k0 + kb + half;
+        if (k >= a.K) break;
+        store_vec(a.out + pix * a.ldo + k, k, a.K, acc[u] + half);
+        if (a.out2) store_vec(a.out2 + pix * a.ldo2 + k, k, a.K, acc[u] + half);
+      }
     }
   }
 }
@@ -440,6 +478,8 @@ template <typename T, int CC, int RR, int SS, int KT>
 static void launch_small(const ConvSmallArgs<T>& a, cudaStream_t st) {
   const int KG = (a.K + KT - 1) / KT;
   const size_t smem = ((size_t)a.K * a.R * a.S * a.C + 2 * a.K) * sizeof(float);
+  const int px = (CC > 0 && CC * RR * SS <= 64) ? 2 : 1;
+  const long long nthreads = (long long)a.P * ((a.Q + px - 1) / px) * KG;
   static bool attr_set[64] = {false};
   int dev = 0;
   cudaGetDevice(&dev);
@@ -448,14 +488,14 @@ static void launch_small(const ConvSmallArgs<T>& a, cudaStream_t st) {
                          200 * 1024);
     attr_set[dev] = true;
   }
-  conv_small_c_kernel<T, CC, RR, SS, KT><<<grid_for((long long)a.P * a.Q * KG, 128), 128, smem, st>>>(a);
+  conv_small_c_kernel<T, CC, RR, SS, KT><<<grid_for(nthreads, 128), 128, smem, st>>>(a);
 }
 
 template <typename T>
 void launch_conv_small_c(const ConvSmallArgs<T>& a, cudaStream_t st) {
-  if (a.C == 3 && a.R == 3 && a.S == 3 && a.K % 32 == 0)
+  if (a.C == 3 && a.R == 3 && a.S == 3 && a.K % 32 == 0 && a.ldx >= Vec<T>::N)
     launch_small<T, 3, 3, 3, 32>(a, st);           // Inception / RandWire stems
-  else if (a.C == 3 && a.R == 7 && a.S == 7)
+  else if (a.C == 3 && a.R == 7 && a.S == 7 && a.ldx >= Vec<T>::N)
     launch_small<T, 3, 7, 7, 16>(a, st);           // SqueezeNet conv1
   else
     launch_small<T, 0, 0, 0, 16>(a, st);
