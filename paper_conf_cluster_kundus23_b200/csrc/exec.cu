@@ -330,10 +330,13 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     if (cost < best_cost * 0.98) { best_cost = cost; c.n_tile = nt; }
   }
   if (!c.halo) {
-    // tap mode: the per-K-step cost is dominated by a fixed ~0.3 us pipeline
-    // handshake (measured), so take the widest N tile (<= 256) that splits K
-    // evenly -- the most MMA work per K-step
-    const int nb = (K + 127) / 128;
+    // tap mode: the per-stage cost is dominated by a fixed handshake
+    // (measured), so take a wide N tile (<= 128) that splits K evenly
+    // (measured: halving helps ops run alone but loses under HIOS stages,
+    // where concurrent ops already fill the SMs -- kept as HIOS_TAPCAP)
+    int cap = 128;
+    if (getenv("HIOS_TAPCAP")) cap = std::max(16, atoi(getenv("HIOS_TAPCAP")));
+    const int nb = (K + cap - 1) / cap;
     c.n_tile = rup((K + nb - 1) / nb, 16);
   }
   c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
