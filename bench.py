@@ -26,6 +26,7 @@ import json
 import os
 import subprocess
 import sys
+import threading
 import time
 
 import numpy as np
@@ -129,40 +130,65 @@ def critical_path_bound(g, F, B, op_gpu, op_stage, n_gpus, pk, esz, shapes):
 
 # ------------------------------------------------------------ clocks
 class Clocks:
+    """SM clock + throttle reasons sampled DURING the timed region.
+
+    A thread polls NVML every ~2 ms (the timed region of a 1 ms inference is
+    only tens of ms, far below nvidia-smi's sampling period); ctypes releases
+    the GIL while the main thread launches, so sampling does not perturb it.
+    Falls back to `nvidia-smi -lms` if NVML is unavailable."""
+
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+
     def __init__(self, idx):
-        self.path = f"/tmp/hios_clocks_{os.getpid()}.csv"
-        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        self.sm, self.mx, self.reasons, self.err = [], [], set(), None
+        self.stop_ev = threading.Event()
         try:
-            self.p = subprocess.Popen(["nvidia-smi", f"--id={idx}", f"--query-gpu={q}",
-                                       "--format=csv,noheader,nounits", "-lms", "100"],
-                                      stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
-        except Exception:
-            self.p = None
+            import pynvml
+            pynvml.nvmlInit()
+            try:
+                import torch
+                nidx = torch.cuda._get_nvml_device_index(idx)
+            except Exception:
+                nidx = idx
+            hd = pynvml.nvmlDeviceGetHandleByIndex(nidx)
+            bits = {"hw_slowdown": pynvml.nvmlClocksEventReasonHwSlowdown,
+                    "hw_thermal_slowdown": pynvml.nvmlClocksEventReasonHwThermalSlowdown,
+                    "sw_thermal_slowdown": pynvml.nvmlClocksEventReasonSwThermalSlowdown,
+                    "sw_power_cap": pynvml.nvmlClocksEventReasonSwPowerCap}
+            self.mx.append(float(pynvml.nvmlDeviceGetMaxClockInfo(hd, pynvml.NVML_CLOCK_SM)))
+
+            def sample():
+                self.sm.append(float(pynvml.nvmlDeviceGetClockInfo(hd, pynvml.NVML_CLOCK_SM)))
+                r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(hd)
+                for n, bit in bits.items():
+                    if r & bit:
+                        self.reasons.add(n)
+
+            def loop():
+                while not self.stop_ev.is_set():
+                    try:
+                        sample()
+                    except Exception as e:  # noqa: BLE001
+                        self.err = str(e)
+                        return
+                    time.sleep(0.002)
+
+            self.t = threading.Thread(target=loop, daemon=True)
+            self.t.start()
+        except Exception as e:  # noqa: BLE001
+            self.t = None
+            self.err = f"nvml unavailable: {e}"
 
     def stop(self):
-        if self.p is None:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        self.p.terminate()
-        self.p.wait()
-        sm, mx, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for line in open(self.path):
-            f = [x.strip() for x in line.split(",")]
-            if len(f) < 9:
-                continue
-            try:
-                sm.append(float(f[1]))
-                mx.append(float(f[2]))
-            except ValueError:
-                continue
-            for n, val in zip(names, f[5:9]):
-                if val.lower() == "active":
-                    reasons.add(n)
-        return {"sm_mhz": float(np.median(sm)) if sm else None,
-                "sm_max_mhz": float(max(mx)) if mx else None,
-                "samples": len(sm), "reasons": sorted(reasons)}
+        self.stop_ev.set()
+        if self.t is not None:
+            self.t.join()
+        out = {"sm_mhz": float(np.median(self.sm)) if self.sm else None,
+               "sm_max_mhz": float(max(self.mx)) if self.mx else None,
+               "samples": len(self.sm), "reasons": sorted(self.reasons), "source": "nvml, 2 ms poll"}
+        if self.err:
+            out["error"] = self.err
+        return out
 
 
 # ------------------------------------------------------------ CPU oracle leg
