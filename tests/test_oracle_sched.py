@@ -243,3 +243,50 @@ def test_fig10_sequential_latency_generator():
         tot.append(sum(t) / 1000.0)
     mean = sum(tot) / len(tot)
     assert 395 < mean < 425
+
+
+# ------------------------------------------------------ HIOS-MR (Alg. 3)
+def test_mr_diamond_worked_by_hand():
+    """Alg. 3 (reading C17) worked by hand on a diamond
+    s(1) -> a(4), b(4) -> t(1), every edge 1, M = 2, w = 1.
+    Priority order s, a, b, t.  Table (finish times, back-pointer k):
+      s: T[0][0]=1
+      a: j0: 1+4=5 (k0) | j1: s cross 1+1, +4 = 6 (k0)
+      b: j0: k0 -> 5+4=9, k1 (a@1) -> 1+4=5  => 5 (k1)
+         j1: k0 (a@0) -> s cross 2, +4 = 6, k1 -> 6+4=10 => 6 (k0)
+      t: j0: k0 (b@0,a@1): max(5, a 6+1) + 1 = 8; k1 (b@1,a@0): max(5, 6+1)+1 = 8 -> 8 (first k)
+         j1: k0: ready 6, a@1 6, b@0 5+1 -> 7; k1: 7 (tie, first k) -> 7 (k0)
+    J = 1; back-track t@1 <- b@0 <- a@1 <- s@0; L = 7 = the optimum (brute force)."""
+    t = [1, 4, 4, 1]
+    E = [(0, 1, 1), (0, 2, 1), (1, 3, 1), (2, 3, 1)]
+    g = S.group_model(t)
+    Q, L, gpu = S.hios_mr(4, t, E, 2, 1, g)
+    assert gpu == {0: 0, 1: 1, 2: 0, 3: 1}
+    assert L == 7 == S.simulate(4, t, E, Q, g)[0]
+    assert S.brute_force(4, t, E, 2, 1, g)[0] == 7
+
+
+def test_mr_chain_and_single_gpu_are_sums():
+    rng = random.Random(11)
+    for _ in range(20):
+        n = rng.randint(1, 10)
+        t = [rng.randint(1, 50) for _ in range(n)]
+        E = [(i, i + 1, rng.randint(1, 30)) for i in range(n - 1)]
+        assert S.hios_mr(n, t, E, 3, 1, S.group_model(t))[1] == sum(t)
+    for _ in range(20):
+        n, t, E = S.random_dag(rng.randint(2, 12), 3, None, 0.8, rng.randint(0, 10**6), unit=10)
+        Q, L, _ = S.hios_mr(n, t, E, 1, 1, S.group_model(t))
+        assert L == sum(t) and len(Q) == 1
+
+
+@pytest.mark.parametrize("w", [1, 2])
+def test_mr_feasible_and_not_below_optimum(w):
+    rng = random.Random(21 + w)
+    for _ in range(30):
+        n, t, E = S.random_dag(rng.randint(3, 7), rng.randint(2, 3), None,
+                               rng.choice([0.4, 0.8, 1.2]), rng.randint(0, 10**6), unit=10)
+        g = S.group_model(t)
+        Q, L, _ = S.hios_mr(n, t, E, 2, w, g)
+        assert S.validate(n, t, E, Q, w, g) is None
+        assert S.simulate(n, t, E, Q, g)[0] == L
+        assert S.brute_force(n, t, E, 2, w, g)[0] <= L
