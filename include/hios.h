@@ -133,6 +133,16 @@ hios_status hios_set_group_model(hios_graph g, int32_t num, int32_t den);
 /* Read back t(v) [n_ops] and t(u, v) [n_edges] (either may be NULL). */
 hios_status hios_get_costs(hios_graph g, int64_t* op_ns, int64_t* edge_ns);
 
+/* t(S) of the stage S = ops[0..n) as the scheduler sees it ("t(S)"; the
+ * profiling step of P:322): n = 1 -> t(v); else a value injected by
+ * hios_set_group_cost, else -- after hios_profile -- the concurrent time of
+ * the ops forked onto n streams of devices[0] and joined (measured once,
+ * memoised; n <= 8), else the group model.  ops are op ids (any order, no
+ * duplicates; the caller states they are independent -- not checked).
+ * Writes *ns.  Errors: HIOS_E_INVALID, HIOS_E_STATE (no way to know t(S)),
+ * HIOS_E_UNSUPPORTED (n > 8 when measuring), HIOS_E_CUDA. */
+hios_status hios_group_cost(hios_graph g, const int32_t* ops, int32_t n, int64_t* ns);
+
 /* ------------------------------------------------------------- profile */
 
 /* Measure t(v) for every op (median of `reps` CUDA-event timings of the op's

@@ -117,6 +117,17 @@ hios_status hios_get_costs(hios_graph g, int64_t* op_ns, int64_t* edge_ns) {
   });
 }
 
+hios_status hios_group_cost(hios_graph g, const int32_t* ops, int32_t n, int64_t* ns) {
+  return guard([&] {
+    NEED(g && ops && ns && n >= 1, HIOS_E_INVALID, "bad arguments");
+    std::vector<int> S(ops, ops + n);
+    for (int v : S) NEED(v >= 0 && v < g->g->n, HIOS_E_INVALID, "op out of range");
+    std::sort(S.begin(), S.end());
+    NEED(std::adjacent_find(S.begin(), S.end()) == S.end(), HIOS_E_INVALID, "duplicate op");
+    *ns = g->g->stage_cost(S);
+  });
+}
+
 hios_status hios_profile(hios_graph g, const int32_t* devices, int32_t n_devices, int32_t reps) {
   return guard([&] {
     NEED(g, HIOS_E_INVALID, "graph is NULL");

@@ -61,6 +61,7 @@ def load() -> C.CDLL:
         "hios_set_group_cost": [VP, P(I32), I32, I64],
         "hios_set_group_model": [VP, I32, I32],
         "hios_get_costs": [VP, P(I64), P(I64)],
+        "hios_group_cost": [VP, P(I32), I32, P(I64)],
         "hios_profile": [VP, P(I32), I32, I32],
         "hios_schedule_lp": [VP, I32, I32, P(VP)],
         "hios_schedule_import": [VP, I32, I32, P(I32), P(I32), P(VP)],
@@ -222,6 +223,13 @@ def hios_get_costs(g: Graph):
     _ck(load().hios_get_costs(g.h, o.ctypes.data_as(C.POINTER(C.c_int64)),
                               e.ctypes.data_as(C.POINTER(C.c_int64))))
     return o, e[:g.n_edges]
+
+
+def hios_group_cost(g: Graph, ops: Sequence[int]) -> int:
+    a = _i32(ops)
+    ns = C.c_int64(0)
+    _ck(load().hios_group_cost(g.h, a.ctypes.data_as(C.POINTER(C.c_int32)), len(a), C.byref(ns)))
+    return ns.value
 
 
 def hios_profile(g: Graph, devices: Sequence[int] = (0,), reps: int = 10):

@@ -252,3 +252,21 @@ def test_simulation_study_orderings():
     assert m["lp"] <= m["mr"]
     assert m["lp"] <= m["lp_inter"]          # Alg. 2 never makes Alg. 1's schedule worse
     assert 350e3 < m["seq"] / 1.0 < 470e3     # ~411 ms sequential (Fig. 10)
+
+
+def test_group_cost_sources():
+    """hios_group_cost: t(v) for singletons, injected t(S) first, else the
+    group model; no source -> HIOS_E_STATE; bad ids -> HIOS_E_INVALID."""
+    n, t, E = S.random_dag(6, 2, None, 0.8, 3, unit=1000)
+    G, N, t_all, E_all = _cost_graph(n, t, E)
+    assert hios.hios_group_cost(G, [1]) == t_all[1]
+    with pytest.raises(hios.HiosError):
+        hios.hios_group_cost(G, [1, 2])          # nothing known yet
+    hios.hios_set_group_cost(G, [2, 1], 12345)
+    assert hios.hios_group_cost(G, [1, 2]) == 12345
+    hios.hios_set_group_model(G, 7, 10)
+    assert hios.hios_group_cost(G, [1, 2]) == 12345  # injected wins
+    assert hios.hios_group_cost(G, [1, 3]) == S.group_model(t_all)((1, 3))
+    for bad in ([1, 1], [N + 5], []):
+        with pytest.raises(hios.HiosError):
+            hios.hios_group_cost(G, bad)
