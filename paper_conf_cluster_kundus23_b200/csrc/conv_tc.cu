@@ -29,6 +29,7 @@
 //              with the conv stride as TMA traversal stride, plus B.
 // Out-of-bounds TMA reads return zero = the convolution's zero padding.
 #include <cstdio>
+#include <cstdlib>
 
 #include "kernels.cuh"
 
@@ -92,6 +93,18 @@ __device__ __forceinline__ void tma_load_3d(uint32_t dst, const CUtensorMap* map
       "[%2];" ::"r"(dst),
       "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
       : "memory");
+}
+__device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, uint32_t src, int c0, int c1, int c2) {
+  asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(src), "r"(c0), "r"(c1), "r"(c2)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 // one lane of a converged warp (the others skip the guarded issue but keep
 // running the warp-uniform loop, so operands stay in uniform registers)
@@ -188,6 +201,7 @@ __host__ __device__ inline uint32_t stage_pitch(int n_tile) { return (uint32_t)n
 
 __global__ void __launch_bounds__(kThreads, 1)
     conv_tc_kernel(const __grid_constant__ CUtensorMap mx, const __grid_constant__ CUtensorMap mw,
+                   const __grid_constant__ CUtensorMap mo, const __grid_constant__ CUtensorMap mo2,
                    const ConvTcArgs a) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -230,6 +244,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mx)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mw)) : "memory");
+    if (a.tma_out) {
+      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mo)) : "memory");
+      if (a.out2) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mo2)) : "memory");
+    }
   }
   if (warp == kProducers) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
@@ -441,7 +459,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (acc == 0) tph ^= 1u;
         continue;
       }
-      // previous tile fully copied out of sOut / s_scale (all 128 threads)
+      // previous tile fully copied out of sOut / s_scale (all 128 threads;
+      // TMA-store mode: the bulk stores have finished reading sOut)
+      if (a.tma_out && et == 0) bulk_wait_read0();
       asm volatile("bar.sync 1, 128;" ::: "memory");
       for (int jj = et; jj < a.n_tile; jj += 128) {
         const int nj = min(n0 + jj, a.K - 1);
@@ -455,6 +475,9 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (tcount == 0 && warp == kEpiWarp0 && lane == 0) TRACE(5);
       const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)a.n_tile;
       const uint32_t srow = smem_u32(sOut) + (uint32_t)m * PITCH;
+      // TMA-store staging: slabs of out_sw channels, [128 rows][out_sw*2 B],
+      // 16-byte chunks XOR-swizzled like the tensor map (bits 4.. ^= bits 7..)
+      const uint32_t SWB = (uint32_t)a.out_sw * 2u, swm = SWB / 16u - 1u;
       for (int col = 0; col < a.n_tile; col += 16) {
         uint32_t r[16];
         tmem_ld16(tbase + (uint32_t)col, r);
@@ -467,16 +490,43 @@ __global__ void __launch_bounds__(kThreads, 1)
           __nv_bfloat162 b2 = __floats2bfloat162_rn(y0, y1);
           pk[q] = *reinterpret_cast<uint32_t*>(&b2);
         }
-        sts128(srow + col * 2, pk[0], pk[1], pk[2], pk[3]);
-        sts128(srow + col * 2 + 16, pk[4], pk[5], pk[6], pk[7]);
+        if (a.tma_out) {
+          const uint32_t slab = (uint32_t)col / (uint32_t)a.out_sw;
+          const uint32_t cb = ((uint32_t)col - slab * (uint32_t)a.out_sw) * 2u;  // byte in the slab row
+          const uint32_t base = smem_u32(sOut) + slab * 128u * SWB;
+          const uint32_t o0 = (uint32_t)m * SWB + cb, o1 = o0 + 16u;
+          sts128(base + (o0 ^ (((o0 >> 7) & swm) << 4)), pk[0], pk[1], pk[2], pk[3]);
+          sts128(base + (o1 ^ (((o1 >> 7) & swm) << 4)), pk[4], pk[5], pk[6], pk[7]);
+        } else {
+          sts128(srow + col * 2, pk[0], pk[1], pk[2], pk[3]);
+          sts128(srow + col * 2 + 16, pk[4], pk[5], pk[6], pk[7]);
+        }
       }
       tc_fence_before();
       mbar_arrive(tempty0 + 8 * acc);  // TMEM accumulator free for the next tile
       if (tcount == 0 && warp == kEpiWarp0 && lane == 0) TRACE(6);
       acc ^= 1u;
       if (acc == 0) tph ^= 1u;
+      if (a.tma_out) fence_proxy_async_smem();  // generic-proxy smem writes -> async proxy
       asm volatile("bar.sync 1, 128;" ::: "memory");
       if (tcount == 0 && et == 0) TRACE3(0);
+      if (a.tma_out) {
+        // one thread ships the tile: one bulk-tensor store per slab (the
+        // tensor map clips pixels beyond P x Q and channels beyond K)
+        if (et == 0) {
+          const uint32_t nslab = (uint32_t)a.n_tile / (uint32_t)a.out_sw;
+          for (uint32_t sl = 0; sl < nslab; ++sl) {
+            const int c0 = n0 + (int)(sl * (uint32_t)a.out_sw);
+            if (c0 >= a.K) break;
+            const uint32_t src = smem_u32(sOut) + sl * 128u * SWB;
+            tma_store_3d(&mo, src, c0, q0, p0);
+            if (a.out2) tma_store_3d(&mo2, src, c0, q0, p0);
+          }
+          bulk_commit();
+        }
+        if (tcount == 0 && et == 0) TRACE3(1);
+        continue;
+      }
       // coalesced copy-out: the 128 epilogue threads walk (row, 16-byte
       // chunk) pairs row-major, so consecutive lanes store consecutive 16 B of
       // one output pixel row (loads issued ahead of the dependent stores)
@@ -521,6 +571,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       if (tcount == 0 && et == 0) TRACE3(1);
     }
+    if (a.tma_out && et == 0) bulk_wait0();  // stores complete before the CTA retires
     if (et == 0) TRACE3(2);
   }
   if (lane == 0 && warp < 8) TRACE3(3 + (warp >> 1));
@@ -582,8 +633,8 @@ size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
          2 * 256 * 4;
 }
 
-void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcArgs& a, int grid, size_t smem,
-                    cudaStream_t st) {
+void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const CUtensorMap& mo, const CUtensorMap& mo2,
+                    const ConvTcArgs& a, int grid, size_t smem, cudaStream_t st) {
   static bool attr_set[64] = {false};
   int dev = 0;
   cudaGetDevice(&dev);
@@ -601,7 +652,7 @@ void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcAr
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  cudaLaunchKernelEx(&cfg, conv_tc_kernel, mx, mw, a);
+  cudaLaunchKernelEx(&cfg, conv_tc_kernel, mx, mw, mo, mo2, a);
 }
 
 }  // namespace hios
@@ -642,7 +693,8 @@ static PFN_encodeTiled get_encode() {
 }
 
 bool make_tmap_3d(CUtensorMap* m, const void* base, uint64_t d0, uint64_t d1, uint64_t d2, uint64_t stride1_bytes,
-                  uint64_t stride2_bytes, uint32_t b0, uint32_t b1, uint32_t b2, uint32_t e1, uint32_t e2) {
+                  uint64_t stride2_bytes, uint32_t b0, uint32_t b1, uint32_t b2, uint32_t e1, uint32_t e2,
+                  int swizzle_bytes) {
   PFN_encodeTiled enc = get_encode();
   if (!enc) return false;
   cuuint64_t dims[3] = {d0, d1, d2};
@@ -650,14 +702,17 @@ bool make_tmap_3d(CUtensorMap* m, const void* base, uint64_t d0, uint64_t d1, ui
   cuuint32_t box[3] = {b0, b1, b2};
   cuuint32_t es[3] = {1, e1, e2};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims, strides, box, es,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   swizzle_bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                   : swizzle_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                         : CU_TENSOR_MAP_SWIZZLE_32B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) {
+  if (r != CUDA_SUCCESS && getenv("HIOS_TMAP_VERBOSE")) {
     fprintf(stderr, "hios: cuTensorMapEncodeTiled failed (%d): dims %llu %llu %llu box %u %u %u es %u %u\n", (int)r,
             (unsigned long long)d0, (unsigned long long)d1, (unsigned long long)d2, b0, b1, b2, e1, e2);
-    return false;
   }
-  return true;
+  return r == CUDA_SUCCESS;
 }
 
 }  // namespace hios

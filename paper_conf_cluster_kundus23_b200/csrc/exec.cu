@@ -434,6 +434,19 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   a.dbg = getenv("HIOS_DBG") ? atoi(getenv("HIOS_DBG")) : 0;
   a.out = (bf16*)out.p; a.ldo = out.ldc;
   a.out2 = out2 ? (bf16*)out2->p : nullptr; a.ldo2 = out2 ? out2->ldc : 0;
+  // epilogue by TMA bulk-tensor stores: output tensor map {K, Q, P} over the
+  // destination slice (clips the ragged pixel / channel edges of a tile)
+  CUtensorMap mo = mx, mo2 = mx;
+  a.out_sw = a.n_tile % 64 == 0 ? 64 : (a.n_tile % 32 == 0 ? 32 : 16);
+  a.tma_out = !getenv("HIOS_NOTMASTORE") && a.ksplit == 1 ? 1 : 0;
+  if (a.tma_out) {
+    const int sb = a.out_sw * 2;
+    const uint32_t bw = a.halo ? 128u : (uint32_t)a.tw, bh = a.halo ? 1u : (uint32_t)a.th;
+    a.tma_out = make_tmap_3d(&mo, out.p, K, Q, P, (uint64_t)out.ldc * 2, (uint64_t)Q * out.ldc * 2, a.out_sw, bw, bh,
+                             1, 1, sb) &&
+                (!out2 || make_tmap_3d(&mo2, out2->p, K, Q, P, (uint64_t)out2->ldc * 2,
+                                       (uint64_t)Q * out2->ldc * 2, a.out_sw, bw, bh, 1, 1, sb));
+  }
   const size_t smem = conv_tc_smem_bytes(a);
   const int grid = std::min(a.tiles_m * a.tiles_n * a.ksplit, 148 * a.occ);
   if (a.ksplit > 1) {
@@ -445,12 +458,12 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
     a.ws = (float*)ws;
     nk += 2;
     return [mx, mw, a, smem, grid](cudaStream_t st) {
-      launch_conv_tc(mx, mw, a, grid, smem, st);
+      launch_conv_tc(mx, mw, mx, mx, a, grid, smem, st);
       launch_conv_splitk_finalize(a, st);
     };
   }
   nk += 1;
-  return [mx, mw, a, smem, grid](cudaStream_t st) { launch_conv_tc(mx, mw, a, grid, smem, st); };
+  return [mx, mw, mo, mo2, a, smem, grid](cudaStream_t st) { launch_conv_tc(mx, mw, mo, mo2, a, grid, smem, st); };
 }
 
 template <>

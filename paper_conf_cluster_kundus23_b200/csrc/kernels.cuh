@@ -40,6 +40,8 @@ struct ConvTcArgs {
   const float* shift;  // [K]
   bf16* out;  int ldo; // primary output (channel offset applied)
   bf16* out2; int ldo2;// optional second destination (peer replica), or null
+  int tma_out;         // epilogue leaves smem by TMA bulk-tensor stores (else st.global)
+  int out_sw;          // TMA-store slab width in channels (64 / 32 / 16 = 128B/64B/32B swizzle)
 };
 
 // CUDA-core implicit GEMM (fp32) for the fp32 path (1e-4 parity).
@@ -93,8 +95,8 @@ struct CopyArgs {
 };
 
 // launchers (stream-ordered, capture-safe)
-void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const ConvTcArgs& a, int grid, size_t smem,
-                    cudaStream_t st);
+void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const CUtensorMap& mo, const CUtensorMap& mo2,
+                    const ConvTcArgs& a, int grid, size_t smem, cudaStream_t st);
 size_t conv_tc_smem_bytes(const ConvTcArgs& a);
 void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st);
 __host__ __device__ inline uint32_t halo_bytes_of(int R, int halo_w) {
@@ -121,6 +123,6 @@ void launch_fill(void* p, size_t bytes, cudaStream_t st);
 // tensor maps (driver entry point resolved at run time; no -lcuda)
 bool make_tmap_3d(CUtensorMap* m, const void* base, uint64_t d0, uint64_t d1, uint64_t d2,
                   uint64_t stride1_bytes, uint64_t stride2_bytes, uint32_t b0, uint32_t b1, uint32_t b2,
-                  uint32_t e1, uint32_t e2);
+                  uint32_t e1, uint32_t e2, int swizzle_bytes = 128);
 
 }  // namespace hios
