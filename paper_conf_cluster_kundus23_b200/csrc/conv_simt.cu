@@ -10,6 +10,7 @@ namespace hios {
 constexpr int SBM = 64, SBN = 64, SBK = 16;
 
 __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
+  pdl_enter();
   __shared__ float As[2][SBK][SBM + 4];
   __shared__ float Bs[2][SBK][SBN + 4];
   const int t = threadIdx.x, tx = t & 15, ty = t >> 4;
@@ -103,7 +104,7 @@ __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
 
 void launch_conv_simt(const ConvSimtArgs& a, cudaStream_t st) {
   dim3 grid((a.P * a.Q + SBM - 1) / SBM, (a.K + SBN - 1) / SBN);
-  conv_simt_kernel<<<grid, 256, 0, st>>>(a);
+  launch_pdl(conv_simt_kernel, grid, dim3(256), 0, st, a);
 }
 
 }  // namespace hios

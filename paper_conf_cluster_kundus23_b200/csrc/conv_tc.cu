@@ -162,10 +162,35 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
+// tcgen05.ld without the wait: the destination registers are only valid after
+// tmem_wait_pin() (which names them as in/out operands, so no use of them can
+// be scheduled ahead of the wait)
+__device__ __forceinline__ void tmem_ld16_nw(uint32_t taddr, uint32_t (&r)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+      "%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_wait_pin(uint32_t (&r)[16]) {
+  asm volatile("tcgen05.wait::ld.sync.aligned;"
+               : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]), "+r"(r[6]), "+r"(r[7]),
+                 "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]), "+r"(r[12]), "+r"(r[13]), "+r"(r[14]),
+                 "+r"(r[15])::"memory");
+}
+__device__ __forceinline__ void pin16(uint32_t (&r)[16]) {
+  asm volatile(""
+               : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]), "+r"(r[6]), "+r"(r[7]),
+                 "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]), "+r"(r[12]), "+r"(r[13]), "+r"(r[14]),
+                 "+r"(r[15])::"memory");
+}
+
 // optional timeline instrumentation (HIOS_TRACE): globaltimer at checkpoints
 __device__ unsigned long long g_conv_trace[256 * 8];
 __device__ unsigned long long g_conv_trace2[32 * 48];  // per CTA: issue[16], full[16], empty_ok[16]
 __device__ unsigned long long g_conv_trace3[32 * 8];   // per CTA: epilogue checkpoints
+__device__ unsigned long long g_conv_trace4[32 * 16];  // per CTA: first-tile epilogue, fine-grained
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
@@ -178,6 +203,10 @@ __device__ __forceinline__ unsigned long long gtimer() {
 #define TRACE3(k)                                                         \
   do {                                                                    \
     if (a.trace && blockIdx.x < 32) g_conv_trace3[blockIdx.x * 8 + (k)] = gtimer(); \
+  } while (0)
+#define TRACE4(k)                                                         \
+  do {                                                                    \
+    if (a.trace && blockIdx.x < 32 && tcount == 0 && et == 0) g_conv_trace4[blockIdx.x * 16 + (k)] = gtimer(); \
   } while (0)
 #define TRACE(k)                                                          \
   do {                                                                    \
@@ -461,38 +490,42 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       // previous tile fully copied out of sOut / s_scale (all 128 threads;
       // TMA-store mode: the bulk stores have finished reading sOut)
-      if (a.tma_out && et == 0) bulk_wait_read0();
+      TRACE4(0);
+      if (a.tma_out && lane == 0) bulk_wait_read0();
       asm volatile("bar.sync 1, 128;" ::: "memory");
       for (int jj = et; jj < a.n_tile; jj += 128) {
         const int nj = min(n0 + jj, a.K - 1);
-        s_scale[jj] = __ldg(a.scale + nj);
-        s_shift[jj] = __ldg(a.shift + nj);
+        asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_scale + jj)), "f"(__ldg(a.scale + nj)) : "memory");
+        asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_shift + jj)), "f"(__ldg(a.shift + nj)) : "memory");
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
+      TRACE4(1);
       mbar_wait(tfull0 + 8 * acc, tph);
       __syncwarp();
       tc_fence_after();
+      TRACE4(2);
       if (tcount == 0 && warp == kEpiWarp0 && lane == 0) TRACE(5);
       const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)a.n_tile;
       const uint32_t srow = smem_u32(sOut) + (uint32_t)m * PITCH;
       // TMA-store staging: slabs of out_sw channels, [128 rows][out_sw*2 B],
       // 16-byte chunks XOR-swizzled like the tensor map (bits 4.. ^= bits 7..)
       const uint32_t SWB = (uint32_t)a.out_sw * 2u, swm = SWB / 16u - 1u;
-      for (int col = 0; col < a.n_tile; col += 16) {
-        uint32_t r[16];
-        tmem_ld16(tbase + (uint32_t)col, r);
+      const uint32_t sw_log = a.out_sw == 64 ? 6u : (a.out_sw == 32 ? 5u : 4u);
+      const uint32_t s_sc = smem_u32(s_scale), s_sh = smem_u32(s_shift);
+      // one 16-column group: folded BN + ReLU -> bf16 -> staging tile
+      auto emit16 = [&](int col, const uint32_t (&r)[16], const float* sc, const float* sf) {
         uint32_t pk[8];
 #pragma unroll
         for (int q = 0; q < 8; ++q) {
-          float y0 = __uint_as_float(r[2 * q]) * s_scale[col + 2 * q] + s_shift[col + 2 * q];
-          float y1 = __uint_as_float(r[2 * q + 1]) * s_scale[col + 2 * q + 1] + s_shift[col + 2 * q + 1];
+          float y0 = __uint_as_float(r[2 * q]) * sc[2 * q] + sf[2 * q];
+          float y1 = __uint_as_float(r[2 * q + 1]) * sc[2 * q + 1] + sf[2 * q + 1];
           if (a.relu) { y0 = fmaxf(y0, 0.f); y1 = fmaxf(y1, 0.f); }
           __nv_bfloat162 b2 = __floats2bfloat162_rn(y0, y1);
           pk[q] = *reinterpret_cast<uint32_t*>(&b2);
         }
         if (a.tma_out) {
-          const uint32_t slab = (uint32_t)col / (uint32_t)a.out_sw;
-          const uint32_t cb = ((uint32_t)col - slab * (uint32_t)a.out_sw) * 2u;  // byte in the slab row
+          const uint32_t slab = (uint32_t)col >> sw_log;
+          const uint32_t cb = ((uint32_t)col - (slab << sw_log)) * 2u;  // byte in the slab row
           const uint32_t base = smem_u32(sOut) + slab * 128u * SWB;
           const uint32_t o0 = (uint32_t)m * SWB + cb, o1 = o0 + 16u;
           sts128(base + (o0 ^ (((o0 >> 7) & swm) << 4)), pk[0], pk[1], pk[2], pk[3]);
@@ -501,32 +534,66 @@ __global__ void __launch_bounds__(kThreads, 1)
           sts128(srow + col * 2, pk[0], pk[1], pk[2], pk[3]);
           sts128(srow + col * 2 + 16, pk[4], pk[5], pk[6], pk[7]);
         }
+      };
+      // 32 columns per round: two TMEM loads in flight, the BN parameters
+      // (broadcast ld.shared.v4; a generic pointer would compile to slow
+      // generic LD.E) fetched under their latency, one wait
+      for (int col = 0; col < a.n_tile; col += 32) {
+        const bool two = col + 16 < a.n_tile;  // warp-uniform
+        uint32_t r0[16], r1[16];
+        tmem_ld16_nw(tbase + (uint32_t)col, r0);
+        if (two) tmem_ld16_nw(tbase + (uint32_t)col + 16u, r1);
+        float sc[32], sf[32];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          const uint4 u = lds128(s_sc + (uint32_t)(col + 4 * q) * 4u);
+          const uint4 w = lds128(s_sh + (uint32_t)(col + 4 * q) * 4u);
+          sc[4 * q] = __uint_as_float(u.x); sc[4 * q + 1] = __uint_as_float(u.y);
+          sc[4 * q + 2] = __uint_as_float(u.z); sc[4 * q + 3] = __uint_as_float(u.w);
+          sf[4 * q] = __uint_as_float(w.x); sf[4 * q + 1] = __uint_as_float(w.y);
+          sf[4 * q + 2] = __uint_as_float(w.z); sf[4 * q + 3] = __uint_as_float(w.w);
+        }
+        tmem_wait_pin(r0);
+        pin16(r1);
+        if (col < 16 * 6) TRACE4(3 + col / 32);
+        emit16(col, r0, sc, sf);
+        if (two) emit16(col + 16, r1, sc + 16, sf + 16);
       }
       tc_fence_before();
       mbar_arrive(tempty0 + 8 * acc);  // TMEM accumulator free for the next tile
       if (tcount == 0 && warp == kEpiWarp0 && lane == 0) TRACE(6);
       acc ^= 1u;
       if (acc == 0) tph ^= 1u;
-      if (a.tma_out) fence_proxy_async_smem();  // generic-proxy smem writes -> async proxy
-      asm volatile("bar.sync 1, 128;" ::: "memory");
-      if (tcount == 0 && et == 0) TRACE3(0);
+      TRACE4(9);
       if (a.tma_out) {
-        // one thread ships the tile: one bulk-tensor store per slab (the
-        // tensor map clips pixels beyond P x Q and channels beyond K)
-        if (et == 0) {
-          const uint32_t nslab = (uint32_t)a.n_tile / (uint32_t)a.out_sw;
+        // each warp ships its own 32 rows as soon as they are staged (the
+        // four warps' bulk-tensor stores issue in parallel; the tensor map
+        // clips pixels beyond P x Q and channels beyond K)
+        fence_proxy_async_smem();  // generic-proxy smem writes -> async proxy
+        __syncwarp();
+        TRACE4(10);
+        if (lane == 0) {
+          const int bw = a.tw < 32 ? a.tw : 32;
+          const int mr = lw * 32, hh0 = mr / a.tw, ww0 = mr - hh0 * a.tw;
+          (void)bw;
+          const uint32_t nslab = (uint32_t)a.n_tile >> sw_log;
           for (uint32_t sl = 0; sl < nslab; ++sl) {
-            const int c0 = n0 + (int)(sl * (uint32_t)a.out_sw);
+            const int c0 = n0 + (int)(sl << sw_log);
             if (c0 >= a.K) break;
-            const uint32_t src = smem_u32(sOut) + sl * 128u * SWB;
-            tma_store_3d(&mo, src, c0, q0, p0);
-            if (a.out2) tma_store_3d(&mo2, src, c0, q0, p0);
+            const uint32_t src = smem_u32(sOut) + sl * 128u * SWB + (uint32_t)mr * SWB;
+            tma_store_3d(&mo, src, c0, q0 + ww0, p0 + hh0);
+            if (a.out2) tma_store_3d(&mo2, src, c0, q0 + ww0, p0 + hh0);
           }
           bulk_commit();
         }
+        __syncwarp();
+        TRACE4(12);
         if (tcount == 0 && et == 0) TRACE3(1);
         continue;
       }
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      TRACE4(11);
+      if (tcount == 0 && et == 0) TRACE3(0);
       // coalesced copy-out: the 128 epilogue threads walk (row, 16-byte
       // chunk) pairs row-major, so consecutive lanes store consecutive 16 B of
       // one output pixel row (loads issued ahead of the dependent stores)
@@ -571,7 +638,9 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       if (tcount == 0 && et == 0) TRACE3(1);
     }
-    if (a.tma_out && et == 0) bulk_wait0();  // stores complete before the CTA retires
+    if (a.tma_out && lane == 0) bulk_wait0();  // stores complete before the CTA retires
+    tcount = 0;
+    TRACE4(13);
     if (et == 0) TRACE3(2);
   }
   if (lane == 0 && warp < 8) TRACE3(3 + (warp >> 1));
@@ -588,6 +657,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 __global__ void conv_splitk_finalize(const float* __restrict__ ws, int ksplit, size_t ws_split, int ws_ld, int PQ,
                                      int K, const float* __restrict__ scale, const float* __restrict__ shift,
                                      int relu, bf16* out, int ldo, bf16* out2, int ldo2) {
+  pdl_enter();
   const int KG = (K + 7) / 8;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= PQ * KG) return;
@@ -622,8 +692,8 @@ __global__ void conv_splitk_finalize(const float* __restrict__ ws, int ksplit, s
 
 void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st) {
   const int PQ = a.P * a.Q, KG = (a.K + 7) / 8;
-  conv_splitk_finalize<<<(PQ * KG + 255) / 256, 256, 0, st>>>(a.ws, a.ksplit, a.ws_split, a.ws_ld, PQ, a.K, a.scale,
-                                                                a.shift, a.relu, a.out, a.ldo, a.out2, a.ldo2);
+  launch_pdl(conv_splitk_finalize, dim3((PQ * KG + 255) / 256), dim3(256), 0, st, (const float*)a.ws, a.ksplit,
+             a.ws_split, a.ws_ld, PQ, a.K, a.scale, a.shift, a.relu, a.out, a.ldo, a.out2, a.ldo2);
 }
 
 size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
@@ -660,6 +730,10 @@ void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const CUtensor
 extern "C" int hios_debug_conv_trace_reset(void) {
   static unsigned long long zero[2048];
   return (int)cudaMemcpyToSymbol(hios::g_conv_trace, zero, sizeof(zero));
+}
+
+extern "C" int hios_debug_conv_trace4(unsigned long long* out) {
+  return (int)cudaMemcpyFromSymbol(out, hios::g_conv_trace4, sizeof(unsigned long long) * 32 * 16);
 }
 
 extern "C" int hios_debug_conv_trace3(unsigned long long* out) {

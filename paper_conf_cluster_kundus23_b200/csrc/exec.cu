@@ -441,7 +441,8 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   a.tma_out = !getenv("HIOS_NOTMASTORE") && a.ksplit == 1 ? 1 : 0;
   if (a.tma_out) {
     const int sb = a.out_sw * 2;
-    const uint32_t bw = a.halo ? 128u : (uint32_t)a.tw, bh = a.halo ? 1u : (uint32_t)a.th;
+    // one box = one epilogue warp's 32 rows of the 128-pixel tile
+    const uint32_t bw = (uint32_t)std::min(a.tw, 32), bh = 32u / bw;
     a.tma_out = make_tmap_3d(&mo, out.p, K, Q, P, (uint64_t)out.ldc * 2, (uint64_t)Q * out.ldc * 2, a.out_sw, bw, bh,
                              1, 1, sb) &&
                 (!out2 || make_tmap_3d(&mo2, out2->p, K, Q, P, (uint64_t)out2->ldc * 2,

@@ -56,6 +56,7 @@ static inline unsigned grid_for(long long n, int block) {
 // unroll the window (loads hoisted, accumulated immediately).
 template <typename T, int KH, int KW>
 __global__ void pool_kernel(const PoolArgs<T> a) {
+  pdl_enter();
   constexpr int N = Vec<T>::N;
   const int kh = KH > 0 ? KH : a.kh, kw = KW > 0 ? KW : a.kw;
   const int CG = (a.C + N - 1) / N;
@@ -105,14 +106,15 @@ void launch_pool(const PoolArgs<T>& a, cudaStream_t st) {
   const int per_row = a.Q * ((a.C + N - 1) / N);
   dim3 grid((per_row + 255) / 256, a.P);
   if (a.kh == 3 && a.kw == 3)
-    pool_kernel<T, 3, 3><<<grid, 256, 0, st>>>(a);
+    launch_pdl(pool_kernel<T, 3, 3>, grid, dim3(256), 0, st, a);
   else
-    pool_kernel<T, 0, 0><<<grid, 256, 0, st>>>(a);
+    launch_pdl(pool_kernel<T, 0, 0>, grid, dim3(256), 0, st, a);
 }
 
 // ------------------------------------------- depthwise (+ aggregation, ReLU)
 template <typename T>
 __global__ void dw_kernel(const DwArgs<T> a) {
+  pdl_enter();
   constexpr int N = Vec<T>::N;
   const int CG = (a.C + N - 1) / N;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
@@ -153,12 +155,13 @@ template <typename T>
 void launch_dw(const DwArgs<T>& a, cudaStream_t st) {
   constexpr int N = Vec<T>::N;
   long long n = (long long)a.P * a.Q * ((a.C + N - 1) / N);
-  dw_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(a);
+  launch_pdl(dw_kernel<T>, dim3(grid_for(n, 256)), dim3(256), 0, st, a);
 }
 
 // ------------------------------------------------------------------- add
 template <typename T>
 __global__ void add_kernel(const AddArgs<T> a) {
+  pdl_enter();
   constexpr int N = Vec<T>::N;
   const int CG = (a.C + N - 1) / N;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
@@ -185,12 +188,13 @@ template <typename T>
 void launch_add(const AddArgs<T>& a, cudaStream_t st) {
   constexpr int N = Vec<T>::N;
   long long n = (long long)a.HW * ((a.C + N - 1) / N);
-  add_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(a);
+  launch_pdl(add_kernel<T>, dim3(grid_for(n, 256)), dim3(256), 0, st, a);
 }
 
 // ------------------------------------------------------------------ copy
 template <typename T>
 __global__ void copy_kernel(const CopyArgs<T> a) {
+  pdl_enter();
   constexpr int N = Vec<T>::N;
   const int CG = (a.C + N - 1) / N;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
@@ -212,13 +216,14 @@ template <typename T>
 void launch_copy(const CopyArgs<T>& a, cudaStream_t st) {
   constexpr int N = Vec<T>::N;
   long long n = (long long)a.HW * ((a.C + N - 1) / N);
-  copy_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(a);
+  launch_pdl(copy_kernel<T>, dim3(grid_for(n, 256)), dim3(256), 0, st, a);
 }
 
 // ------------------------------------------------------------------- GAP
 // one block per 8/4-channel group; threads stride over pixels; smem reduce
 template <typename T>
 __global__ void gap_kernel(const T* x, int HW, int C, int ldx, T* out) {
+  pdl_enter();
   constexpr int N = Vec<T>::N;
   const int c = blockIdx.x * N;
   float acc[N], v[N];
@@ -253,13 +258,14 @@ __global__ void gap_kernel(const T* x, int HW, int C, int ldx, T* out) {
 template <typename T>
 void launch_gap(const T* x, int HW, int C, int ldx, T* out, cudaStream_t st) {
   constexpr int N = Vec<T>::N;
-  gap_kernel<T><<<(C + N - 1) / N, 512, 0, st>>>(x, HW, C, ldx, out);
+  launch_pdl(gap_kernel<T>, dim3((C + N - 1) / N), dim3(512), 0, st, x, HW, C, ldx, out);
 }
 
 // ---------------------------------------------------------------- linear
 // one warp per output: y[k] = sum_c W[k,c] x[c] + b[k]
 template <typename T>
 __global__ void linear_kernel(const T* x, int Cin, const T* w, int ldw, const float* b, int K, T* out) {
+  pdl_enter();
   const int k = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const int lane = threadIdx.x & 31;
   if (k >= K) return;
@@ -278,12 +284,13 @@ __global__ void linear_kernel(const T* x, int Cin, const T* w, int ldw, const fl
 
 template <typename T>
 void launch_linear(const T* x, int Cin, const T* w, int ldw, const float* b, int K, T* out, cudaStream_t st) {
-  linear_kernel<T><<<(K + 7) / 8, 256, 0, st>>>(x, Cin, w, ldw, b, K, out);
+  launch_pdl(linear_kernel<T>, dim3((K + 7) / 8), dim3(256), 0, st, x, Cin, w, ldw, b, K, out);
 }
 
 // ------------------------------------------------- layout conversion
 template <typename T>
 __global__ void input_kernel(const float* nchw, int C, int HW, T* out, int ldo) {
+  pdl_enter();
   constexpr int N = Vec<T>::N;
   const int pix = blockIdx.x * blockDim.x + threadIdx.x;
   if (pix >= HW) return;
@@ -296,11 +303,12 @@ __global__ void input_kernel(const float* nchw, int C, int HW, T* out, int ldo) 
 }
 template <typename T>
 void launch_input(const float* nchw, int C, int H, int W, T* out, int ldo, cudaStream_t st) {
-  input_kernel<T><<<grid_for((long long)H * W, 256), 256, 0, st>>>(nchw, C, H * W, out, ldo);
+  launch_pdl(input_kernel<T>, dim3(grid_for((long long)H * W, 256)), dim3(256), 0, st, nchw, C, H * W, out, ldo);
 }
 
 template <typename T>
 __global__ void output_kernel(const T* x, int C, int HW, int ldx, float* nchw) {
+  pdl_enter();
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= (long long)C * HW) return;
   const int c = (int)(i / HW);
@@ -309,7 +317,7 @@ __global__ void output_kernel(const T* x, int C, int HW, int ldx, float* nchw) {
 }
 template <typename T>
 void launch_output(const T* x, int C, int H, int W, int ldx, float* nchw, cudaStream_t st) {
-  output_kernel<T><<<grid_for((long long)C * H * W, 256), 256, 0, st>>>(x, C, H * W, ldx, nchw);
+  launch_pdl(output_kernel<T>, dim3(grid_for((long long)C * H * W, 256)), dim3(256), 0, st, x, C, H * W, ldx, nchw);
 }
 
 // ----------------------------------------------- cross-GPU epoch flags
@@ -387,6 +395,7 @@ __global__ void __launch_bounds__(128) conv_small_c_kernel(const ConvSmallArgs<T
     sw[a.K * RSC + i] = a.scale[i];
     sw[a.K * RSC + a.K + i] = a.shift[i];
   }
+  pdl_enter();  // weights staged under the predecessor's tail
   __syncthreads();
   const int KG = (a.K + KT - 1) / KT;
   const int QP = (a.Q + PX - 1) / PX;
@@ -488,7 +497,7 @@ static void launch_small(const ConvSmallArgs<T>& a, cudaStream_t st) {
                          200 * 1024);
     attr_set[dev] = true;
   }
-  conv_small_c_kernel<T, CC, RR, SS, KT><<<grid_for(nthreads, 128), 128, smem, st>>>(a);
+  launch_pdl(conv_small_c_kernel<T, CC, RR, SS, KT>, dim3(grid_for(nthreads, 128)), dim3(128), smem, st, a);
 }
 
 template <typename T>

@@ -47,6 +47,13 @@ for (name, C, K, H, W, kh, kw, s, ph, pw) in SHAPES:
     lib.hios_debug_conv_trace3(b3)
     t3 = (np.array(b3, dtype=np.int64).reshape(32, 8)[0] - t0) / 1e3
     print("   cta0 epi: staged-sync %.2f copied %.2f loop-done %.2f | warps0-1 %.2f 2-3 %.2f 4-5 %.2f 6-7 %.2f" % tuple(t3[:7]))
+    b4 = (ctypes.c_ulonglong * (32 * 16))()
+    lib.hios_debug_conv_trace4(b4)
+    t4 = (np.array(b4, dtype=np.int64).reshape(32, 16) - t0) / 1e3
+    lab4 = ["top", "scale", "tfull", "ld0", "ld1", "ld2", "ld3", "ld4", "ld5", "tmem_done", "fence", "bar",
+            "tma_issued", "drained"]
+    for c in range(min(3, t4.shape[0])):
+        print(f"   cta{c} epi4  " + " ".join(f"{n}={v:.2f}" for n, v in zip(lab4, t4[c][:14]) if v > -1e6))
     print("   cta0 issue   ", " ".join(f"{v:6.2f}" for v in t2[0]))
     print("   cta0 full    ", " ".join(f"{v:6.2f}" for v in t2[1]))
     print("   cta0 emptyok ", " ".join(f"{v:6.2f}" for v in t2[2]))
