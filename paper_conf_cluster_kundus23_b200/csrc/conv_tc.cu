@@ -415,9 +415,13 @@ __global__ void __launch_bounds__(kThreads, 1)
             const uint64_t ad = umma_desc_sw128(a_addr, a.bo_mode);
             const uint64_t bd = umma_desc_sw128(sB0 + st * B_STAGE + jj * B_BYTES);
             if (el && !(a.dbg & 1)) {
-#pragma unroll
-              for (int k = 0; k < 4; ++k)  // 4 x K=16 inside the 128-byte swizzle row
-                mma_bf16(d, ad + 2 * k, bd + 2 * k, idesc, accum | (uint32_t)k);
+              // 4 x K=16 inside the 128-byte swizzle row; K=16 slices past the
+              // last real input channel are all zero (TMA fill) and skipped
+              const int kv = min(4, (a.C - cc * 64 + 15) >> 4);
+              mma_bf16(d, ad, bd, idesc, accum);
+              if (kv > 1) mma_bf16(d, ad + 2, bd + 2, idesc, 1u);
+              if (kv > 2) mma_bf16(d, ad + 4, bd + 4, idesc, 1u);
+              if (kv > 3) mma_bf16(d, ad + 6, bd + 6, idesc, 1u);
             }
             accum = 1;
             if (++s == a.S) { s = 0; aoff_r += row_r; aoff = aoff_r; } else { aoff += row_s; }

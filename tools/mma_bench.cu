@@ -18,13 +18,13 @@ __device__ __forceinline__ uint64_t desc(uint32_t saddr) {
   return d;
 }
 
-__global__ void mma_kernel(int iters, int n, int g, int wait_each, unsigned long long* out) {
+__global__ void mma_kernel(int iters, int n, int g, int wait_each, unsigned long long* out, int m = 128, int atmem = 0) {
   extern __shared__ uint8_t raw[];
   uint8_t* sm = (uint8_t*)(((uintptr_t)raw + 1023) & ~(uintptr_t)1023);
   __shared__ uint32_t tslot;
   __shared__ __align__(8) uint64_t bars[4];
   if (threadIdx.x < 32) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 256;" ::"r"(smem_u32(&tslot)));
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(&tslot)));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   if (threadIdx.x == 0) {
@@ -39,16 +39,21 @@ __global__ void mma_kernel(int iters, int n, int g, int wait_each, unsigned long
   if ((threadIdx.x & 31) == 0) {
     const int w = threadIdx.x >> 5;
     uint64_t& bar = bars[w];
-    const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+    const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(m >> 4) << 24);
     const uint64_t ad = desc(smem_u32(sm)), bd = desc(smem_u32(sm + 16384));
     uint32_t ph = 0;
     int gc = 0;
     long long t0 = clock64();
     for (int i = w; i < iters; i += issuers) {
       uint32_t acc = i > w;
-      asm volatile("{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\ntcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(
-                       tm + (uint32_t)(w * (256 / issuers))),
-                   "l"(ad + 2 * (i & 3)), "l"(bd + 2 * (i & 3)), "r"(idesc), "r"(acc));
+      if (atmem)
+        asm volatile("{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\ntcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(
+                         tm + (uint32_t)(w * (256 / issuers))),
+                     "r"(tm + 256u + 8u * (uint32_t)(i & 3)), "l"(bd + 2 * (i & 3)), "r"(idesc), "r"(acc));
+      else
+        asm volatile("{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\ntcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(
+                         tm + (uint32_t)(w * (256 / issuers))),
+                     "l"(ad + 2 * (i & 3)), "l"(bd + 2 * (i & 3)), "r"(idesc), "r"(acc));
       if (g > 0 && ++gc == g) {
         gc = 0;
         asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(&bar))
@@ -74,7 +79,7 @@ __global__ void mma_kernel(int iters, int n, int g, int wait_each, unsigned long
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
-  if (threadIdx.x < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 256;" ::"r"(tm));
+  if (threadIdx.x < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tm));
 }
 
 int main() {
@@ -97,5 +102,18 @@ int main() {
              we ? "+wait" : "     ", (double)h[0] / iters, (double)h[1] / iters, ideal,
              cudaGetErrorString(cudaGetLastError()));
     }
+  // operand-source study: M = 64 vs 128 (A bytes halve), A from smem vs TMEM
+  for (int atmem : {0, 1})
+    for (int m : {64, 128})
+      for (int n : {16, 32, 64, 128, 256}) {
+        int iters = 2048;
+        mma_kernel<<<148, 32, 70 * 1024>>>(iters, n, 0, 0, d, m, atmem);
+        mma_kernel<<<148, 32, 70 * 1024>>>(iters, n, 0, 0, d, m, atmem);
+        cudaDeviceSynchronize();
+        unsigned long long h[2];
+        cudaMemcpy(h, d, 16, cudaMemcpyDeviceToHost);
+        printf("A from %s M=%3d N=%3d: complete %.1f cyc/MMA (floor %.0f) %s\n", atmem ? "TMEM" : "smem", m, n,
+               (double)h[1] / iters, 128.0 * n / 256.0, cudaGetErrorString(cudaGetLastError()));
+      }
   return 0;
 }
