@@ -147,6 +147,30 @@ __device__ __forceinline__ void mma_bf16(uint32_t d_tmem, uint64_t a, uint64_t b
       "}\n" ::"r"(d_tmem),
       "l"(a), "l"(b), "r"(idesc), "r"(acc));
 }
+// the same, issued only where `on` != 0 (elected lane) -- predicated instead
+// of branched, so the issuing warp's loop stays convergent and its operands
+// stay in uniform registers
+__device__ __forceinline__ void mma_bf16_on(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc,
+                                            uint32_t on) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p, q;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "setp.ne.b32 q, %5, 0;\n"
+      "@q tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n"
+      "}\n" ::"r"(d_tmem),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc), "r"(on));
+}
+__device__ __forceinline__ void mma_commit_on(uint32_t bar, uint32_t on) {
+  asm volatile(
+      "{\n"
+      ".reg .pred q;\n"
+      "setp.ne.b32 q, %1, 0;\n"
+      "@q tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n"
+      "}\n" ::"r"(bar),
+      "r"(on)
+      : "memory");
+}
 __device__ __forceinline__ void mma_commit(uint32_t bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar)
                : "memory");
@@ -241,12 +265,14 @@ __global__ void __launch_bounds__(kThreads, 1)
   const uint32_t PITCH = stage_pitch(a.n_tile);
   uint8_t* sA = smem;  // halo: a_bufs x H_BYTES ; tap: ST x kps x A_BYTES
   uint8_t* sB = smem + (a.halo ? a.a_bufs * H_BYTES : ST * a.kps * A_BYTES);
-  uint8_t* sOut = sB + ST * a.kps * B_BYTES;  // epilogue staging [128][PITCH]
+  // B: a ring of ST stages x kps K-steps, or (bres) every K-step's weights resident
+  uint8_t* sOut = sB + (a.bres ? (uint32_t)(a.c_chunks * a.R * a.S) : (uint32_t)(ST * a.kps)) * B_BYTES;
   uint64_t* bars = reinterpret_cast<uint64_t*>(sOut + 128 * PITCH);
   // barriers: full[ST] empty[ST] afull[2] aempty[2] tfull[2] tempty[2]
   const uint32_t full0 = smem_u32(bars), empty0 = full0 + 8 * ST;
   const uint32_t afull0 = empty0 + 8 * ST, aempty0 = afull0 + 16, tfull0 = aempty0 + 16, tempty0 = tfull0 + 16;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * ST + 8);
+  const uint32_t bres_bar = smem_u32(bars + 2 * ST + 9);  // resident weights landed
   float* s_scale = reinterpret_cast<float*>(bars + 2 * ST + 10);  // [256]
   float* s_shift = s_scale + 256;                                  // [256]
 
@@ -264,6 +290,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(full0 + 8 * i, 1);
       mbar_init(empty0 + 8 * i, nmma);
     }
+    mbar_init(bres_bar, 1);
     for (int i = 0; i < 2; ++i) {
       mbar_init(afull0 + 8 * i, 1);
       mbar_init(aempty0 + 8 * i, nmma);
@@ -307,8 +334,22 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (warp < n_prod || (a.halo && warp == 0)) {
       // ------------------------------------------------------ TMA producers
       uint32_t st = 0, ph = 0, ab = 0, aph = 0, ks = 0;
+      int hcount = 0;  // halo loads issued (trace only)
       int mine = warp < n_prod ? warp : 1 << 30;
       const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
+      if (a.bres && warp == 0) {
+        // the CTA's whole B (tiles_n == 1): every (chunk, tap) box once
+        if (elect_one()) {
+          const int nb = a.c_chunks * RS;
+          mbar_expect_tx(bres_bar, (uint32_t)nb * B_BYTES);
+          for (int i = 0; i < nb; ++i) {
+            const int c2 = i / RS;
+            tma_load_3d(sB0 + (uint32_t)i * B_BYTES, &mw, bres_bar, c2 * 64, i - c2 * RS, 0);
+          }
+        }
+        __syncwarp();
+      }
+      if (a.bres) mine = 1 << 30;  // no B ring
       for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
         const int split = tile / tiles_mn, tmn = tile - split * tiles_mn;
         const int m_blk = tmn / a.tiles_n, n_blk = tmn - m_blk * a.tiles_n;
@@ -321,6 +362,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (a.halo && rs == 0 && warp == 0) {
             mbar_wait(aempty0 + 8 * ab, aph ^ 1u);
             if (elect_one()) {
+              if (a.bres) TRACE2(0, hcount);
               mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.R * a.halo_w * 128u);
               tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, cc * 64, x0, y0);
             }
@@ -328,6 +370,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
           if (a.halo && rs == 0) {
             if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
+            ++hcount;
           }
           // K-steps of this stage: up to KPS, never crossing a chunk in halo mode
           int nk = KPS;
@@ -386,6 +429,68 @@ __global__ void __launch_bounds__(kThreads, 1)
       const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB) + (uint32_t)(j * n_sub) * 128u;
       const uint32_t row_r = (uint32_t)a.halo_w * 128u, row_s = (uint32_t)a.dw * 128u;
       int tcount = 0;
+      if (a.bres) {
+        mbar_wait(bres_bar, 0);
+        tc_fence_after();
+      }
+      if (a.halo) {
+        // halo mode, lean issue loop: per tap two 64-bit descriptor adds and
+        // up to 4 predicated MMAs (no branches on the elected lane, no
+        // per-K-step parameter reloads)
+        const int C = a.C, nchunks = a.c_chunks, S_ = a.S, kps = KPS, bres = a.bres, abufs = a.a_bufs;
+        const uint32_t on = elect_one() ? 1u : 0u;
+        const uint32_t ST_ = (uint32_t)ST;
+        const uint64_t row_r16 = row_r >> 4, row_s16 = row_s >> 4, b16 = B_BYTES >> 4, bst16 = B_STAGE >> 4;
+        const uint64_t bres0 = umma_desc_sw128(sB0);
+        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
+          mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
+          tc_fence_after();
+          const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
+          uint32_t accum = 0;
+          for (int cc = 0; cc < nchunks; ++cc) {
+            mbar_wait(afull0 + 8 * ab, aph);
+            tc_fence_after();
+            if (bres && lane == 0 && j == 0) TRACE2(1, tcount);
+            const uint64_t a0 = umma_desc_sw128(sA0 + ab * H_BYTES);
+            const int kv = min(4, (C - cc * 64 + 15) >> 4);
+            uint64_t aoff_r = 0, aoff = 0;
+            int s_ = 0;
+            for (int t = 0; t < RS;) {
+              const int nk = min(kps, RS - t);
+              uint64_t b0;
+              if (!bres) {
+                mbar_wait(full0 + 8 * st, ph);
+                tc_fence_after();
+                b0 = umma_desc_sw128(sB0 + st * B_STAGE);
+              } else {
+                b0 = bres0 + (uint64_t)(cc * RS + t) * b16;
+              }
+              for (int jj = 0; jj < nk; ++jj) {
+                const uint64_t ad = a0 + aoff, bd = b0 + (uint64_t)jj * b16;
+                mma_bf16_on(d, ad, bd, idesc, accum, on);
+                if (kv > 1) mma_bf16_on(d, ad + 2, bd + 2, idesc, 1u, on);
+                if (kv > 2) mma_bf16_on(d, ad + 4, bd + 4, idesc, 1u, on);
+                if (kv > 3) mma_bf16_on(d, ad + 6, bd + 6, idesc, 1u, on);
+                accum = 1;
+                if (++s_ == S_) { s_ = 0; aoff_r += row_r16; aoff = aoff_r; } else { aoff += row_s16; }
+              }
+              t += nk;
+              if (!bres) {
+                mma_commit_on(empty0 + 8 * st, on);
+                if (++st == ST_) { st = 0; ph ^= 1u; }
+              }
+            }
+            mma_commit_on(aempty0 + 8 * ab, on);
+            if (abufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
+          }
+          if (bres && lane == 0 && j == 0) TRACE2(2, tcount);
+          mma_commit_on(tfull0 + 8 * acc, on);
+          __syncwarp();
+          if (lane == 0 && tcount == 0 && j == 0) TRACE(4);
+          acc ^= 1u;
+          if (acc == 0) tph ^= 1u;
+        }
+      } else
       for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
         mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
         tc_fence_after();
@@ -402,18 +507,22 @@ __global__ void __launch_bounds__(kThreads, 1)
             abase = sA0 + ab * H_BYTES;
             mbar_wait(afull0 + 8 * ab, aph);
             tc_fence_after();
+            if (a.bres && lane == 0 && j == 0) TRACE2(1, tcount);
           }
           int nk = KPS;
           if (a.halo) nk = min(nk, RS - rs);
-          mbar_wait(full0 + 8 * st, ph);
-          tc_fence_after();
+          if (!a.bres) {
+            mbar_wait(full0 + 8 * st, ph);
+            tc_fence_after();
+          }
           if (lane == 0 && ks == 0 && j == 0) TRACE(3);
           if (lane == 0 && j == 0) TRACE2(1, ks);
           const bool el = elect_one();
           for (int jj = 0; jj < nk && cc < cc_hi; ++jj, ++ks) {
             const uint32_t a_addr = a.halo ? abase + aoff : sA0 + st * A_STAGE + jj * A_BYTES;
             const uint64_t ad = umma_desc_sw128(a_addr, a.bo_mode);
-            const uint64_t bd = umma_desc_sw128(sB0 + st * B_STAGE + jj * B_BYTES);
+            const uint64_t bd = umma_desc_sw128(a.bres ? sB0 + (uint32_t)(cc * RS + rs) * B_BYTES
+                                                       : sB0 + st * B_STAGE + jj * B_BYTES);
             if (el && !(a.dbg & 1)) {
               // 4 x K=16 inside the 128-byte swizzle row; K=16 slices past the
               // last real input channel are all zero (TMA fill) and skipped
@@ -435,10 +544,11 @@ __global__ void __launch_bounds__(kThreads, 1)
               }
             }
           }
-          if (el) mma_commit(empty0 + 8 * st);
+          if (el && !a.bres) mma_commit(empty0 + 8 * st);
           __syncwarp();
           if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
         }
+        if (a.bres && lane == 0 && j == 0) TRACE2(2, tcount);
         if (elect_one()) mma_commit(tfull0 + 8 * acc);
         __syncwarp();
         if (lane == 0 && tcount == 0 && j == 0) TRACE(4);
@@ -701,9 +811,9 @@ void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st) {
 }
 
 size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
-  const size_t B = (size_t)a.n_tile * 128 * a.kps;
+  const size_t B = a.bres ? (size_t)a.n_tile * 128 * a.c_chunks * a.R * a.S : (size_t)a.n_tile * 128 * a.kps * a.stages;
   const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.R, a.halo_w) : (size_t)a.stages * a.kps * 128 * 128;
-  return 1024 + A + (size_t)a.stages * B + 128 * (size_t)stage_pitch(a.n_tile) + (2 * a.stages + 10) * 8 +
+  return 1024 + A + B + 128 * (size_t)stage_pitch(a.n_tile) + (2 * a.stages + 10) * 8 +
          2 * 256 * 4;
 }
 

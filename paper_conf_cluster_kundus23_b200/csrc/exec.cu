@@ -359,7 +359,19 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   const size_t budget = (c.occ == 2 ? 104 * 1024 : 212 * 1024) - stage_out;
   // K-steps per stage: amortise the ~0.3 us full/empty handshake (measured)
   c.kps = getenv("HIOS_KPS") ? std::max(1, atoi(getenv("HIOS_KPS"))) : 0;
-  if (c.halo) {
+  // resident weights (halo mode, one N tile, CTAs that walk several tiles):
+  // the whole B is loaded once per CTA instead of once per tile (measured:
+  // Conv2d_2a re-read 36 KB of weights per 25 KB input tile)
+  const size_t b_all = (size_t)c.c_chunks * R * S * B;
+  c.bres = 0;
+  if (c.halo && c.tiles_n == 1 && c.tiles_m > 148 * c.occ && b_all <= 96 * 1024 && !getenv("HIOS_NOBRES") &&
+      halo_bytes_of(R, hw) + b_all <= budget) {
+    c.bres = 1;
+    c.kps = std::min(4, R * S);
+    c.a_bufs = (2 * halo_bytes_of(R, hw) + b_all <= budget) ? 2 : 1;
+    c.stages = 2;
+  }
+  if (c.halo && !c.bres) {
     const size_t H = halo_bytes_of(R, hw);
     if (!c.kps) c.kps = std::min(4, R * S);
     while (c.kps > 1 && H + 2 * c.kps * B > budget) --c.kps;
@@ -411,6 +423,7 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   ConvTcArgs a = plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw);
   if (getenv("HIOS_NOHALO") && a.halo) {  // debug: force tap mode on the same tiles
     a.halo = 0;
+    a.bres = 0;
     a.kps = 1;
     a.stages = std::max(2, std::min(8, (int)((212 * 1024 - 128 * (a.n_tile * 2 + 16)) / (16384 + a.n_tile * 128))));
   }

@@ -72,6 +72,7 @@ struct ConvTcArgs {
   const float* shift;  // [K]
   bf16* out;  int ldo; // primary output (channel offset applied)
   bf16* out2; int ldo2;// optional second destination (peer replica), or null
+  int bres;            // halo mode, one N tile: all weights resident in smem (loaded once per CTA)
   int tma_out;         // epilogue leaves smem by TMA bulk-tensor stores (else st.global)
   int out_sw;          // TMA-store slab width in channels (64 / 32 / 16 = 128B/64B/32B swizzle)
 };

@@ -33,7 +33,7 @@ __device__ __forceinline__ void mma_ts(uint32_t d, uint32_t a, uint64_t b, uint3
 
 // each issuing warp: `iters` rounds of 4 MMAs (one 64-channel K-step), into
 // its own accumulator columns; commit + wait at the end only
-__global__ void bench(int iters, int n, int m, int atmem, unsigned long long* out) {
+__global__ void bench(int iters, int n, int m, int atmem, unsigned long long* out, int aoff = 0, int rot = 0) {
   extern __shared__ uint8_t raw[];
   uint8_t* sm = (uint8_t*)(((uintptr_t)raw + 1023) & ~(uintptr_t)1023);
   __shared__ uint32_t tslot;
@@ -55,7 +55,7 @@ __global__ void bench(int iters, int n, int m, int atmem, unsigned long long* ou
   const uint32_t cols_per = atmem ? 256u / nw : 512u / nw;
   const uint32_t d = tm + (uint32_t)warp * cols_per;
   const uint32_t at = tm + 256u + (uint32_t)warp * 8u;  // A in TMEM (only with atmem: nw*n <= 256)
-  const uint64_t ad = desc(smem_u32(sm) + warp * 16384), bd = desc(smem_u32(sm + 65536));
+  const uint64_t ad = desc(smem_u32(sm) + warp * 16384 + aoff), bd = desc(smem_u32(sm + 65536));
   long long t0 = clock64();
   const bool el = elect_one();
   for (int i = 0; i < iters; ++i) {
@@ -63,7 +63,7 @@ __global__ void bench(int iters, int n, int m, int atmem, unsigned long long* ou
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
         if (atmem) mma_ts(d, at + 2u * k, bd + 2 * k, idesc, (i | k) ? 1u : 0u);
-        else mma_ss(d, ad + 2 * k, bd + 2 * k, idesc, (i | k) ? 1u : 0u);
+        else mma_ss(d, ad + 2 * k + (rot ? (uint64_t)(8 * (i % 3)) : 0), bd + 2 * k, idesc, (i | k) ? 1u : 0u);
       }
     }
     __syncwarp();
@@ -86,21 +86,18 @@ int main() {
   unsigned long long* d;
   cudaMalloc(&d, 64);
   cudaFuncSetAttribute(bench, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-  for (int atmem : {0, 1})
-    for (int nw : {1, 2, 4})
-      for (int m : {64, 128})
-        for (int n : {32, 64, 128, 256}) {
-          if (atmem ? (n * nw > 256) : (n * nw > 512)) continue;
-          const int iters = 1024;
-          bench<<<148, 32 * nw, 140 * 1024>>>(iters, n, m, atmem, d);
-          bench<<<148, 32 * nw, 140 * 1024>>>(iters, n, m, atmem, d);
-          cudaError_t e = cudaDeviceSynchronize();
-          unsigned long long h[8];
-          cudaMemcpy(h, d, 64, cudaMemcpyDeviceToHost);
-          const double per = (double)h[0] / (iters * 4.0);  // cycles per MMA per issuer
-          printf("A=%s warps=%d M=%3d N=%3d: %.1f cyc/MMA per issuer, %.1f cyc/MMA per SM (floor %.0f) %s\n",
-                 atmem ? "tmem" : "smem", nw, m, n, per, per / nw, (m > 128 ? m : 128) * n / 256.0,
-                 cudaGetErrorString(e));
-        }
+  // A window alignment study (halo mode starts A windows at any 128-B row)
+  for (int n : {32, 64, 128, 256})
+    for (int aoff : {0, 128, 384, 1152})
+      for (int rot : {0, 1}) {
+        const int iters = 1024;
+        bench<<<148, 32, 140 * 1024>>>(iters, n, 128, 0, d, aoff, rot);
+        bench<<<148, 32, 140 * 1024>>>(iters, n, 128, 0, d, aoff, rot);
+        cudaError_t e = cudaDeviceSynchronize();
+        unsigned long long h[8];
+        cudaMemcpy(h, d, 64, cudaMemcpyDeviceToHost);
+        printf("N=%3d A start +%4d B %s: %.1f cyc/MMA (floor %.0f) %s\n", n, aoff, rot ? "(rotating +0/128/256 B)" : "                       ",
+               (double)h[0] / (iters * 4.0), 128.0 * n / 256.0, cudaGetErrorString(e));
+      }
   return 0;
 }
