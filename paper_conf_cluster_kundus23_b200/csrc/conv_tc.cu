@@ -490,70 +490,52 @@ __global__ void __launch_bounds__(kThreads, 1)
           acc ^= 1u;
           if (acc == 0) tph ^= 1u;
         }
-      } else
-      for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
-        mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
-        tc_fence_after();
-        const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
-        uint32_t accum = 0;
-        const int split = tile / tiles_mn;
-        const int cc_lo = split * a.cps, cc_hi = min(a.c_chunks, cc_lo + a.cps);
-        int cc = cc_lo, rs = 0;
-        uint32_t aoff_r = 0, aoff = 0;
-        int s = 0;
-        uint32_t abase = sA0 + ab * H_BYTES;
-        while (cc < cc_hi) {
-          if (a.halo && rs == 0) {
-            abase = sA0 + ab * H_BYTES;
-            mbar_wait(afull0 + 8 * ab, aph);
-            tc_fence_after();
-            if (a.bres && lane == 0 && j == 0) TRACE2(1, tcount);
-          }
-          int nk = KPS;
-          if (a.halo) nk = min(nk, RS - rs);
-          if (!a.bres) {
+      } else {
+        // tap mode, lean issue loop: a stage carries up to kps K-steps (may
+        // cross a 64-channel chunk); descriptors are stage bases + strides
+        const int C = a.C, kps = KPS;
+        const uint32_t on = elect_one() ? 1u : 0u;
+        const uint32_t ST_ = (uint32_t)ST;
+        const uint64_t aD0 = umma_desc_sw128(sA0), bD0 = umma_desc_sw128(sB0);
+        const uint64_t ast16 = A_STAGE >> 4, bst16 = B_STAGE >> 4, a16 = A_BYTES >> 4, b16 = B_BYTES >> 4;
+        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
+          mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
+          tc_fence_after();
+          const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
+          uint32_t accum = 0;
+          const int split = tile / tiles_mn;
+          const int cc_lo = split * a.cps, cc_hi = min(a.c_chunks, cc_lo + a.cps);
+          int cc = cc_lo, rs = 0;
+          int kv = min(4, (C - cc * 64 + 15) >> 4);
+          const int ktot = (cc_hi - cc_lo) * RS;
+          for (int k = 0; k < ktot;) {
+            const int nk = min(kps, ktot - k);
             mbar_wait(full0 + 8 * st, ph);
             tc_fence_after();
-          }
-          if (lane == 0 && ks == 0 && j == 0) TRACE(3);
-          if (lane == 0 && j == 0) TRACE2(1, ks);
-          const bool el = elect_one();
-          for (int jj = 0; jj < nk && cc < cc_hi; ++jj, ++ks) {
-            const uint32_t a_addr = a.halo ? abase + aoff : sA0 + st * A_STAGE + jj * A_BYTES;
-            const uint64_t ad = umma_desc_sw128(a_addr, a.bo_mode);
-            const uint64_t bd = umma_desc_sw128(a.bres ? sB0 + (uint32_t)(cc * RS + rs) * B_BYTES
-                                                       : sB0 + st * B_STAGE + jj * B_BYTES);
-            if (el && !(a.dbg & 1)) {
-              // 4 x K=16 inside the 128-byte swizzle row; K=16 slices past the
-              // last real input channel are all zero (TMA fill) and skipped
-              const int kv = min(4, (a.C - cc * 64 + 15) >> 4);
-              mma_bf16(d, ad, bd, idesc, accum);
-              if (kv > 1) mma_bf16(d, ad + 2, bd + 2, idesc, 1u);
-              if (kv > 2) mma_bf16(d, ad + 4, bd + 4, idesc, 1u);
-              if (kv > 3) mma_bf16(d, ad + 6, bd + 6, idesc, 1u);
+            if (lane == 0 && k == 0 && j == 0 && tcount == 0) TRACE(3);
+            if (lane == 0 && j == 0) TRACE2(1, k);
+            const uint64_t a0 = aD0 + st * ast16, b0 = bD0 + st * bst16;
+            for (int jj = 0; jj < nk; ++jj) {
+              const uint64_t ad = a0 + (uint64_t)jj * a16, bd = b0 + (uint64_t)jj * b16;
+              // 4 x K=16 inside the 128-byte swizzle row; K=16 slices past
+              // the last real input channel are all zero and skipped
+              mma_bf16_on(d, ad, bd, idesc, accum, on);
+              if (kv > 1) mma_bf16_on(d, ad + 2, bd + 2, idesc, 1u, on);
+              if (kv > 2) mma_bf16_on(d, ad + 4, bd + 4, idesc, 1u, on);
+              if (kv > 3) mma_bf16_on(d, ad + 6, bd + 6, idesc, 1u, on);
+              accum = 1;
+              if (++rs == RS) { rs = 0; ++cc; kv = min(4, (C - cc * 64 + 15) >> 4); }
             }
-            accum = 1;
-            if (++s == a.S) { s = 0; aoff_r += row_r; aoff = aoff_r; } else { aoff += row_s; }
-            if (++rs == RS) {
-              rs = 0; s = 0; aoff_r = 0; aoff = 0;
-              ++cc;
-              if (a.halo) {
-                if (el) mma_commit(aempty0 + 8 * ab);
-                if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
-                break;  // a halo stage never crosses a chunk
-              }
-            }
+            k += nk;
+            mma_commit_on(empty0 + 8 * st, on);
+            if (++st == ST_) { st = 0; ph ^= 1u; }
           }
-          if (el && !a.bres) mma_commit(empty0 + 8 * st);
+          mma_commit_on(tfull0 + 8 * acc, on);
           __syncwarp();
-          if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
+          if (lane == 0 && tcount == 0 && j == 0) TRACE(4);
+          acc ^= 1u;
+          if (acc == 0) tph ^= 1u;
         }
-        if (a.bres && lane == 0 && j == 0) TRACE2(2, tcount);
-        if (elect_one()) mma_commit(tfull0 + 8 * acc);
-        __syncwarp();
-        if (lane == 0 && tcount == 0 && j == 0) TRACE(4);
-        acc ^= 1u;
-        if (acc == 0) tph ^= 1u;
       }
     }
     __syncwarp();
