@@ -356,9 +356,12 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
         const int p0 = tp * a.th, q0 = tq * a.tw, n0 = n_blk * a.n_tile;
         const int x0 = q0 * a.sw - a.pw, y0 = p0 * a.sh - a.ph;
-        const int cc_lo = split * a.cps, cc_hi = min(a.c_chunks, cc_lo + a.cps);
-        int cc = cc_lo, rs = 0, r = 0, s = 0;
-        while (cc < cc_hi) {
+        // split-K: this split's K-steps [k_lo, k_hi) (any (chunk, tap) boundary)
+        const int k_lo = split * a.kpsplit, k_hi = min(a.c_chunks * RS, k_lo + a.kpsplit);
+        int cc = k_lo / RS, rs = k_lo - (k_lo / RS) * RS;
+        int r = rs / a.S, s = rs - (rs / a.S) * a.S;
+        int k = k_lo;
+        while (k < k_hi) {
           if (a.halo && rs == 0 && warp == 0) {
             mbar_wait(aempty0 + 8 * ab, aph ^ 1u);
             if (elect_one()) {
@@ -375,16 +378,13 @@ __global__ void __launch_bounds__(kThreads, 1)
           // K-steps of this stage: up to KPS, never crossing a chunk in halo mode
           int nk = KPS;
           if (a.halo) nk = min(nk, RS - rs);
+          nk = min(nk, k_hi - k);
           if (mine == 0) {
             mbar_wait(empty0 + 8 * st, ph ^ 1u);
             if (elect_one()) {
               TRACE2(2, ks);
-              // count this stage's K-steps (tap mode may cross chunks)
-              int c2 = cc, rs2 = rs, r2 = r, s2 = s, cnt = 0;
-              for (int j = 0; j < nk && c2 < cc_hi; ++j) {
-                ++cnt;
-                if (++rs2 == RS) { rs2 = 0; ++c2; }
-              }
+              int c2, rs2, r2, s2;
+              const int cnt = nk;  // this stage's K-steps (tap mode may cross chunks)
               if (a.dbg & 2) {
                 mbar_arrive(full0 + 8 * st);
               } else {
@@ -408,10 +408,11 @@ __global__ void __launch_bounds__(kThreads, 1)
           --mine;
           if (++st == (uint32_t)ST) { st = 0; ph ^= 1u; }
           // advance by nk K-steps
-          for (int j = 0; j < nk && cc < cc_hi; ++j, ++ks) {
+          for (int j = 0; j < nk; ++j, ++ks) {
             if (++s == a.S) { s = 0; ++r; }
             if (++rs == RS) { rs = 0; r = 0; s = 0; ++cc; }
           }
+          k += nk;
         }
       }
     }
@@ -504,10 +505,10 @@ __global__ void __launch_bounds__(kThreads, 1)
           const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
           uint32_t accum = 0;
           const int split = tile / tiles_mn;
-          const int cc_lo = split * a.cps, cc_hi = min(a.c_chunks, cc_lo + a.cps);
-          int cc = cc_lo, rs = 0;
+          const int k_lo = split * a.kpsplit, k_hi = min(a.c_chunks * RS, k_lo + a.kpsplit);
+          int cc = k_lo / RS, rs = k_lo - (k_lo / RS) * RS;
           int kv = min(4, (C - cc * 64 + 15) >> 4);
-          const int ktot = (cc_hi - cc_lo) * RS;
+          const int ktot = k_hi - k_lo;
           for (int k = 0; k < ktot;) {
             const int nk = min(kps, ktot - k);
             mbar_wait(full0 + 8 * st, ph);

@@ -386,18 +386,27 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   }
   const int n_stage_steps = (KI + c.kps - 1) / c.kps;
   c.stages = std::max(2, std::min(c.stages, std::max(n_stage_steps, 2)));
-  // split-K (tap mode): a CTA's pipeline is latency-bound (~0.3 us per K-step,
-  // DESIGN.md §6), so deep layers with few output tiles split their
-  // 64-channel chunks across CTAs; fp32 partials are reduced by a finalize
-  // kernel that applies the folded BN + ReLU.
+  // split-K (tap mode): deep layers with few output tiles can split their
+  // K-steps across CTAs; fp32 partials are reduced by a finalize kernel that
+  // applies the folded BN + ReLU.
   c.ksplit = 1;
-  c.cps = c.c_chunks;
+  c.kpsplit = KI;
   const int tiles = c.tiles_m * c.tiles_n;
-  if (!c.halo && !getenv("HIOS_NOSPLIT") && tiles < 48 && c.c_chunks >= 2 && R * S * c.c_chunks >= 24) {
-    int want = std::min(c.c_chunks, std::max(1, (148 * c.occ + tiles - 1) / tiles));
-    want = std::min(want, std::max(1, R * S * c.c_chunks / 8));  // keep >= ~8 K-steps per split
-    c.cps = (c.c_chunks + want - 1) / want;
-    c.ksplit = (c.c_chunks + c.cps - 1) / c.cps;
+  // Measured (Inception-v3 1024, HIOS w=4, same box): split-K makes a deep
+  // small-spatial conv faster alone (7c_3x3 18.3 -> 14.5 us) but the step
+  // slower (0.865 -> 0.88-0.90 ms): the extra CTAs and the finalize launch
+  // crowd out the stage's concurrent ops.  So it is opt-in (HIOS_SPLITK=1).
+  if (!c.halo && getenv("HIOS_SPLITK") && tiles < 48 && KI >= 16) {
+    // at most one wave of CTAs, >= ~6 K-steps each; splits may start at any
+    // (chunk, tap) K-step
+    static const int cta_cap = getenv("HIOS_SPLIT_CTAS") ? atoi(getenv("HIOS_SPLIT_CTAS")) : 148;
+    static const int min_k = getenv("HIOS_SPLIT_MINK") ? std::max(1, atoi(getenv("HIOS_SPLIT_MINK"))) : 6;
+    int want = std::max(1, (cta_cap * c.occ) / tiles);
+    want = std::min(want, KI / min_k);
+    if (want >= 2) {
+      c.kpsplit = (KI + want - 1) / want;
+      c.ksplit = (KI + c.kpsplit - 1) / c.kpsplit;
+    }
   }
   if (getenv("HIOS_STAGES")) c.stages = std::max(2, atoi(getenv("HIOS_STAGES")));
   return c;

@@ -63,7 +63,7 @@ struct ConvTcArgs {
   int n_mma;                 // MMA warps splitting the N tile (n_tile % (16 * n_mma) == 0)
   int occ;                   // co-resident CTAs per SM the smem plan allows (1 or 2)
   int dbg;                   // debug switches (timing experiments; 0 in production)
-  int ksplit, cps;           // split-K: splits and 64-channel chunks per split
+  int ksplit, kpsplit;       // split-K: splits and K-steps (chunk x tap) per split
   int kps;                   // K-steps (64-channel x tap) per pipeline stage
   float* ws;                 // split-K fp32 workspace [ksplit][P*Q][ws_ld]
   size_t ws_split;           // elements per split

@@ -80,12 +80,20 @@ CONV_CASES = [
     (80, 192, 9, 252, 3, 3, 1, 0, 0),
     (96, 96, 7, 300, 1, 7, 1, 0, 3),
     (64, 80, 13, 100, 7, 1, 1, 3, 0),
+    # halo mode with resident weights (one N tile, > 148 output tiles per CTA wave)
+    (32, 32, 160, 200, 3, 3, 1, 1, 1),
+    (64, 80, 150, 130, 1, 1, 1, 0, 0),
+]
+
+SPLITK_CASES = [
+    (448, 384, 10, 10, 3, 3, 1, 1, 1),    # split boundaries inside a chunk's taps
+    (2048, 384, 8, 8, 1, 1, 1, 0, 0),
+    (288, 384, 35, 35, 3, 3, 2, 0, 0),
 ]
 
 
-@pytest.mark.parametrize("dtype", ["bf16", "f32"])
-@pytest.mark.parametrize("case", CONV_CASES)
-def test_conv_parity(dtype, case):
+def conv_case(dtype, case):
+    """(normwise error vs the oracle, kernels in the schedule's graph)."""
     C, K, H, Wd, kh, kw, s, ph, pw = case
     g = graphs.GraphSpec("conv", C, H, Wd)
     x0 = g.input()
@@ -94,7 +102,24 @@ def test_conv_parity(dtype, case):
     x = gen.make_input(g) - 0.5
     _, S, y = run_graph_gpu(g, W, x, dtype, profile=False)
     ref = infer.run_graph(g, W, x)[1]
-    assert nerr(y.reshape(ref.shape), ref) <= TOL[dtype] / (4 if dtype == "bf16" else 1)
+    return nerr(y.reshape(ref.shape), ref), hios().hios_kernel_count(S)
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+@pytest.mark.parametrize("case", CONV_CASES)
+def test_conv_parity(dtype, case):
+    err, _ = conv_case(dtype, case)
+    assert err <= TOL[dtype] / (4 if dtype == "bf16" else 1)
+
+
+@pytest.mark.parametrize("case", SPLITK_CASES)
+def test_conv_parity_splitk(case, monkeypatch):
+    """The opt-in split-K path (K-step-granular splits + finalize kernel)."""
+    _, n_plain = conv_case("bf16", case)
+    monkeypatch.setenv("HIOS_SPLITK", "1")
+    err, n_split = conv_case("bf16", case)
+    assert n_split == n_plain + 1  # the finalize kernel: split-K really ran
+    assert err <= TOL["bf16"] / 4
 
 
 @pytest.mark.parametrize("dtype", ["bf16", "f32"])
