@@ -487,11 +487,22 @@ def main():
     # single-GPU references measured in the same run (rank 0, N == 1 only)
     extra = {}
     if world == 1:
-        for name, (m_, w_) in {"sequential": (1, 1), "ios_style": (1, args.window),
+        for name, (m_, w_) in {"sequential": (1, 1), "ios_style": (1, args.window), "ios": (1, args.window),
                                "lp_inter_only": (M, 1), "hios_mr": (M, args.window)}.items():
             if name in ("lp_inter_only", "hios_mr") and M == 1:
                 continue
-            Sx = h.hios_schedule_mr(G, m_, w_) if name == "hios_mr" else h.hios_schedule_lp(G, m_, w_)
+            t_s0 = time.perf_counter()
+            try:
+                if name == "hios_mr":
+                    Sx = h.hios_schedule_mr(G, m_, w_)
+                elif name == "ios":  # exact single-GPU DP, t(S) profiled lazily
+                    Sx = h.hios_schedule_ios(G, w_)
+                else:
+                    Sx = h.hios_schedule_lp(G, m_, w_)
+            except h.HiosError as ex:
+                extra[name] = {"unavailable": str(ex)}
+                continue
+            t_sched_x = time.perf_counter() - t_s0
             if m_ > 1:
                 ndev = torch.cuda.device_count()
                 h.hios_schedule_place(Sx, [i % ndev for i in range(m_)])
@@ -500,7 +511,8 @@ def main():
             tx = timed_loop(Sx, args.steps)
             extra[name] = {"ms": float(np.mean(tx)),
                            "predicted_ms": h.hios_schedule_latency_ns(Sx) / 1e6,
-                           "gpus_used": int(len(set(h.hios_schedule_stages(Sx)[0].tolist())))}
+                           "gpus_used": int(len(set(h.hios_schedule_stages(Sx)[0].tolist()))),
+                           "schedule_s": t_sched_x}
             del Sx
 
     sweep = {}
@@ -570,6 +582,8 @@ def main():
             line["speedup_vs_sequential"] = extra["sequential"]["ms"] / ms
         if "ios_style" in extra:
             line["speedup_vs_ios_style"] = extra["ios_style"]["ms"] / ms
+        if "ms" in extra.get("ios", {}):
+            line["speedup_vs_ios"] = extra["ios"]["ms"] / ms
         print(json.dumps(line))
     if world > 1:
         dist.barrier()

@@ -174,6 +174,19 @@ hios_status hios_schedule_lp(hios_graph g, int32_t n_gpus, int32_t window, hios_
  * "MR-based inter-GPU" only. */
 hios_status hios_schedule_mr(hios_graph g, int32_t n_gpus, int32_t window, hios_schedule* out);
 
+/* IOS, the paper's single-GPU comparator (P:158, P:254, P:316 -- "an exact
+ * algorithm for the optimal schedule in a single GPU", dynamic programming):
+ * on one GPU, the sequence of stages of <= window pairwise-independent ops
+ * minimising L = sum t(S).  Exact DP over finished-op sets, decomposed at cut
+ * vertices (ops comparable with every other op); a block of more than 32 ops
+ * is cut into topological-order chunks (as IOS partitions large graphs; exact
+ * per chunk -- Inception-v3, SqueezeNet, RandWire need no cut).  t(S)
+ * as for hios_schedule_lp (measured lazily after hios_profile, injected, or
+ * the group model).  max_states bounds the DP (<= 0: 2^22).  Writes *out
+ * (caller owns).  Errors: HIOS_E_INVALID, HIOS_E_STATE, HIOS_E_UNSUPPORTED
+ * (state budget exceeded), HIOS_E_CUDA. */
+hios_status hios_schedule_ios(hios_graph g, int32_t window, int64_t max_states, hios_schedule* out);
+
 /* Import a schedule: op_gpu[v] in [0, n_gpus), op_stage[v] = stage index on
  * that GPU (stages numbered 0..K_i-1; ops sharing an index form one stage).
  * Checked for feasibility (C6): HIOS_E_INVALID (dependent ops in a stage,

@@ -546,3 +546,48 @@ def hios_mr(n, t, edges, M, w, gcost):
     reach = reachability(n, edges)
     Q, L = parallelize(n, t, edges, Q, w, gcost, order, reach)  # L27
     return Q, L, gpu
+
+
+# ------------------------------------- exact single-GPU optimum ("IOS")
+def ios_dp(n, t, edges, w, gcost):
+    """The IOS comparator ("an exact algorithm for the
+    optimal schedule in a single GPU", dynamic programming): on one GPU, the
+    sequence of stages -- sets of <= w pairwise-independent ops whose inputs
+    are all produced by earlier stages -- minimising L = sum t(S) (P:86-100 at
+    M = 1).  Plain DP over the set D of finished ops (always downward closed):
+        f(V) = 0,  f(D) = min over E of t(E) + f(D | E),
+    E ranging over the independent subsets of ready(D) of size 1..w,
+    enumerated in itertools.combinations order of the ready ops sorted by id,
+    sizes ascending, first strict minimum kept.  Exponential; for small
+    graphs.  Returns (Q, L) with Q = [[stage, ...]] on GPU 0."""
+    reach = reachability(n, edges)
+    _, preds = succ_lists(n, edges)
+    pset = [set(u for (u, _) in preds[v]) for v in range(n)]
+    full = frozenset(range(n))
+    memo: Dict[frozenset, Tuple[int, Optional[tuple]]] = {full: (0, None)}
+
+    def cost(E):
+        return t[E[0]] if len(E) == 1 else gcost(frozenset(E))
+
+    def f(D: frozenset):
+        if D in memo:
+            return memo[D][0]
+        ready = sorted(v for v in range(n) if v not in D and pset[v] <= D)
+        best, arg = INF, None
+        for k in range(1, min(w, len(ready)) + 1):
+            for E in itertools.combinations(ready, k):
+                if any(not independent(a, b, reach) for a, b in itertools.combinations(E, 2)):
+                    continue
+                c = cost(E) + f(D | frozenset(E))
+                if c < best:
+                    best, arg = c, E
+        memo[D] = (best, arg)
+        return best
+
+    L = f(frozenset())
+    stages, D = [], frozenset()
+    while D != full:
+        E = memo[D][1]
+        stages.append(tuple(E))
+        D = D | frozenset(E)
+    return [stages], L

@@ -169,6 +169,21 @@ hios_status hios_schedule_mr(hios_graph g, int32_t n_gpus, int32_t window, hios_
   });
 }
 
+hios_status hios_schedule_ios(hios_graph g, int32_t window, int64_t max_states, hios_schedule* out) {
+  if (out) *out = nullptr;
+  return guard([&] {
+    NEED(g && out, HIOS_E_INVALID, "NULL argument");
+    NEED(window >= 1 && window <= 8, HIOS_E_INVALID, "window out of [1, 8]");
+    std::unique_ptr<hios::Schedule> s(new hios::Schedule);
+    s->g = g->g;
+    hios::hios_ios(*g->g, window, *s, max_states > 0 ? max_states : (int64_t)1 << 22);
+    hios::finalize_schedule(*s);
+    auto* h = new hios_schedule_s;
+    h->s = std::move(s);
+    *out = h;
+  });
+}
+
 hios_status hios_schedule_import(hios_graph g, int32_t n_gpus, int32_t window, const int32_t* op_gpu,
                                  const int32_t* op_stage, hios_schedule* out) {
   if (out) *out = nullptr;

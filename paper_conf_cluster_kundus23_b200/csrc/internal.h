@@ -98,6 +98,7 @@ struct SimResult { bool ok; int64_t L; std::vector<std::vector<int64_t>> start, 
 SimResult simulate(Graph& g, const std::vector<std::vector<std::vector<int>>>& Q);
 void hios_lp(Graph& g, int M, int w, Schedule& s);
 void hios_mr(Graph& g, int M, int w, Schedule& s);
+void hios_ios(Graph& g, int w, Schedule& s, int64_t max_states);
 void finalize_schedule(Schedule& s);  // gpu_of/stage_of + validation (C6)
 
 }  // namespace hios

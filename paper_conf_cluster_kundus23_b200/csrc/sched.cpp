@@ -13,6 +13,8 @@
 #include <algorithm>
 #include <limits>
 
+#include <functional>
+#include <unordered_map>
 #include "internal.h"
 
 namespace hios {
@@ -322,6 +324,124 @@ void hios_mr(Graph& g, int M, int w, Schedule& s) {
   s.Q.assign(M, {});
   for (int v : order) s.Q[gpu[v]].push_back({v});
   parallelize(g, s, order);  // L27
+}
+
+// ------------------------------------------------ IOS (exact, one GPU)
+// The paper's single-GPU comparator ("an exact
+// algorithm for the optimal schedule in a single GPU", dynamic programming):
+// the stage sequence (stages = <= w pairwise-independent ready ops) that
+// minimises L = sum t(S).  DP over the finished set D:
+//   f(V) = 0,  f(D) = min_E t(E) + f(D | E).
+// Exact decomposition at cut vertices (ops comparable with every other op:
+// such an op is always a stage of its own and splits G into independent
+// sub-problems), then a memoised DP per block (bitmasks).  Blocks of more
+// than 32 ops are cut into topological-order chunks (exact per chunk).
+// Enumeration: ready ops ascending, subsets in combinations order, sizes
+// ascending, first strict minimum -- as oracle/sched.py: ios_dp.
+void hios_ios(Graph& g, int w, Schedule& s, int64_t max_states) {
+  s.M = 1;
+  s.w = w;
+  const int n = g.n;
+  // cut vertices
+  std::vector<int> before(n, 0), after(n, 0);
+  for (int u = 0; u < n; ++u)
+    for (int v = 0; v < n; ++v)
+      if (g.reaches(u, v)) { ++after[u]; ++before[v]; }
+  std::vector<char> cut(n, 0);
+  for (int v = 0; v < n; ++v) cut[v] = before[v] + after[v] == n - 1;
+  // block of a non-cut op = number of cut vertices before it
+  std::vector<int> cuts;
+  for (int v : g.topo) if (cut[v]) cuts.push_back(v);
+  std::vector<std::vector<int>> blocks(cuts.size() + 1);
+  for (int v : g.topo) {
+    if (cut[v]) continue;
+    int b = 0;
+    for (int c : cuts) b += g.reaches(c, v) ? 1 : 0;
+    blocks[b].push_back(v);
+  }
+  std::vector<std::vector<int>> stages;
+  int64_t states = 0;
+  auto solve_block = [&](std::vector<int> ops) {
+    if (ops.empty()) return;
+    std::sort(ops.begin(), ops.end());
+    const int m = (int)ops.size();
+    std::vector<uint64_t> pred_mask(m, 0), indep(m, 0);
+    for (int i = 0; i < m; ++i)
+      for (int j = 0; j < m; ++j) {
+        if (g.reaches(ops[j], ops[i])) {
+          // only direct preds matter for readiness, but any ancestor in the
+          // block being finished first is implied by downward closure
+          pred_mask[i] |= 1ull << j;
+        }
+        if (g.independent(ops[i], ops[j])) indep[i] |= 1ull << j;
+      }
+    const uint64_t full = m == 64 ? ~0ull : ((1ull << m) - 1);
+    std::unordered_map<uint64_t, std::pair<int64_t, uint64_t>> memo;
+    memo[full] = {0, 0};
+    std::function<int64_t(uint64_t)> f = [&](uint64_t D) -> int64_t {
+      auto it = memo.find(D);
+      if (it != memo.end()) return it->second.first;
+      if (++states > max_states) fail(HIOS_E_UNSUPPORTED, "IOS DP: state budget exceeded");
+      int ready[64];
+      int r = 0;
+      for (int i = 0; i < m; ++i)
+        if (!((D >> i) & 1) && (pred_mask[i] & ~D) == 0) ready[r++] = i;
+      int64_t best = std::numeric_limits<int64_t>::max();
+      uint64_t arg = 0;
+      int idx[8];
+      for (int k = 1; k <= std::min(w, r); ++k) {
+        for (int q = 0; q < k; ++q) idx[q] = q;
+        while (true) {
+          bool ok = true;
+          uint64_t E = 0;
+          for (int q = 0; q < k && ok; ++q) {
+            const int a = ready[idx[q]];
+            for (int q2 = 0; q2 < q; ++q2)
+              if (!((indep[a] >> ready[idx[q2]]) & 1)) { ok = false; break; }
+            E |= 1ull << a;
+          }
+          if (ok) {
+            std::vector<int> S;
+            for (int q = 0; q < k; ++q) S.push_back(ops[ready[idx[q]]]);
+            const int64_t c = g.stage_cost(S) + f(D | E);
+            if (c < best) { best = c; arg = E; }
+          }
+          // next combination (lexicographic)
+          int q = k - 1;
+          while (q >= 0 && idx[q] == r - k + q) --q;
+          if (q < 0) break;
+          ++idx[q];
+          for (int q2 = q + 1; q2 < k; ++q2) idx[q2] = idx[q2 - 1] + 1;
+        }
+      }
+      memo[D] = {best, arg};
+      return best;
+    };
+    f(0);
+    uint64_t D = 0;
+    while (D != full) {
+      const uint64_t E = memo[D].second;
+      std::vector<int> S;
+      for (int i = 0; i < m; ++i)
+        if ((E >> i) & 1) S.push_back(ops[i]);
+      stages.push_back(S);
+      D |= E;
+    }
+  };
+  // blocks of more than `chunk` ops (no cut vertex inside, e.g. NASNet's
+  // two-input cells) are cut into consecutive topological-order chunks, as
+  // IOS itself partitions large graphs; the DP is then exact per chunk
+  const int chunk = 32;
+  auto solve = [&](const std::vector<int>& ops) {  // ops in topological order
+    for (size_t i = 0; i < ops.size(); i += chunk)
+      solve_block(std::vector<int>(ops.begin() + i, ops.begin() + std::min(ops.size(), i + chunk)));
+  };
+  solve(blocks[0]);
+  for (size_t c = 0; c < cuts.size(); ++c) {
+    stages.push_back({cuts[c]});
+    solve(blocks[c + 1]);
+  }
+  s.Q.assign(1, stages);
 }
 
 void finalize_schedule(Schedule& s) {

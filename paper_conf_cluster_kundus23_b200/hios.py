@@ -66,6 +66,7 @@ def load() -> C.CDLL:
         "hios_schedule_lp": [VP, I32, I32, P(VP)],
         "hios_schedule_import": [VP, I32, I32, P(I32), P(I32), P(VP)],
         "hios_schedule_mr": [VP, I32, I32, P(VP)],
+        "hios_schedule_ios": [VP, I32, I64, P(VP)],
         "hios_schedule_latency_ns": [VP, P(I64)],
         "hios_schedule_stages": [VP, P(I32), P(I32), P(I32)],
         "hios_schedule_place": [VP, P(I32), I32],
@@ -248,6 +249,12 @@ def hios_schedule_mr(g: Graph, n_gpus: int, window: int) -> Schedule:
     h = C.c_void_p()
     _ck(load().hios_schedule_mr(g.h, n_gpus, window, C.byref(h)))
     return Schedule(h, g, n_gpus)
+
+
+def hios_schedule_ios(g: Graph, window: int, max_states: int = 0) -> Schedule:
+    h = C.c_void_p()
+    _ck(load().hios_schedule_ios(g.h, window, int(max_states), C.byref(h)))
+    return Schedule(h, g, 1)
 
 
 def hios_schedule_import(g: Graph, n_gpus: int, window: int, op_gpu, op_stage) -> Schedule:

@@ -270,3 +270,33 @@ def test_group_cost_sources():
     for bad in ([1, 1], [N + 5], []):
         with pytest.raises(hios.HiosError):
             hios.hios_group_cost(G, bad)
+
+
+@pytest.mark.parametrize("w", [1, 2, 3])
+def test_ios_latency_equals_oracle_dp(w):
+    """hios_schedule_ios (C++ DP, cut-vertex decomposition) reaches the same
+    optimum L as the oracle's plain DP (ties may pick different stages, so
+    the schedule is checked for feasibility, not equality)."""
+    rng = random.Random(70 + w)
+    for _ in range(30):
+        n, t, E = S.random_dag(rng.randint(2, 9), rng.randint(2, 4), None, 0.8, rng.randint(0, 10**6), unit=1000)
+        G, N, t_all, E_all = _cost_graph(n, t, E)
+        hios.hios_set_group_model(G, 7, 10)
+        s = hios.hios_schedule_ios(G, w)
+        Qo, Lo = S.ios_dp(N, t_all, E_all, w, S.group_model(t_all))
+        assert hios.hios_schedule_latency_ns(s) == Lo
+        Q = hios.stages_to_Q(s)
+        assert S.validate(N, t_all, E_all, Q, w, S.group_model(t_all)) is None
+
+
+def test_ios_on_benchmark_dags_not_worse_than_hios_m1():
+    for name, size in [("inception_v3", 299), ("squeezenet", 224), ("randwire_ws", 224)]:
+        g = graphs.build(name, size)
+        G = hios.hios_graph_create(g.ops, g.edges, g.in_c, g.in_h, g.in_w, "bf16", gen.make_weights(g))
+        for op in g.ops:
+            hios.hios_set_op_cost(G, op.id, 1000 + (37 * op.id) % 500)
+        for e in range(g.n_edges):
+            hios.hios_set_edge_cost(G, e, 100)
+        hios.hios_set_group_model(G, 7, 10)
+        L_ios = hios.hios_schedule_latency_ns(hios.hios_schedule_ios(G, 4))
+        assert L_ios <= hios.hios_schedule_latency_ns(hios.hios_schedule_lp(G, 1, 4))

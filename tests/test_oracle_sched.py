@@ -290,3 +290,39 @@ def test_mr_feasible_and_not_below_optimum(w):
         assert S.validate(n, t, E, Q, w, g) is None
         assert S.simulate(n, t, E, Q, g)[0] == L
         assert S.brute_force(n, t, E, 2, w, g)[0] <= L
+
+
+# ------------------------------------- IOS comparator (exact, one GPU)
+@pytest.mark.parametrize("w", [1, 2, 3])
+def test_ios_dp_is_the_single_gpu_optimum(w):
+    """P:316 'IOS is an exact algorithm for the optimal schedule in a single
+    GPU': the DP equals the brute-force optimum at M = 1, is feasible, and is
+    never worse than HIOS-LP at M = 1 (a heuristic over the same space)."""
+    rng = random.Random(31 + w)
+    for _ in range(40):
+        n, t, E = S.random_dag(rng.randint(2, 8), rng.randint(2, 4), None,
+                               rng.choice([0.4, 0.8, 1.2]), rng.randint(0, 10**6), unit=10)
+        g = S.group_model(t)
+        Q, L = S.ios_dp(n, t, E, w, g)
+        assert L == S.brute_force(n, t, E, 1, w, g)[0]
+        assert S.validate(n, t, E, Q, w, g) is None
+        assert S.simulate(n, t, E, Q, g)[0] == L
+        assert L <= S.hios_lp(n, t, E, 1, w, g)[1]
+        if w == 1:
+            assert L == sum(t)
+
+
+def test_ios_dp_fig5_single_gpu():
+    """Fig. 5's graph and group-cost table (pairs the table does not
+    list take the C12 model) on one GPU with w = 2: the DP's optimum equals
+    brute force and beats running the ops one by one."""
+    d = load("fig5_alg2.json")
+    n, t, E = d["n"], d["t"], edges_of(d)
+    tab = {frozenset(s): c for s, c in d["group_costs"]}
+    model = S.group_model(t)
+
+    def g(Sg):
+        return tab.get(frozenset(Sg), model(Sg))
+    Q, L = S.ios_dp(n, t, E, 2, g)
+    assert L == S.brute_force(n, t, E, 1, 2, g)[0]
+    assert L < sum(t)
