@@ -294,6 +294,64 @@ def max_over_ranks(dist, x, world):
     return float(t.item())
 
 
+# ------------------------------------------------------------ workload sweep
+def measure_workload(h, torch, model, sz, M, args, dev, stream, flush, pk, esz):
+    """One more BASELINE.json workload (another size or another benchmark DAG)
+    in the same run: profile, then HIOS-LP (M, w), sequential (1, 1) and the
+    IOS-style stand-in (1, w), each timed like the main line (device events,
+    L2 flushed between steps), plus the schedule's critical-path bound."""
+    from workloads import gen, graphs
+    gs = graphs.build(model, sz)
+    Ws = gen.make_weights(gs)
+    xs = gen.make_input(gs)
+    Gs = h.hios_graph_create(gs.ops, gs.edges, gs.in_c, gs.in_h, gs.in_w, args.dtype, Ws)
+    shp = {o.id: h.hios_graph_shape(Gs, o.id) for o in gs.ops}
+    t0 = time.perf_counter()
+    h.hios_profile(Gs, [dev], 5)
+    row = {"input": f"1x{gs.in_c}x{sz}x{sz}", "ops": gs.n_ops, "deps": gs.n_edges,
+           "profile_s": time.perf_counter() - t0}
+    din = torch.from_numpy(xs).to(f"cuda:{dev}")
+    dout = None
+    for name, (m_, w_) in {"hios_lp": (M, args.window), "sequential": (1, 1),
+                           "ios_style": (1, args.window)}.items():
+        t0 = time.perf_counter()
+        Sx = h.hios_schedule_lp(Gs, m_, w_)
+        t_s = time.perf_counter() - t0
+        if m_ > 1:
+            ndev = torch.cuda.device_count()
+            h.hios_schedule_place(Sx, [i % ndev for i in range(m_)])
+        if dout is None:
+            dout = torch.empty(h.hios_output_numel(Sx), dtype=torch.float32, device=f"cuda:{dev}")
+        for _ in range(3):
+            h.hios_run_device(Sx, din.data_ptr(), dout.data_ptr(), stream.cuda_stream)
+        ev = []
+        for i in range(max(5, args.steps // 3)):
+            flush.fill_(float(i))
+            a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a_.record(stream)
+            h.hios_run_device(Sx, din.data_ptr(), dout.data_ptr(), stream.cuda_stream)
+            b_.record(stream)
+            ev.append((a_, b_))
+        torch.cuda.synchronize()
+        row[name + "_ms"] = float(np.mean([a_.elapsed_time(b_) for a_, b_ in ev]))
+        row[name + "_predicted_ms"] = h.hios_schedule_latency_ns(Sx) / 1e6
+        if name == "hios_lp":
+            og, ost, _ = h.hios_schedule_stages(Sx)
+            Fs, Bs = op_work(gs, shp, esz)
+            row["cp_bound_ms"] = critical_path_bound(gs, Fs, Bs, og, ost, M, pk, esz, shp) * 1e3
+            row["seq_roofline_ms"] = float(np.maximum(Fs / (pk["bf16_tflops"] * 1e12),
+                                                      Bs / (pk["hbm_gbs"] * 1e9)).sum() * 1e3)
+            row["gflop"] = float(Fs.sum() / 1e9)
+            row["gpus_used"] = int(len(set(og.tolist())))
+            row["schedule_s"] = t_s
+        del Sx
+    row["cp_frac"] = row["cp_bound_ms"] / row["hios_lp_ms"]
+    row["speedup_vs_sequential"] = row["sequential_ms"] / row["hios_lp_ms"]
+    row["speedup_vs_ios_style"] = row["ios_style_ms"] / row["hios_lp_ms"]
+    del Gs
+    return row
+
+
 # ------------------------------------------------------------ main
 def main():
     ap = argparse.ArgumentParser()
@@ -307,7 +365,7 @@ def main():
     ap.add_argument("--impl", default="hios", choices=["hios", "reference"])
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--sweep", default="2048,4096",
+    ap.add_argument("--sweep", default="2048,4096,randwire_ws@2048,nasnet_a_large@2048,squeezenet@2048",
                     help="extra input sizes timed on 1 GPU (HIOS-LP / sequential / IOS-style), '' to skip")
     ap.add_argument("--logical", type=int, default=0,
                     help="single process: schedule over this many logical GPUs (aliased on visible devices)")
@@ -517,40 +575,13 @@ def main():
 
     sweep = {}
     if world == 1 and args.sweep and not os.environ.get("HIOS_NCU"):
-        for sz in [int(v) for v in args.sweep.split(",") if v]:
-            gs = graphs.build(args.model, sz)
-            Ws = gen.make_weights(gs)
-            xs = gen.make_input(gs)
-            Gs = h.hios_graph_create(gs.ops, gs.edges, gs.in_c, gs.in_h, gs.in_w, args.dtype, Ws)
-            shp = {o.id: h.hios_graph_shape(Gs, o.id) for o in gs.ops}
-            h.hios_profile(Gs, [dev], 5)
-            din = torch.from_numpy(xs).to(f"cuda:{dev}")
-            dout = torch.empty(h.hios_output_numel(h.hios_schedule_lp(Gs, 1, 1)), dtype=torch.float32,
-                               device=f"cuda:{dev}")
-            row = {"input": f"1x{gs.in_c}x{sz}x{sz}"}
-            for name, (m_, w_) in {"hios_lp": (M, args.window), "sequential": (1, 1),
-                                   "ios_style": (1, args.window)}.items():
-                Sx = h.hios_schedule_lp(Gs, m_, w_)
-                for _ in range(3):
-                    h.hios_run_device(Sx, din.data_ptr(), dout.data_ptr(), stream.cuda_stream)
-                ev = []
-                for i in range(max(5, args.steps // 3)):
-                    flush.fill_(float(i))
-                    a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                    a_.record(stream)
-                    h.hios_run_device(Sx, din.data_ptr(), dout.data_ptr(), stream.cuda_stream)
-                    b_.record(stream)
-                    ev.append((a_, b_))
-                torch.cuda.synchronize()
-                row[name + "_ms"] = float(np.mean([a_.elapsed_time(b_) for a_, b_ in ev]))
-                if name == "hios_lp":
-                    og, ost, _ = h.hios_schedule_stages(Sx)
-                    Fs, Bs = op_work(gs, shp, esz)
-                    row["cp_bound_ms"] = critical_path_bound(gs, Fs, Bs, og, ost, M, pk, esz, shp) * 1e3
-                del Sx
-            row["cp_frac"] = row["cp_bound_ms"] / row["hios_lp_ms"]
-            sweep[str(sz)] = row
-            del Gs
+        for item in [v for v in args.sweep.split(",") if v]:
+            model, sz = (item.split("@") if "@" in item else (args.model, item))
+            try:
+                sweep[f"{model}@{sz}"] = measure_workload(h, torch, model, int(sz), M, args, dev, stream,
+                                                          flush, pk, esz)
+            except Exception as ex:  # noqa: BLE001 -- reported, never silently dropped
+                sweep[f"{model}@{sz}"] = {"error": f"{type(ex).__name__}: {ex}"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
