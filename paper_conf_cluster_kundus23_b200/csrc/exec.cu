@@ -23,6 +23,20 @@
 
 namespace hios {
 
+// Stride-2 stems with <= 4 input channels on the tensor-core path (bf16):
+// space-to-depth turns conv(R x S, stride 2, pad p) over C channels into
+// conv(ceil(R/2) x ceil(S/2), stride 1, pad 0) over 4C channels of
+//   X'[i][j][(a*2+b)*C + c] = X[2i+a-p][2j+b-p][c]      (zero outside X),
+// with W'[k][r'][s'][(a*2+b)*C + c] = W[k][c][2r'+a][2s'+b] (zero past R, S).
+// Every product of the original sum appears exactly once; K per tap is one
+// K=16 MMA slice (4C <= 16) instead of a 64-channel chunk that is 95 % zero,
+// and stride 1 lets the conv run in halo mode.
+static bool s2d_conv(const Op& o) {
+  return o.kind == HIOS_OP_CONV && o.in_c <= 4 && o.sh == 2 && o.sw == 2 && o.dh == 1 && o.dw == 1 &&
+         o.kh * o.kw >= 4 && !getenv("HIOS_NOS2D");
+}
+
+
 void ck(cudaError_t e, const char* what) {
   if (e != cudaSuccess) fail(HIOS_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
 }
@@ -121,6 +135,11 @@ void Executor::plan() {
   for (int v = 0; v < n; ++v) {
     const Op& o = g.ops[v];
     const int l = s.gpu_of[v];
+    if (o.kind == HIOS_OP_CONV && g.dtype == HIOS_BF16 && s2d_conv(o)) {
+      OpExec& x = ox[v];
+      x.s2d_ldc = rup(4 * o.in_c, 8);
+      x.s2dbuf = alloc(l, (int64_t)(o.H + (o.kh + 1) / 2 - 1) * (o.W + (o.kw + 1) / 2 - 1) * x.s2d_ldc * esz);
+    }
     if (o.kind == HIOS_OP_SEPCONV) {
       OpExec& x = ox[v];
       x.dw_ldc = rup(std::max(o.in_c, o.out_c), 8);
@@ -182,6 +201,7 @@ static std::vector<T> conv_layout(const float* W, int K, int C, int R, int S, in
 }
 
 // stems (C <= 8, receptive field <= 49 taps, weights fit in smem): direct CUDA-core kernel
+// (the fp32 path; the bf16 path takes s2d_conv first)
 static bool small_c_conv(const Op& o) {
   return o.in_c <= 8 && o.kh * o.kw <= 49 && (size_t)o.out_c * o.kh * o.kw * o.in_c * 4 <= 96 * 1024 && o.dh == 1 &&
          o.dw == 1;
@@ -196,6 +216,23 @@ static void upload_weights_T(Executor& ex, int v) {
   switch (o.kind) {
     case HIOS_OP_CONV: {
       const int Cp = tc ? rup(o.in_c, 8) : o.in_c;
+      if (tc && s2d_conv(o)) {
+        // W'[k][r'*S'+s'][(a*2+b)*C + c] (see s2d_conv)
+        const int R2 = (o.kh + 1) / 2, S2 = (o.kw + 1) / 2, C = o.in_c, Cp2 = rup(4 * C, 8);
+        std::vector<T> w2((size_t)o.out_c * R2 * S2 * Cp2, to_dev_t<T>(0.f));
+        for (int k = 0; k < o.out_c; ++k)
+          for (int c = 0; c < C; ++c)
+            for (int r = 0; r < o.kh; ++r)
+              for (int s2 = 0; s2 < o.kw; ++s2) {
+                const int ch = ((r & 1) * 2 + (s2 & 1)) * C + c;
+                w2[((size_t)k * R2 * S2 + (r >> 1) * S2 + (s2 >> 1)) * Cp2 + ch] =
+                    to_dev_t<T>(o.weight[(((size_t)k * C + c) * o.kh + r) * o.kw + s2]);
+              }
+        x.w = upload(L, w2);
+        x.scale.push_back((float*)upload(L, o.scale));
+        x.shift.push_back((float*)upload(L, o.shift));
+        break;
+      }
       x.w = upload(L, conv_layout<T>(o.weight.data(), o.out_c, o.in_c, o.kh, o.kw, Cp));
       if (small_c_conv(o)) x.w_small = (float*)upload(L, conv_layout<float>(o.weight.data(), o.out_c, o.in_c, o.kh, o.kw, o.in_c));
       x.scale.push_back((float*)upload(L, o.scale));
@@ -529,6 +566,18 @@ static void build_op(Executor& ex, int v) {
     case HIOS_OP_CONV: {
       const int u = in_op(0);
       const Op& xi = g.ops[u];
+      if (x.s2dbuf >= 0) {
+        View iv = view_of(u, l);
+        const int R2 = (o.kh + 1) / 2, S2 = (o.kw + 1) / 2;
+        const int H2 = o.H + R2 - 1, W2 = o.W + S2 - 1;
+        View sv{ex.ptr(l, x.s2dbuf), x.s2d_ldc};
+        S2dArgs<T> d{(const T*)iv.p, xi.H, xi.W, xi.C, iv.ldc, o.ph, o.pw, (T*)sv.p, H2, W2, sv.ldc};
+        fns.push_back([d](cudaStream_t st) { launch_s2d<T>(d, st); });
+        ++nk;
+        fns.push_back(conv_closure<T>(ex, sv, H2, W2, 4 * xi.C, x.w, x.scale[0], x.shift[0], o.out_c, R2, S2, 1, 1,
+                                      0, 0, 1, 1, o.H, o.W, o.relu, out, out2, nk));
+        break;
+      }
       if (small_c_conv(o)) {
         View iv = view_of(u, l);
         ConvSmallArgs<T> c{};

@@ -25,6 +25,9 @@ struct OpExec {
   // sepconv scratch (arena offsets)
   int64_t dwbuf = -1, midbuf = -1;
   int dw_ldc = 0, mid_ldc = 0;
+  // stride-2 small-C stem (bf16): space-to-depth copy of the input (arena offset)
+  int64_t s2dbuf = -1;
+  int s2d_ldc = 0;
   // remote deliveries of this op's output: (consumer lgpu, fused-into-epilogue?)
   std::vector<std::pair<int, bool>> remote;
   std::function<void(cudaStream_t)> run;  // enqueue the op's kernels (incl. fused out2)

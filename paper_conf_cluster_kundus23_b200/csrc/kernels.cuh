@@ -122,6 +122,13 @@ struct ConvSmallArgs {
   T* out; int ldo; T* out2; int ldo2;
 };
 
+// space-to-depth of a stride-2 small-C stem input (exec.cu: s2d_conv)
+template <typename T>
+struct S2dArgs {
+  const T* x; int H, W, C, ldx, ph, pw;
+  T* out; int P2, Q2, ldo;  // X' is P2 x Q2 x 4C (pixel stride ldo)
+};
+
 template <typename T>
 struct CopyArgs {
   const T* x; int ldx; int HW, C; T* out; int ldo;
@@ -141,6 +148,7 @@ template <typename T> void launch_dw(const DwArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_pool(const PoolArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_add(const AddArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_copy(const CopyArgs<T>& a, cudaStream_t st);
+template <typename T> void launch_s2d(const S2dArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_gap(const T* x, int HW, int C, int ldx, T* out, cudaStream_t st);
 template <typename T> void launch_linear(const T* x, int Cin, const T* w, int ldw, const float* b, int K,
                                          T* out, cudaStream_t st);

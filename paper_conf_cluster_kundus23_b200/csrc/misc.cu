@@ -46,6 +46,19 @@ __device__ __forceinline__ void store_vec(T* p, int c, int C, const float* v) {
   }
 }
 
+// 8 channels (one 16-byte bf16 vector, two 16-byte fp32 vectors)
+template <typename T>
+__device__ __forceinline__ void load8(const T* p, int c, int C, float* v) {
+#pragma unroll
+  for (int h = 0; h < 8; h += Vec<T>::N) load_vec(p + h, c + h, C, v + h);
+}
+template <typename T>
+__device__ __forceinline__ void store8(T* p, int c, int C, const float* v) {
+#pragma unroll
+  for (int h = 0; h < 8; h += Vec<T>::N)
+    if (c + h < C) store_vec(p + h, c + h, C, v + h);
+}
+
 static inline unsigned grid_for(long long n, int block) {
   long long g = (n + block - 1) / block;
   return (unsigned)(g < 1 ? 1 : g);
@@ -100,9 +113,111 @@ __global__ void pool_kernel(const PoolArgs<T> a) {
   if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
 }
 
+// Tiled pooling (same tiling as the depthwise kernel below): a CTA stages
+// the input window of 8 output rows x 32 output columns x 16 channels once in
+// smem (out-of-bounds = -inf for max, 0 for average; columns de-interleaved by
+// parity when sw == 2), then each thread reduces its two output pixels' k x k
+// windows from smem.  The average divisor is computed from the window bounds
+// (count_include_pad or in-bounds count), as in pool_kernel.
+constexpr int kPoolTP = 8, kPoolTQ = 32;
+
+template <typename T, int KS>
+__global__ void __launch_bounds__(256) pool_tiled_kernel(const PoolArgs<T> a) {
+  extern __shared__ __align__(16) uint8_t psm[];
+  constexpr int N = 8;
+  constexpr int VB = N * (int)sizeof(T);
+  const int kh = KS > 0 ? KS : a.kh, kw = KS > 0 ? KS : a.kw;
+  const int IH = (kPoolTP - 1) * a.sh + kh, IW = (kPoolTQ - 1) * a.sw + kw;
+  const int half = (IW + 1) / 2;
+  // channel slab fastest in the grid: the CTAs of one spatial tile run together
+  // and between them read whole pixel rows (DRAM page locality)
+  const int q0 = blockIdx.y * kPoolTQ, p0 = blockIdx.z * kPoolTP, c0 = blockIdx.x * 16;
+  pdl_enter();
+  const int hb = p0 * a.sh - a.ph, wb = q0 * a.sw - a.pw;
+  const float pad = a.is_max ? -INFINITY : 0.f;
+  const int nel = 2 * IH * IW;
+  for (int e = threadIdx.x; e < nel; e += blockDim.x) {
+    const int cv = e & 1, pix = e >> 1;
+    const int row = pix / IW, col = pix - row * IW;
+    const int h = hb + row, w = wb + col, c = c0 + cv * N;
+    float v[N];
+    if (h >= 0 && h < a.H && w >= 0 && w < a.W && c < a.C) {
+      load8(a.x + ((size_t)h * a.W + w) * a.ldx + c, c, a.C, v);
+    } else {
+#pragma unroll
+      for (int j = 0; j < N; ++j) v[j] = pad;
+    }
+    const int pos = a.sw == 2 ? ((col & 1) * half + (col >> 1)) : col;
+    T* d = reinterpret_cast<T*>(psm + ((size_t)(cv * IH + row) * IW + pos) * VB);
+#pragma unroll
+    for (int j = 0; j < N; ++j) d[j] = from_f<T>(v[j]);
+  }
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int cv = warp & 1, pr0 = warp >> 1;
+  const int q = q0 + lane, c = c0 + cv * N;
+  if (q >= a.Q || c >= a.C) return;
+  const uint8_t* plane = psm + (size_t)cv * IH * IW * VB;
+#pragma unroll
+  for (int k = 0; k < 2; ++k) {
+    const int pl = pr0 + 4 * k, p = p0 + pl;
+    if (p >= a.P) break;
+    float acc[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) acc[j] = pad;
+#pragma unroll
+    for (int r = 0; r < (KS > 0 ? KS : 1); ++r) {
+      for (int r2 = 0; r2 < (KS > 0 ? 1 : kh); ++r2) {
+        const int row = pl * a.sh + (KS > 0 ? r : r2);
+#pragma unroll
+        for (int s2 = 0; s2 < (KS > 0 ? KS : 1); ++s2) {
+          for (int s3 = 0; s3 < (KS > 0 ? 1 : kw); ++s3) {
+            const int col = lane * a.sw + (KS > 0 ? s2 : s3);
+            const int pos = a.sw == 2 ? ((col & 1) * half + (col >> 1)) : col;
+            float v[N];
+            load8(reinterpret_cast<const T*>(plane + ((size_t)row * IW + pos) * VB), 0, N, v);
+#pragma unroll
+            for (int j = 0; j < N; ++j) acc[j] = a.is_max ? fmaxf(acc[j], v[j]) : acc[j] + v[j];
+          }
+        }
+      }
+    }
+    if (!a.is_max) {
+      const int h0 = p * a.sh - a.ph, w0 = q * a.sw - a.pw;
+      int div;
+      if (a.cip) div = (min(h0 + kh, a.H + a.ph) - h0) * (min(w0 + kw, a.W + a.pw) - w0);
+      else div = (min(h0 + kh, a.H) - max(h0, 0)) * (min(w0 + kw, a.W) - max(w0, 0));
+      const float inv = 1.f / (float)div;
+#pragma unroll
+      for (int j = 0; j < N; ++j) acc[j] *= inv;
+    }
+    const size_t pix = (size_t)p * a.Q + q;
+    store8(a.out + pix * a.ldo + c, c, a.C, acc);
+    if (a.out2) store8(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+  }
+}
+
+template <typename T, int KS>
+static void launch_pool_tiled(const PoolArgs<T>& a, size_t smem, cudaStream_t st) {
+  static bool attr_set[64] = {false};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 64 && !attr_set[dev]) {
+    cudaFuncSetAttribute(pool_tiled_kernel<T, KS>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    attr_set[dev] = true;
+  }
+  dim3 grid((a.C + 15) / 16, (a.Q + kPoolTQ - 1) / kPoolTQ, (a.P + kPoolTP - 1) / kPoolTP);
+  launch_pdl(pool_tiled_kernel<T, KS>, grid, dim3(256), smem, st, a);
+}
+
 template <typename T>
 void launch_pool(const PoolArgs<T>& a, cudaStream_t st) {
   constexpr int N = Vec<T>::N;
+  const size_t smem = (size_t)2 * ((kPoolTP - 1) * a.sh + a.kh) * ((kPoolTQ - 1) * a.sw + a.kw) * 8 * sizeof(T);
+  if ((a.sw == 1 || a.sw == 2) && a.kh * a.kw > 1 && smem <= 200 * 1024 && !getenv("HIOS_POOL_OLD")) {
+    if (a.kh == 3 && a.kw == 3) return launch_pool_tiled<T, 3>(a, smem, st);
+    return launch_pool_tiled<T, 0>(a, smem, st);
+  }
   const int per_row = a.Q * ((a.C + N - 1) / N);
   dim3 grid((per_row + 255) / 256, a.P);
   if (a.kh == 3 && a.kw == 3)
@@ -151,9 +266,138 @@ __global__ void dw_kernel(const DwArgs<T> a) {
   store_vec(a.out + (size_t)pix * a.ldo + c, c, a.C, acc);
 }
 
+// Tiled depthwise: a CTA owns 8 output rows x 32 output columns x 16
+// channels.  The (aggregated, pre-ReLU'd, zero-padded) input window of the
+// tile is staged once in smem as [channel vector][row][col] planes (columns
+// de-interleaved by parity when sw == 2, so a warp's 32 lanes read 32
+// consecutive 16-byte vectors at every tap), the 16 channels' weights as fp32.
+// Warp w: channel vector w & 1, output rows (w >> 1) and (w >> 1) + 4; lane:
+// output column.  Per kernel row r the thread holds the S weight vectors in
+// registers (KS > 0) and reuses them for its two output rows.
+constexpr int kDwTP = 8, kDwTQ = 32;
+__host__ __device__ inline int dw_tile_rows(int R, int sh) { return (kDwTP - 1) * sh + R; }
+__host__ __device__ inline int dw_tile_cols(int S, int sw) { return (kDwTQ - 1) * sw + S; }
+
+template <typename T, int KS>
+__global__ void __launch_bounds__(256) dw_tiled_kernel(const DwArgs<T> a) {
+  extern __shared__ __align__(16) uint8_t dsm[];
+  constexpr int N = 8;                       // channels per vector (16 B bf16, 32 B fp32)
+  constexpr int VB = N * (int)sizeof(T);     // bytes per staged vector
+  const int R = KS > 0 ? KS : a.R, S = KS > 0 ? KS : a.S;
+  const int IH = dw_tile_rows(R, a.sh), IW = dw_tile_cols(S, a.sw);
+  const int half = (IW + 1) / 2;
+  // channel slab fastest in the grid (see pool_tiled_kernel)
+  const int q0 = blockIdx.y * kDwTQ, p0 = blockIdx.z * kDwTP, c0 = blockIdx.x * 16;
+  float* sw_ = reinterpret_cast<float*>(dsm);                  // [R*S][16]
+  uint8_t* tile = dsm + (size_t)R * S * 16 * sizeof(float);   // [2][IH][IW] vectors
+  for (int i = threadIdx.x; i < R * S * 16; i += blockDim.x) {
+    const int rs = i >> 4, j = i & 15;
+    sw_[i] = (c0 + j < a.C) ? __ldg(a.w + (size_t)rs * a.C + c0 + j) : 0.f;
+  }
+  pdl_enter();
+  const int hb = p0 * a.sh - a.ph, wb = q0 * a.sw - a.pw;
+  const int nel = 2 * IH * IW;
+  for (int e = threadIdx.x; e < nel; e += blockDim.x) {
+    const int cv = e & 1, pix = e >> 1;
+    const int row = pix / IW, col = pix - row * IW;
+    const int h = hb + row, w = wb + col, c = c0 + cv * N;
+    float u[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) u[j] = 0.f;
+    if (h >= 0 && h < a.H && w >= 0 && w < a.W && c < a.C) {
+      const size_t off = (size_t)h * a.W + w;
+      for (int i = 0; i < a.n_in; ++i) {
+        float v[N];
+        load8(a.x[i] + off * a.ldx[i] + c, c, a.C, v);
+#pragma unroll
+        for (int j = 0; j < N; ++j) u[j] += a.agg[i] * v[j];
+      }
+      if (a.pre_relu) {
+#pragma unroll
+        for (int j = 0; j < N; ++j) u[j] = fmaxf(u[j], 0.f);
+      }
+    }
+    const int pos = a.sw == 2 ? ((col & 1) * half + (col >> 1)) : col;
+    T* d = reinterpret_cast<T*>(tile + ((size_t)(cv * IH + row) * IW + pos) * VB);
+#pragma unroll
+    for (int j = 0; j < N; ++j) d[j] = from_f<T>(u[j]);
+  }
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int cv = warp & 1, pr0 = warp >> 1;
+  const int q = q0 + lane;
+  const uint8_t* plane = tile + (size_t)cv * IH * IW * VB;
+  const float* wv = sw_ + cv * N;
+  float acc[2][N];
+#pragma unroll
+  for (int k = 0; k < 2; ++k)
+#pragma unroll
+    for (int j = 0; j < N; ++j) acc[k][j] = 0.f;
+  auto tap = [&](float (&ac)[N], int row, int s, const float* wt) {
+    const int col = lane * a.sw + s;
+    const int pos = a.sw == 2 ? ((col & 1) * half + (col >> 1)) : col;
+    const T* src = reinterpret_cast<const T*>(plane + ((size_t)row * IW + pos) * VB);
+    float v[N];
+    load8(src, 0, N, v);
+#pragma unroll
+    for (int j = 0; j < N; ++j) ac[j] = fmaf(v[j], wt[j], ac[j]);
+  };
+  for (int r = 0; r < R; ++r) {
+    if (KS > 0) {
+      float wr[KS > 0 ? KS : 1][N];
+#pragma unroll
+      for (int s2 = 0; s2 < (KS > 0 ? KS : 1); ++s2)
+#pragma unroll
+        for (int j = 0; j < N; ++j) wr[s2][j] = wv[(r * S + s2) * 16 + j];
+#pragma unroll
+      for (int k = 0; k < 2; ++k) {
+        const int row = (pr0 + 4 * k) * a.sh + r;
+#pragma unroll
+        for (int s2 = 0; s2 < (KS > 0 ? KS : 1); ++s2) tap(acc[k], row, s2, wr[s2]);
+      }
+    } else {
+      for (int s2 = 0; s2 < S; ++s2) {
+        float wt[N];
+#pragma unroll
+        for (int j = 0; j < N; ++j) wt[j] = wv[(r * S + s2) * 16 + j];
+#pragma unroll
+        for (int k = 0; k < 2; ++k) tap(acc[k], (pr0 + 4 * k) * a.sh + r, s2, wt);
+      }
+    }
+  }
+  const int c = c0 + cv * N;
+  if (q >= a.Q || c >= a.C) return;
+#pragma unroll
+  for (int k = 0; k < 2; ++k) {
+    const int p = p0 + pr0 + 4 * k;
+    if (p < a.P) store8(a.out + ((size_t)p * a.Q + q) * a.ldo + c, c, a.C, acc[k]);
+  }
+}
+
+template <typename T, int KS>
+static void launch_dw_tiled(const DwArgs<T>& a, size_t smem, cudaStream_t st) {
+  static bool attr_set[64] = {false};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 64 && !attr_set[dev]) {
+    cudaFuncSetAttribute(dw_tiled_kernel<T, KS>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    attr_set[dev] = true;
+  }
+  dim3 grid((a.C + 15) / 16, (a.Q + kDwTQ - 1) / kDwTQ, (a.P + kDwTP - 1) / kDwTP);
+  launch_pdl(dw_tiled_kernel<T, KS>, grid, dim3(256), smem, st, a);
+}
+
 template <typename T>
 void launch_dw(const DwArgs<T>& a, cudaStream_t st) {
   constexpr int N = Vec<T>::N;
+  const size_t smem = (size_t)a.R * a.S * 16 * sizeof(float) +
+                      (size_t)2 * dw_tile_rows(a.R, a.sh) * dw_tile_cols(a.S, a.sw) * 8 * sizeof(T);
+  if ((a.sw == 1 || a.sw == 2) && smem <= 200 * 1024 && !getenv("HIOS_DW_OLD")) {
+    if (a.R == 3 && a.S == 3) return launch_dw_tiled<T, 3>(a, smem, st);
+    if (a.R == 5 && a.S == 5) return launch_dw_tiled<T, 5>(a, smem, st);
+    if (a.R == 7 && a.S == 7) return launch_dw_tiled<T, 7>(a, smem, st);
+    return launch_dw_tiled<T, 0>(a, smem, st);
+  }
   long long n = (long long)a.P * a.Q * ((a.C + N - 1) / N);
   launch_pdl(dw_kernel<T>, dim3(grid_for(n, 256)), dim3(256), 0, st, a);
 }
@@ -359,12 +603,45 @@ void launch_fill(void* p, size_t bytes, cudaStream_t st) {
   fill_kernel<<<148 * 8, 512, 0, st>>>(reinterpret_cast<uint4*>(p), bytes / 16);
 }
 
+// ------------------------------------------------- space-to-depth (stems)
+// one thread per X' pixel: 4 source pixels (a, b) in {0,1}^2, C <= 4 channels
+// each, packed to (a*2+b)*C + c and zero-padded to the pixel stride
+template <typename T>
+__global__ void s2d_kernel(const S2dArgs<T> a) {
+  pdl_enter();
+  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= (long long)a.P2 * a.Q2) return;
+  const int i = (int)(idx / a.Q2), j = (int)(idx - (long long)i * a.Q2);
+  T v[16];
+#pragma unroll
+  for (int e = 0; e < 16; ++e) v[e] = from_f<T>(0.f);
+#pragma unroll
+  for (int ab = 0; ab < 4; ++ab) {
+    const int h = 2 * i + (ab >> 1) - a.ph, w = 2 * j + (ab & 1) - a.pw;
+    if (h < 0 || h >= a.H || w < 0 || w >= a.W) continue;
+    const T* src = a.x + ((size_t)h * a.W + w) * a.ldx;
+#pragma unroll
+    for (int c = 0; c < 4; ++c)
+      if (c < a.C) v[ab * a.C + c] = src[c];
+  }
+  T* dst = a.out + (size_t)idx * a.ldo;
+  // 4C <= 16 channels, ldo is a multiple of 8: 16-byte stores (bf16) / 4 x 16 B (fp32)
+  constexpr int N = Vec<T>::N;
+  for (int e = 0; e < a.ldo && e < 16; e += N) *reinterpret_cast<uint4*>(dst + e) = *reinterpret_cast<const uint4*>(v + e);
+}
+
+template <typename T>
+void launch_s2d(const S2dArgs<T>& a, cudaStream_t st) {
+  launch_pdl(s2d_kernel<T>, dim3(grid_for((long long)a.P2 * a.Q2, 256)), dim3(256), 0, st, a);
+}
+
 // explicit instantiations
 #define HIOS_INST(T)                                                                                   \
   template void launch_pool<T>(const PoolArgs<T>&, cudaStream_t);                                      \
   template void launch_dw<T>(const DwArgs<T>&, cudaStream_t);                                          \
   template void launch_add<T>(const AddArgs<T>&, cudaStream_t);                                        \
   template void launch_copy<T>(const CopyArgs<T>&, cudaStream_t);                                      \
+  template void launch_s2d<T>(const S2dArgs<T>&, cudaStream_t);                                        \
   template void launch_gap<T>(const T*, int, int, int, T*, cudaStream_t);                              \
   template void launch_linear<T>(const T*, int, const T*, int, const float*, int, T*, cudaStream_t);        \
   template void launch_input<T>(const float*, int, int, int, T*, int, cudaStream_t);                   \

@@ -80,6 +80,11 @@ CONV_CASES = [
     (80, 192, 9, 252, 3, 3, 1, 0, 0),
     (96, 96, 7, 300, 1, 7, 1, 0, 3),
     (64, 80, 13, 100, 7, 1, 1, 3, 0),
+    # stride-2 stems with C <= 4 (bf16: space-to-depth + tensor-core conv)
+    (3, 96, 61, 229, 7, 7, 2, 0, 0),      # SqueezeNet conv1 shape, odd sizes, halo width
+    (3, 96, 45, 260, 3, 3, 2, 1, 1),      # NASNet-like conv0 with padding
+    (3, 39, 33, 37, 3, 3, 2, 1, 1),       # RandWire conv1: K = 39 (ragged N), tap mode
+    (2, 24, 30, 31, 5, 5, 2, 2, 2),       # C = 2, 5x5 (taps past R, S in W')
     # halo mode with resident weights (one N tile, > 148 output tiles per CTA wave)
     (32, 32, 160, 200, 3, 3, 1, 1, 1),
     (64, 80, 150, 130, 1, 1, 1, 0, 0),
@@ -120,6 +125,61 @@ def test_conv_parity_splitk(case, monkeypatch):
     err, n_split = conv_case("bf16", case)
     assert n_split == n_plain + 1  # the finalize kernel: split-K really ran
     assert err <= TOL["bf16"] / 4
+
+
+SEP_CASES = [
+    # (C, K, H, W, k, s, n_in, reps)
+    (42, 42, 47, 70, 7, 2, 1, 2),         # NASNet stem shape: 7x7 stride 2, C % 16 != 0
+    (78, 78, 40, 45, 3, 1, 5, 1),         # RandWire node: 5-input weighted aggregation
+    (168, 168, 20, 33, 5, 1, 1, 2),       # NASNet cell: 5x5, several 16-channel slabs
+    (20, 24, 19, 37, 4, 2, 2, 1),         # generic kernel size (even), stride 2, aggregation
+    (336, 336, 17, 9, 7, 2, 1, 2),        # deep, narrow (tile mostly padding)
+]
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+@pytest.mark.parametrize("case", SEP_CASES)
+def test_sepconv_parity(dtype, case):
+    """Depthwise (smem-tiled kernel) + pointwise per repetition, per-op check
+    and end to end."""
+    C, K, H, Wd, k, s, n_in, reps = case
+    g = graphs.GraphSpec("sep", C, H, Wd)
+    x0 = g.input()
+    ins = [g.conv(x0, C, 1, relu=0) for _ in range(n_in)] if n_in > 1 else [x0]
+    g.sepconv(ins, K, k, s=s, pre_relu=1, relu=1, reps=reps)
+    W = gen.make_weights(g)
+    x = gen.make_input(g) - 0.5
+    _, S, y = run_graph_gpu(g, W, x, dtype, profile=False)
+    per_op_check(g, W, S, dtype)
+    ref = infer.run_graph(g, W, x)[g.n_ops - 1].reshape(-1)
+    assert nerr(y, ref) <= TOL[dtype]
+
+
+POOL_CASES = [
+    # (kind, C, H, W, k, s, p, ceil_mode, count_include_pad)
+    ("max", 96, 61, 75, 3, 2, 0, 1, 0),     # SqueezeNet: ceil mode, several column tiles
+    ("avg", 288, 35, 41, 3, 1, 1, 0, 1),    # Inception avgpool branch
+    ("avg", 42, 33, 29, 3, 2, 1, 0, 0),     # NASNet: C % 16 != 0, in-bounds divisor
+    ("max", 40, 20, 70, 3, 2, 1, 0, 0),     # padded max
+    ("avg", 24, 17, 40, 2, 2, 0, 1, 1),     # generic k (even), ceil + count_include_pad
+]
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+@pytest.mark.parametrize("case", POOL_CASES)
+def test_pool_parity(dtype, case):
+    kind, C, H, Wd, k, s, p, cm, cip = case
+    g = graphs.GraphSpec("pool", C, H, Wd)
+    x0 = g.input()
+    if kind == "max":
+        g.maxpool(x0, k, s, p, ceil_mode=cm)
+    else:
+        g.avgpool(x0, k, s, p, ceil_mode=cm, count_include_pad=cip)
+    W = gen.make_weights(g)
+    x = gen.make_input(g) - 0.5
+    _, S, y = run_graph_gpu(g, W, x, dtype, profile=False)
+    ref = infer.run_graph(g, W, x)[g.n_ops - 1].reshape(-1)
+    assert nerr(y, ref) <= TOL[dtype] / (4 if dtype == "bf16" else 1)
 
 
 @pytest.mark.parametrize("dtype", ["bf16", "f32"])

@@ -1,0 +1,14 @@
+#!/bin/bash
+# parity of the touched kernels + the four workloads' latency
+cd "$GRAFT_REPO_ROOT" || exit 1
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "conv_parity or sepconv or zoo or end_to_end" > gpurun_out/tq.log 2>&1; echo tq_rc=$?; tail -15 gpurun_out/tq.log
+timeout 900 python bench.py --steps 10 --no-cpu-baseline --sweep "4096,randwire_ws@2048,nasnet_a_large@2048,squeezenet@2048" > gpurun_out/bq.json 2> gpurun_out/bq.err; echo bq_rc=$?
+python - <<'PY'
+import json
+d=json.load(open('gpurun_out/bq.json'))
+print('ms', d['value'], 'cp', d['critical_path']['frac'], 'conv', d['roofline']['frac'])
+for k,v in d['size_sweep'].items():
+    print(k, {a: (round(b,3) if isinstance(b,float) else b) for a,b in v.items() if a in ('hios_lp_ms','cp_bound_ms','cp_frac','sequential_ms','error')})
+PY
+tail -3 gpurun_out/bq.err
