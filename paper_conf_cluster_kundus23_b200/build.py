@@ -10,9 +10,11 @@ import subprocess
 import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-CSRC = os.path.join(HERE, "csrc")
-BUILD = os.path.join(HERE, "_build")
-LIB = os.path.join(HERE, "libhios.so")
+# HIOS_CSRC / HIOS_BUILD / HIOS_LIB_OUT: build another source tree into another
+# library (A/B timing experiments, tools/build_variant.sh); defaults = in-tree
+CSRC = os.environ.get("HIOS_CSRC", os.path.join(HERE, "csrc"))
+BUILD = os.environ.get("HIOS_BUILD", os.path.join(HERE, "_build"))
+LIB = os.environ.get("HIOS_LIB_OUT", os.path.join(HERE, "libhios.so"))
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",

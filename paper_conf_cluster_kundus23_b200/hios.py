@@ -11,7 +11,8 @@ from typing import Dict, List, Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libhios.so")
+# HIOS_LIB: load another build of the library (A/B timing experiments only)
+LIB_PATH = os.environ.get("HIOS_LIB", os.path.join(_HERE, "libhios.so"))
 
 KIND = {"input": 0, "conv": 1, "sepconv": 2, "maxpool": 3, "avgpool": 4, "gap": 5,
         "concat": 6, "add": 7, "linear": 8, "identity": 9}
