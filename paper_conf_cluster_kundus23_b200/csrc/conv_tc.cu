@@ -215,6 +215,7 @@ __device__ unsigned long long g_conv_trace[256 * 8];
 __device__ unsigned long long g_conv_trace2[32 * 48];  // per CTA: issue[16], full[16], empty_ok[16]
 __device__ unsigned long long g_conv_trace3[32 * 8];   // per CTA: epilogue checkpoints
 __device__ unsigned long long g_conv_trace4[32 * 16];  // per CTA: first-tile epilogue, fine-grained
+__device__ unsigned long long g_conv_trace5[32 * 48];  // per CTA: epilogue tfull[16], stores issued[16]
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
@@ -231,6 +232,10 @@ __device__ __forceinline__ unsigned long long gtimer() {
 #define TRACE4(k)                                                         \
   do {                                                                    \
     if (a.trace && blockIdx.x < 32 && tcount == 0 && et == 0) g_conv_trace4[blockIdx.x * 16 + (k)] = gtimer(); \
+  } while (0)
+#define TRACE5(slot, k)                                                   \
+  do {                                                                    \
+    if (a.trace && blockIdx.x < 32 && (k) < 16 && et == 0) g_conv_trace5[blockIdx.x * 48 + (slot) * 16 + (k)] = gtimer(); \
   } while (0)
 #define TRACE(k)                                                          \
   do {                                                                    \
@@ -267,14 +272,16 @@ __global__ void __launch_bounds__(kThreads, 1)
   uint8_t* sB = smem + (a.halo ? a.a_bufs * H_BYTES : ST * a.kps * A_BYTES);
   // B: a ring of ST stages x kps K-steps, or (bres) every K-step's weights resident
   uint8_t* sOut = sB + (a.bres ? (uint32_t)(a.c_chunks * a.R * a.S) : (uint32_t)(ST * a.kps)) * B_BYTES;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sOut + 128 * PITCH);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sOut + (uint32_t)a.out_bufs * 128u * PITCH);
   // barriers: full[ST] empty[ST] afull[2] aempty[2] tfull[2] tempty[2]
   const uint32_t full0 = smem_u32(bars), empty0 = full0 + 8 * ST;
-  const uint32_t afull0 = empty0 + 8 * ST, aempty0 = afull0 + 16, tfull0 = aempty0 + 16, tempty0 = tfull0 + 16;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * ST + 8);
-  const uint32_t bres_bar = smem_u32(bars + 2 * ST + 9);  // resident weights landed
-  float* s_scale = reinterpret_cast<float*>(bars + 2 * ST + 10);  // [256]
-  float* s_shift = s_scale + 256;                                  // [256]
+  const uint32_t afull0 = empty0 + 8 * ST, aempty0 = afull0 + 8 * kMaxABufs, tfull0 = aempty0 + 8 * kMaxABufs,
+                 tempty0 = tfull0 + 16;
+  constexpr int kBarX = 2 * kMaxABufs + 4;  // afull/aempty[kMaxABufs], tfull/tempty[2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * ST + kBarX);
+  const uint32_t bres_bar = smem_u32(bars + 2 * ST + kBarX + 1);  // resident weights landed
+  float* s_scale = reinterpret_cast<float*>(bars + 2 * ST + kBarX + 2);  // [kScaleRes]
+  float* s_shift = s_scale + kScaleRes;                            // [kScaleRes]
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t ncols = tmem_cols(2 * a.n_tile);
@@ -291,9 +298,11 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(empty0 + 8 * i, nmma);
     }
     mbar_init(bres_bar, 1);
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < kMaxABufs; ++i) {
       mbar_init(afull0 + 8 * i, 1);
       mbar_init(aempty0 + 8 * i, nmma);
+    }
+    for (int i = 0; i < 2; ++i) {
       mbar_init(tfull0 + 8 * i, nmma);
       mbar_init(tempty0 + 8 * i, 32 * kEpi);
     }
@@ -372,7 +381,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             __syncwarp();
           }
           if (a.halo && rs == 0) {
-            if (a.a_bufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
+            if (++ab == (uint32_t)a.a_bufs) { ab = 0; aph ^= 1u; }
             ++hcount;
           }
           // K-steps of this stage: up to KPS, never crossing a chunk in halo mode
@@ -482,7 +491,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               }
             }
             mma_commit_on(aempty0 + 8 * ab, on);
-            if (abufs == 2) { ab ^= 1u; if (ab == 0) aph ^= 1u; } else { aph ^= 1u; }
+            if (++ab == (uint32_t)abufs) { ab = 0; aph ^= 1u; }
           }
           if (bres && lane == 0 && j == 0) TRACE2(2, tcount);
           mma_commit_on(tfull0 + 8 * acc, on);
@@ -551,6 +560,17 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int m = lw * 32 + lane;
     const int et = threadIdx.x - 32 * kEpiWarp0;  // 0..127
     uint32_t tcount = 0, acc = 0, tph = 0;
+    if (a.sres) {
+      // all K channels' folded BN once per CTA (rounded up to the N tile;
+      // channels past K read the last one and are clipped at the store)
+      const int kr = a.tiles_n * a.n_tile;
+      for (int jj = et; jj < kr; jj += 128) {
+        const int nj = min(jj, a.K - 1);
+        asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_scale + jj)), "f"(__ldg(a.scale + nj)) : "memory");
+        asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_shift + jj)), "f"(__ldg(a.shift + nj)) : "memory");
+      }
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+    }
     for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
       const int split = tile / tiles_mn, tmn = tile - split * tiles_mn;
       const int m_blk = tmn / a.tiles_n, n_blk = tmn - m_blk * a.tiles_n;
@@ -585,30 +605,120 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (acc == 0) tph ^= 1u;
         continue;
       }
-      // previous tile fully copied out of sOut / s_scale (all 128 threads;
-      // TMA-store mode: the bulk stores have finished reading sOut)
+      // staging tile of this tile (two alternate when out_bufs == 2, so the
+      // bulk stores of tile i drain while tile i+1 is staged)
+      const uint32_t ob = a.out_bufs == 2 ? (tcount & 1u) : 0u;
+      const uint32_t sOut_t = smem_u32(sOut) + ob * 128u * PITCH;
       TRACE4(0);
-      if (a.tma_out && lane == 0) bulk_wait_read0();
-      asm volatile("bar.sync 1, 128;" ::: "memory");
-      for (int jj = et; jj < a.n_tile; jj += 128) {
-        const int nj = min(n0 + jj, a.K - 1);
-        asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_scale + jj)), "f"(__ldg(a.scale + nj)) : "memory");
-        asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_shift + jj)), "f"(__ldg(a.shift + nj)) : "memory");
+      if (a.sres && (a.tma_out || a.epi == 2)) {
+        // scale/shift resident; each warp stages and ships only its own 32
+        // rows, so it only waits for its own earlier stores out of this buffer
+        // (direct-store mode: no staging at all)
+        if (a.tma_out) {
+          if (lane == 0) {
+            if (a.out_bufs == 2) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+            else bulk_wait_read0();
+          }
+          __syncwarp();
+        }
+      } else {
+        // previous tile fully copied out of sOut / s_scale (all 128 threads;
+        // TMA-store mode: the bulk stores have finished reading sOut)
+        if (a.tma_out && lane == 0) bulk_wait_read0();
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+        if (!a.sres) {
+          for (int jj = et; jj < a.n_tile; jj += 128) {
+            const int nj = min(n0 + jj, a.K - 1);
+            asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_scale + jj)), "f"(__ldg(a.scale + nj)) : "memory");
+            asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_shift + jj)), "f"(__ldg(a.shift + nj)) : "memory");
+          }
+          asm volatile("bar.sync 1, 128;" ::: "memory");
+        }
       }
-      asm volatile("bar.sync 1, 128;" ::: "memory");
       TRACE4(1);
       mbar_wait(tfull0 + 8 * acc, tph);
       __syncwarp();
       tc_fence_after();
       TRACE4(2);
+      TRACE5(0, tcount);
       if (tcount == 0 && warp == kEpiWarp0 && lane == 0) TRACE(5);
       const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)a.n_tile;
-      const uint32_t srow = smem_u32(sOut) + (uint32_t)m * PITCH;
+      if (a.epi == 2) {
+        // direct stores: each thread owns one output pixel (its TMEM lane)
+        // and writes its n_valid channels as 16-byte vectors straight from
+        // registers -- no staging, no proxy fence, no bulk-group waits
+        const float* scs = s_scale + (a.sres ? n0 : 0);
+        const float* shs = s_shift + (a.sres ? n0 : 0);
+        const int hh = m / a.tw, ww = m - hh * a.tw;
+        const int p = p0 + hh, q = q0 + ww;
+        const bool valid = p < a.P && q < a.Q;
+        const size_t pix = (size_t)p * a.Q + q;
+        bf16* o1 = a.out + pix * a.ldo + n0;
+        bf16* o2 = a.out2 ? a.out2 + pix * a.ldo2 + n0 : nullptr;
+        for (int col = 0; col < a.n_tile; col += 32) {
+          const bool two = col + 16 < a.n_tile;  // warp-uniform
+          uint32_t r0[16], r1[16];
+          tmem_ld16_nw(tbase + (uint32_t)col, r0);
+          if (two) tmem_ld16_nw(tbase + (uint32_t)col + 16u, r1);
+          float sc[32], sf[32];
+#pragma unroll
+          for (int q4 = 0; q4 < 8; ++q4) {
+            const uint4 u = lds128(smem_u32(scs + col + 4 * q4));
+            const uint4 w = lds128(smem_u32(shs + col + 4 * q4));
+            sc[4 * q4] = __uint_as_float(u.x); sc[4 * q4 + 1] = __uint_as_float(u.y);
+            sc[4 * q4 + 2] = __uint_as_float(u.z); sc[4 * q4 + 3] = __uint_as_float(u.w);
+            sf[4 * q4] = __uint_as_float(w.x); sf[4 * q4 + 1] = __uint_as_float(w.y);
+            sf[4 * q4 + 2] = __uint_as_float(w.z); sf[4 * q4 + 3] = __uint_as_float(w.w);
+          }
+          tmem_wait_pin(r0);
+          pin16(r1);
+#pragma unroll
+          for (int hlf = 0; hlf < 2; ++hlf) {
+            const int c16 = col + 16 * hlf;
+            if (hlf == 1 && !two) break;
+            const uint32_t* r = hlf ? r1 : r0;
+            uint32_t pk[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+              float y0 = __uint_as_float(r[2 * e]) * sc[16 * hlf + 2 * e] + sf[16 * hlf + 2 * e];
+              float y1 = __uint_as_float(r[2 * e + 1]) * sc[16 * hlf + 2 * e + 1] + sf[16 * hlf + 2 * e + 1];
+              if (a.relu) { y0 = fmaxf(y0, 0.f); y1 = fmaxf(y1, 0.f); }
+              __nv_bfloat162 b2 = __floats2bfloat162_rn(y0, y1);
+              pk[e] = *reinterpret_cast<uint32_t*>(&b2);
+            }
+            if (!valid) continue;
+#pragma unroll
+            for (int v8 = 0; v8 < 2; ++v8) {
+              const int c8 = c16 + 8 * v8;
+              if (c8 + 8 <= n_valid) {
+                const uint4 v = make_uint4(pk[4 * v8], pk[4 * v8 + 1], pk[4 * v8 + 2], pk[4 * v8 + 3]);
+                *reinterpret_cast<uint4*>(o1 + c8) = v;
+                if (o2) *reinterpret_cast<uint4*>(o2 + c8) = v;
+              } else {
+                for (int e = 0; e < 8 && c8 + e < n_valid; ++e) {
+                  const uint16_t hv = (uint16_t)(pk[4 * v8 + (e >> 1)] >> (16 * (e & 1)));
+                  reinterpret_cast<uint16_t*>(o1)[c8 + e] = hv;
+                  if (o2) reinterpret_cast<uint16_t*>(o2)[c8 + e] = hv;
+                }
+              }
+            }
+          }
+        }
+        tc_fence_before();
+        mbar_arrive(tempty0 + 8 * acc);
+        TRACE5(1, tcount);
+        acc ^= 1u;
+        if (acc == 0) tph ^= 1u;
+        continue;
+      }
+      const uint32_t srow = sOut_t + (uint32_t)m * PITCH;
       // TMA-store staging: slabs of out_sw channels, [128 rows][out_sw*2 B],
       // 16-byte chunks XOR-swizzled like the tensor map (bits 4.. ^= bits 7..)
       const uint32_t SWB = (uint32_t)a.out_sw * 2u, swm = SWB / 16u - 1u;
       const uint32_t sw_log = a.out_sw == 64 ? 6u : (a.out_sw == 32 ? 5u : 4u);
-      const uint32_t s_sc = smem_u32(s_scale), s_sh = smem_u32(s_shift);
+      // resident scale/shift are indexed by absolute channel (n0 + col)
+      const uint32_t s_sc = smem_u32(s_scale) + (a.sres ? (uint32_t)n0 * 4u : 0u),
+                     s_sh = smem_u32(s_shift) + (a.sres ? (uint32_t)n0 * 4u : 0u);
       // one 16-column group: folded BN + ReLU -> bf16 -> staging tile
       auto emit16 = [&](int col, const uint32_t (&r)[16], const float* sc, const float* sf) {
         uint32_t pk[8];
@@ -623,7 +733,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (a.tma_out) {
           const uint32_t slab = (uint32_t)col >> sw_log;
           const uint32_t cb = ((uint32_t)col - (slab << sw_log)) * 2u;  // byte in the slab row
-          const uint32_t base = smem_u32(sOut) + slab * 128u * SWB;
+          const uint32_t base = sOut_t + slab * 128u * SWB;
           const uint32_t o0 = (uint32_t)m * SWB + cb, o1 = o0 + 16u;
           sts128(base + (o0 ^ (((o0 >> 7) & swm) << 4)), pk[0], pk[1], pk[2], pk[3]);
           sts128(base + (o1 ^ (((o1 >> 7) & swm) << 4)), pk[4], pk[5], pk[6], pk[7]);
@@ -677,7 +787,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (uint32_t sl = 0; sl < nslab; ++sl) {
             const int c0 = n0 + (int)(sl << sw_log);
             if (c0 >= a.K) break;
-            const uint32_t src = smem_u32(sOut) + sl * 128u * SWB + (uint32_t)mr * SWB;
+            const uint32_t src = sOut_t + sl * 128u * SWB + (uint32_t)mr * SWB;
             tma_store_3d(&mo, src, c0, q0 + ww0, p0 + hh0);
             if (a.out2) tma_store_3d(&mo2, src, c0, q0 + ww0, p0 + hh0);
           }
@@ -685,6 +795,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         __syncwarp();
         TRACE4(12);
+        TRACE5(1, tcount);
         if (tcount == 0 && et == 0) TRACE3(1);
         continue;
       }
@@ -696,7 +807,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // one output pixel row (loads issued ahead of the dependent stores)
       const int row_bytes = n_valid * 2;
       const int chunks = row_bytes >> 4;
-      const uint32_t sbase = smem_u32(sOut);
+      const uint32_t sbase = sOut_t;
       const int total = 128 * chunks;
       for (int i0 = et; i0 < total; i0 += 128 * 4) {
         uint4 v[4];
@@ -796,8 +907,9 @@ void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st) {
 size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
   const size_t B = a.bres ? (size_t)a.n_tile * 128 * a.c_chunks * a.R * a.S : (size_t)a.n_tile * 128 * a.kps * a.stages;
   const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.R, a.halo_w) : (size_t)a.stages * a.kps * 128 * 128;
-  return 1024 + A + B + 128 * (size_t)stage_pitch(a.n_tile) + (2 * a.stages + 10) * 8 +
-         2 * 256 * 4;
+  return 1024 + A + B + (size_t)a.out_bufs * 128 * (size_t)stage_pitch(a.n_tile) +
+         (2 * a.stages + 2 * kMaxABufs + 6) * 8 +
+         2 * kScaleRes * 4;
 }
 
 void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const CUtensorMap& mo, const CUtensorMap& mo2,
@@ -837,6 +949,9 @@ extern "C" int hios_debug_conv_trace3(unsigned long long* out) {
   return (int)cudaMemcpyFromSymbol(out, hios::g_conv_trace3, sizeof(unsigned long long) * 32 * 8);
 }
 
+extern "C" int hios_debug_conv_trace5(unsigned long long* out) {
+  return (int)cudaMemcpyFromSymbol(out, hios::g_conv_trace5, sizeof(unsigned long long) * 32 * 48);
+}
 extern "C" int hios_debug_conv_trace2(unsigned long long* out) {
   return (int)cudaMemcpyFromSymbol(out, hios::g_conv_trace2, sizeof(unsigned long long) * 32 * 48);
 }

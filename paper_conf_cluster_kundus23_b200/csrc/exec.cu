@@ -391,9 +391,16 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   }
   const size_t B = (size_t)c.n_tile * 128;
   const size_t stage_out = 128 * ((size_t)c.n_tile * 2 + 16);
-  // occupancy: 1 CTA/SM (212 KB) or 2 CTAs/SM (104 KB each, TMEM <= 256 cols)
+  // epilogue: two staging tiles for N tiles <= 128 (the stores of tile i
+  // drain while tile i+1 is staged), folded BN resident when K is small
   c.occ = (getenv("HIOS_OCC") ? atoi(getenv("HIOS_OCC")) : 1) == 2 && c.n_tile <= 128 ? 2 : 1;
-  const size_t budget = (c.occ == 2 ? 104 * 1024 : 212 * 1024) - stage_out;
+  // epilogue mode (HIOS_EPI overrides): direct register stores for N tiles
+  // <= 128 (no staging tile), TMA bulk-tensor stores for wider tiles
+  c.epi = getenv("HIOS_EPI") ? atoi(getenv("HIOS_EPI")) : (c.n_tile <= 128 ? 2 : 1);
+  c.out_bufs = c.epi == 2 ? 0 : ((c.n_tile <= (c.occ == 2 ? 48 : 128) && !getenv("HIOS_OUT1")) ? 2 : 1);
+  c.sres = (c.tiles_n * c.n_tile <= kScaleRes && !getenv("HIOS_NOSRES")) ? 1 : 0;
+  // occupancy: 1 CTA/SM (212 KB) or 2 CTAs/SM (104 KB each, TMEM <= 256 cols)
+  const size_t budget = (c.occ == 2 ? 104 * 1024 : 212 * 1024) - c.out_bufs * stage_out;
   // K-steps per stage: amortise the ~0.3 us full/empty handshake (measured)
   c.kps = getenv("HIOS_KPS") ? std::max(1, atoi(getenv("HIOS_KPS"))) : 0;
   // resident weights (halo mode, one N tile, CTAs that walk several tiles):
@@ -405,7 +412,11 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
       halo_bytes_of(R, hw) + b_all <= budget) {
     c.bres = 1;
     c.kps = std::min(4, R * S);
-    c.a_bufs = (2 * halo_bytes_of(R, hw) + b_all <= budget) ? 2 : 1;
+    // as many input boxes in flight as fit (measured: the halo TMA latency,
+    // ~2 us, bounds a 2-deep ring at small K; tools/conv_trace2.py)
+    const int cap = getenv("HIOS_ABUFS") ? std::max(1, std::min(kMaxABufs, atoi(getenv("HIOS_ABUFS")))) : kMaxABufs;
+    c.a_bufs = 1;
+    while (c.a_bufs < cap && (c.a_bufs + 1) * halo_bytes_of(R, hw) + b_all <= budget) ++c.a_bufs;
     c.stages = 2;
   }
   if (c.halo && !c.bres) {
@@ -413,6 +424,10 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     if (!c.kps) c.kps = std::min(4, R * S);
     while (c.kps > 1 && H + 2 * c.kps * B > budget) --c.kps;
     c.a_bufs = (2 * H + 2 * c.kps * B <= budget) ? 2 : 1;
+    {  // deeper input ring while >= 4 B stages still fit
+      const int cap = getenv("HIOS_ABUFS") ? std::max(1, std::min(kMaxABufs, atoi(getenv("HIOS_ABUFS")))) : 4;
+      while (c.a_bufs < cap && (c.a_bufs + 1) * H + 4 * c.kps * B <= budget) ++c.a_bufs;
+    }
     if (H + 2 * c.kps * B > budget) c.halo = 0;  // does not fit: fall back to tap mode
     else c.stages = (int)std::min<size_t>(8, (budget - c.a_bufs * H) / (c.kps * B));
   }
@@ -497,7 +512,8 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   // destination slice (clips the ragged pixel / channel edges of a tile)
   CUtensorMap mo = mx, mo2 = mx;
   a.out_sw = a.n_tile % 64 == 0 ? 64 : (a.n_tile % 32 == 0 ? 32 : 16);
-  a.tma_out = !getenv("HIOS_NOTMASTORE") && a.ksplit == 1 ? 1 : 0;
+  a.tma_out = !getenv("HIOS_NOTMASTORE") && a.ksplit == 1 && a.epi == 1 ? 1 : 0;
+  if (a.ksplit > 1 || (a.epi == 1 && !a.tma_out)) a.epi = 0;
   if (a.tma_out) {
     const int sb = a.out_sw * 2;
     // one box = one epilogue warp's 32 rows of the 128-pixel tile
@@ -506,6 +522,7 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
                              1, 1, sb) &&
                 (!out2 || make_tmap_3d(&mo2, out2->p, K, Q, P, (uint64_t)out2->ldc * 2,
                                        (uint64_t)Q * out2->ldc * 2, a.out_sw, bw, bh, 1, 1, sb));
+    if (!a.tma_out) a.epi = 0;
   }
   const size_t smem = conv_tc_smem_bytes(a);
   const int grid = std::min(a.tiles_m * a.tiles_n * a.ksplit, 148 * a.occ);

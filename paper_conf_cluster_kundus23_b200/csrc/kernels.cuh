@@ -75,7 +75,12 @@ struct ConvTcArgs {
   int bres;            // halo mode, one N tile: all weights resident in smem (loaded once per CTA)
   int tma_out;         // epilogue leaves smem by TMA bulk-tensor stores (else st.global)
   int out_sw;          // TMA-store slab width in channels (64 / 32 / 16 = 128B/64B/32B swizzle)
+  int out_bufs;        // epilogue staging tiles (2: tile i's stores drain while tile i+1 is staged)
+  int sres;            // folded-BN scale/shift of all K channels staged once per CTA (K <= kScaleRes)
+  int epi;             // epilogue: 0 smem staging + st.global, 1 TMA bulk-tensor stores, 2 direct register stores
 };
+constexpr int kScaleRes = 512;
+constexpr int kMaxABufs = 6;  // halo-mode input boxes in flight
 
 // CUDA-core implicit GEMM (fp32) for the fp32 path (1e-4 parity).
 struct ConvSimtArgs {

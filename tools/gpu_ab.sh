@@ -1,12 +1,13 @@
 #!/bin/bash
-# A/B of a conv-kernel change: parity subset, micro (both arms), trace, bench (both arms)
+# A/B: committed HEAD build (ab/libhios_head.so) vs the working-tree build:
+# op micro-benchmarks ($1: op_micro name prefixes) and the bench (1024 + 4096)
 cd "$GRAFT_REPO_ROOT" || exit 1
-mkdir -p gpurun_out
-timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "conv_parity or tiny or zoo or end_to_end_bf16" > gpurun_out/tq.log 2>&1; echo tq_rc=$?; tail -3 gpurun_out/tq.log
-echo "== micro new"; timeout 300 python tools/conv_micro.py --check
-echo "== micro old ($AB_ENV)"; env $AB_ENV timeout 300 python tools/conv_micro.py
-timeout 300 python tools/conv_trace.py 6e_1x1 7c_3x3 2>&1 | grep -E "==|epi:|start|tma0|data0|mma_end|exit"
-for arm in new old; do
-  E=""; [ $arm = old ] && E="$AB_ENV"
-  env $E timeout 300 python bench.py --no-cpu-baseline --sweep '' --steps 30 2>/dev/null | python -c 'import json,sys; d=json.loads(sys.stdin.read()); print("bench '$arm'", round(d["value"],4), "seq", round(d["single_gpu_refs"]["sequential"]["ms"],4), "conv TF/s", round(d["roofline"]["achieved"],1))'
+OPS=${1:-i4096}
+for rep in 1 2; do
+for v in head cur; do
+  if [ $v = head ]; then export HIOS_LIB=$PWD/ab/libhios_head.so; else unset HIOS_LIB; fi
+  echo "== $v (rep $rep)"
+  timeout 300 python tools/op_micro.py $OPS 2>&1 | cut -c1-90
+  timeout 600 python bench.py --steps 20 --no-cpu-baseline --sweep "4096" 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('bench', round(d['value'],4), 'ios', round(d['single_gpu_refs']['ios']['ms'],4), '4096', round(d['size_sweep']['inception_v3@4096']['hios_lp_ms'],3))"
+done
 done
