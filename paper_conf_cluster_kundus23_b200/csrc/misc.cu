@@ -4,6 +4,9 @@
 // for cross-GPU edges (a10/a11).  NHWC with a pixel stride; each thread owns
 // one pixel x VEC channels (16-byte vectors: 8 bf16 or 4 fp32) so a warp reads
 // contiguous 512-byte runs.
+#include <algorithm>
+#include <type_traits>
+
 #include "kernels.cuh"
 
 namespace hios {
@@ -140,17 +143,25 @@ __global__ void __launch_bounds__(256) pool_tiled_kernel(const PoolArgs<T> a) {
     const int cv = e & 1, pix = e >> 1;
     const int row = pix / IW, col = pix - row * IW;
     const int h = hb + row, w = wb + col, c = c0 + cv * N;
-    float v[N];
-    if (h >= 0 && h < a.H && w >= 0 && w < a.W && c < a.C) {
-      load8(a.x + ((size_t)h * a.W + w) * a.ldx + c, c, a.C, v);
-    } else {
-#pragma unroll
-      for (int j = 0; j < N; ++j) v[j] = pad;
-    }
     const int pos = a.sw == 2 ? ((col & 1) * half + (col >> 1)) : col;
     T* d = reinterpret_cast<T*>(psm + ((size_t)(cv * IH + row) * IW + pos) * VB);
+    const bool inb = h >= 0 && h < a.H && w >= 0 && w < a.W && c < a.C;
+    if (inb && c + N <= a.C) {
+      // whole vector in bounds: raw 16-byte copies, no conversions
+      const uint4* src = reinterpret_cast<const uint4*>(a.x + ((size_t)h * a.W + w) * a.ldx + c);
 #pragma unroll
-    for (int j = 0; j < N; ++j) d[j] = from_f<T>(v[j]);
+      for (int u = 0; u < VB / 16; ++u) reinterpret_cast<uint4*>(d)[u] = src[u];
+    } else {
+      float v[N];
+      if (inb) {
+        load8(a.x + ((size_t)h * a.W + w) * a.ldx + c, c, a.C, v);
+      } else {
+#pragma unroll
+        for (int j = 0; j < N; ++j) v[j] = pad;
+      }
+#pragma unroll
+      for (int j = 0; j < N; ++j) d[j] = from_f<T>(v[j]);
+    }
   }
   __syncthreads();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -158,6 +169,44 @@ __global__ void __launch_bounds__(256) pool_tiled_kernel(const PoolArgs<T> a) {
   const int q = q0 + lane, c = c0 + cv * N;
   if (q >= a.Q || c >= a.C) return;
   const uint8_t* plane = psm + (size_t)cv * IH * IW * VB;
+  if constexpr (std::is_same<T, bf16>::value && KS > 0) {
+    if (a.is_max) {
+      // bf16 max is exact: packed __hmax2 on the staged vectors (no
+      // conversions; -inf padding compares like any value)
+#pragma unroll
+      for (int k = 0; k < 2; ++k) {
+        const int pl = pr0 + 4 * k, p = p0 + pl;
+        if (p >= a.P) break;
+        __nv_bfloat162 m[4];
+#pragma unroll
+        for (int r = 0; r < KS; ++r) {
+          const int row = pl * a.sh + r;
+#pragma unroll
+          for (int s2 = 0; s2 < KS; ++s2) {
+            const int col = lane * a.sw + s2;
+            const int pos = a.sw == 2 ? ((col & 1) * half + (col >> 1)) : col;
+            const uint4 u = *reinterpret_cast<const uint4*>(plane + ((size_t)row * IW + pos) * VB);
+            const __nv_bfloat162* b = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) m[j] = (r == 0 && s2 == 0) ? b[j] : __hmax2(m[j], b[j]);
+          }
+        }
+        const size_t pix = (size_t)p * a.Q + q;
+        const uint4 o = *reinterpret_cast<const uint4*>(m);
+        if (c + 8 <= a.C) {
+          *reinterpret_cast<uint4*>(a.out + pix * a.ldo + c) = o;
+          if (a.out2) *reinterpret_cast<uint4*>(a.out2 + pix * a.ldo2 + c) = o;
+        } else {
+          const bf16* e = reinterpret_cast<const bf16*>(&o);
+          for (int j = 0; j < 8 && c + j < a.C; ++j) {
+            a.out[pix * a.ldo + c + j] = e[j];
+            if (a.out2) a.out2[pix * a.ldo2 + c + j] = e[j];
+          }
+        }
+      }
+      return;
+    }
+  }
 #pragma unroll
   for (int k = 0; k < 2; ++k) {
     const int pl = pr0 + 4 * k, p = p0 + pl;
@@ -210,13 +259,96 @@ static void launch_pool_tiled(const PoolArgs<T>& a, size_t smem, cudaStream_t st
   launch_pdl(pool_tiled_kernel<T, KS>, grid, dim3(256), smem, st, a);
 }
 
+// Row-streaming 3x3 pooling (stride SS = 1 or 2): a thread owns one output
+// column x one 16-byte channel vector and walks a strip of TP output rows
+// down the image, keeping the horizontal 3-tap reductions of the last three
+// input rows in registers, so every input row is read from HBM once per
+// strip (the horizontal neighbours come from L1: adjacent columns are
+// adjacent threads of the same warp) and each output vector is written once,
+// coalesced -- (1 + 2/TP) x input + 1 x output bytes per launch.
+template <typename T, int SS>
+__global__ void __launch_bounds__(256) pool_rows_kernel(const PoolArgs<T> a, int TP) {
+  pdl_enter();
+  constexpr int N = Vec<T>::N;
+  const int CG = (a.C + N - 1) / N;
+  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= (long long)a.Q * CG) return;
+  const int q = (int)(idx / CG), cg = (int)(idx - (long long)q * CG), c = cg * N;
+  const int p0 = blockIdx.y * TP, p1 = min(a.P, p0 + TP);
+  const int w0 = q * SS - a.pw;
+  const bool is_max = a.is_max != 0;
+  const float pad = is_max ? -INFINITY : 0.f;
+  auto hrow = [&](int h, float* o) {
+#pragma unroll
+    for (int j = 0; j < N; ++j) o[j] = pad;
+    if (h < 0 || h >= a.H) return;
+    const T* rp = a.x + (size_t)h * a.W * a.ldx + c;
+#pragma unroll
+    for (int s = 0; s < 3; ++s) {
+      const int w = w0 + s;
+      if (w < 0 || w >= a.W) continue;
+      float v[N];
+      load_vec(rp + (size_t)w * a.ldx, c, a.C, v);
+#pragma unroll
+      for (int j = 0; j < N; ++j) o[j] = is_max ? fmaxf(o[j], v[j]) : o[j] + v[j];
+    }
+  };
+  float r0[N], r1[N], r2[N];
+  int h = p0 * SS - a.ph;
+  hrow(h, r0);
+  hrow(h + 1, r1);
+  hrow(h + 2, r2);
+  const int wlo = max(w0, 0), whi = min(w0 + 3, a.W);
+  for (int p = p0; p < p1; ++p) {
+    float acc[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j)
+      acc[j] = is_max ? fmaxf(fmaxf(r0[j], r1[j]), r2[j]) : r0[j] + r1[j] + r2[j];
+    if (!is_max) {
+      int div;
+      if (a.cip) div = (min(h + 3, a.H + a.ph) - h) * (min(w0 + 3, a.W + a.pw) - w0);
+      else div = (min(h + 3, a.H) - max(h, 0)) * (whi - wlo);
+      const float inv = 1.f / (float)div;
+#pragma unroll
+      for (int j = 0; j < N; ++j) acc[j] *= inv;
+    }
+    if (p + 1 < p1) {  // next rows' loads issued ahead of this row's store
+      if (SS == 1) {
+#pragma unroll
+        for (int j = 0; j < N; ++j) { r0[j] = r1[j]; r1[j] = r2[j]; }
+        hrow(h + 3, r2);
+      } else {
+#pragma unroll
+        for (int j = 0; j < N; ++j) r0[j] = r2[j];
+        hrow(h + 3, r1);
+        hrow(h + 4, r2);
+      }
+    }
+    const size_t pix = (size_t)p * a.Q + q;
+    store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
+    if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+    h += SS;
+  }
+}
+
 template <typename T>
 void launch_pool(const PoolArgs<T>& a, cudaStream_t st) {
   constexpr int N = Vec<T>::N;
+  if (a.kh == 3 && a.kw == 3 && a.sh == a.sw && (a.sh == 1 || a.sh == 2) && getenv("HIOS_POOL_ROWS")) {
+    // strip height: >= ~2 waves of 2048-thread SMs, at most 16 rows
+    const long long cols = (long long)a.Q * ((a.C + N - 1) / N);
+    const int TP = (int)std::max(1LL, std::min(16LL, cols * a.P / (148LL * 2048 * 2)));
+    dim3 grid(grid_for(cols, 256), (a.P + TP - 1) / TP);
+    if (a.sh == 1) launch_pdl(pool_rows_kernel<T, 1>, grid, dim3(256), 0, st, a, TP);
+    else launch_pdl(pool_rows_kernel<T, 2>, grid, dim3(256), 0, st, a, TP);
+    return;
+  }
   const size_t smem = (size_t)2 * ((kPoolTP - 1) * a.sh + a.kh) * ((kPoolTQ - 1) * a.sw + a.kw) * 8 * sizeof(T);
   // measured (tools/op_micro.py, B200): tiled 3x3/s1 avgpool 139 us vs 187 us
   // direct; 3x3/s2 maxpool 297 us vs 205 us direct -- stride 1 only
-  if (a.sw == 1 && a.sh == 1 && a.kh * a.kw > 1 && smem <= 200 * 1024 && !getenv("HIOS_POOL_OLD")) {
+  static const bool s2_tiled = getenv("HIOS_POOL_S2TILED") != nullptr;
+  if (((a.sw == 1 && a.sh == 1) || (s2_tiled && a.sw == 2 && a.sh == 2)) && a.kh * a.kw > 1 && smem <= 200 * 1024 &&
+      !getenv("HIOS_POOL_OLD")) {
     if (a.kh == 3 && a.kw == 3) return launch_pool_tiled<T, 3>(a, smem, st);
     return launch_pool_tiled<T, 0>(a, smem, st);
   }

@@ -81,9 +81,12 @@ int main() {
   cudaFuncSetAttribute(tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
   struct Cfg { const char* name; int b1, b2; uint32_t C_dim; };
   std::vector<Cfg> cfgs = {{"box {64,128,1} 16KB", 128, 1, (uint32_t)C},
-                           {"box {64,32,1} 4KB", 32, 1, (uint32_t)C}};
+                           {"box {64,32,1} 4KB", 32, 1, (uint32_t)C},
+                           {"box {64,64,2} 16KB", 64, 2, (uint32_t)C},
+                           {"box {64,128,2} 32KB", 128, 2, (uint32_t)C},
+                           {"box {64,64,8} 64KB", 64, 8, (uint32_t)C}};
   for (auto& c : cfgs) {
-    for (int depth : {8}) for (int lm : {0, 1}) for (int issuers : {1, 2, 4, 8}) {
+    for (int depth : {3, 8}) for (int lm : {0, 1}) for (int issuers : {1, 2, 4, 8}) {
       if (issuers > depth) continue;
       if (!lm && issuers > 4) continue;
       CUtensorMap m;
