@@ -300,3 +300,34 @@ def test_ios_on_benchmark_dags_not_worse_than_hios_m1():
         hios.hios_set_group_model(G, 7, 10)
         L_ios = hios.hios_schedule_latency_ns(hios.hios_schedule_ios(G, 4))
         assert L_ios <= hios.hios_schedule_latency_ns(hios.hios_schedule_lp(G, 1, 4))
+
+
+def test_simulation_study_trends():
+    """Figs. 7, 10, 11 trends through the C-ABI on the
+    §V generator (4 seeds; tools/sim_study.py runs the full sweeps): HIOS-LP's
+    speedup over sequential grows with the number of GPUs and beats HIOS-MR
+    from 4 GPUs on; HIOS-LP latency falls as the layer count falls (more
+    parallelism); its speedup falls as the transfer/compute ratio p grows.
+    (Magnitudes differ from the paper's: its generator is underspecified, C18,
+    DESIGN.md §10.)"""
+    def mean_lat(M=4, layers=14, p=0.8, kind="lp", seeds=4):
+        tot = 0
+        for seed in range(seeds):
+            n, t, E = S.random_dag(200, layers, None, p, seed, unit=1000)
+            G, N, t_all, E_all = _cost_graph(n, t, E)
+            hios.hios_set_group_model(G, 9, 10)
+            if kind == "seq":
+                s = hios.hios_schedule_lp(G, 1, 1)
+            elif kind == "mr":
+                s = hios.hios_schedule_mr(G, M, 3)
+            else:
+                s = hios.hios_schedule_lp(G, M, 3)
+            tot += hios.hios_schedule_latency_ns(s)
+        return tot / seeds
+    seq = mean_lat(kind="seq")
+    sp = [seq / mean_lat(M=m) for m in (2, 4, 8)]
+    assert sp[0] < sp[1] < sp[2]                                    # Fig. 7
+    assert mean_lat(M=4) < mean_lat(M=4, kind="mr")                # Fig. 7/8: LP beats MR
+    assert mean_lat(M=8) < mean_lat(M=8, kind="mr")
+    assert mean_lat(layers=6) < mean_lat(layers=14) < mean_lat(layers=22)   # Fig. 10
+    assert mean_lat(p=0.4, seeds=12) < mean_lat(p=1.2, seeds=12)   # Fig. 11
