@@ -66,7 +66,7 @@ __global__ void bench(int tiles, int taps, int n, int variant, unsigned long lon
   // warp index via shfl from lane 0: provably warp-uniform for ptxas (as
   // CUTLASS's canonical_warp_idx_sync), so the role branch is not divergent
   const int warp_u = variant >= 3 ? __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0) : (int)(threadIdx.x >> 5);
-  if (variant >= 8 && threadIdx.x < 32) {
+  if (variant >= 8 && variant < 10 && threadIdx.x < 32) {
     long long t0 = clock64();
     int cnt = 0;
     if (threadIdx.x == 0) {
@@ -102,16 +102,28 @@ __global__ void bench(int tiles, int taps, int n, int variant, unsigned long lon
     wait_asm(smem_u32(&done), 0);
     long long t2 = clock64();
     if (blockIdx.x == 0 && threadIdx.x == 0) { out[0] = t1 - t0; out[1] = t2 - t0; out[2] = cnt; }
-  } else if ((variant >= 3 && warp_u == 0) || (variant < 3 && threadIdx.x < 32)) {
+  } else if ((variant >= 3 && variant < 8 && warp_u == 0) || (variant >= 10 && warp_u == 0) || (variant < 3 && threadIdx.x < 32)) {
     const uint32_t on = elect_one() ? 1u : 0u;
     long long t0 = clock64();
     int cnt = 0;
     for (int tile = 0; tile < tiles; ++tile) {
-      const uint32_t d = tm + (uint32_t)(tile & 1) * 64u;
-      if (variant == 0 || variant == 3) wait_asm(smem_u32(&bar), 0); else wait_vote(smem_u32(&bar), 0);
+      const uint32_t d = (variant >= 10 ? 0u : tm) + (uint32_t)(tile & 1) * 64u;
+      if (variant == 0 || variant == 3 || variant >= 10) wait_asm(smem_u32(&bar), 0); else wait_vote(smem_u32(&bar), 0);
       uint64_t aoff = 0;
       uint32_t accum = 0;
       const uint64_t ad0 = desc(a0), bd0 = desc(b0);
+      if (variant == 11) {
+        // runtime tap loop, TMEM base a compile-time 0
+        for (int t = 0; t < taps; ++t) {
+          const uint64_t ad = ad0 + aoff, bd = bd0 + (uint64_t)(t & 3) * (uint64_t)(n * 8);
+          mma_pred(d, ad, bd, idesc, accum, on);
+          mma_pred(d, ad + 2, bd + 2, idesc, 1u, on);
+          accum = 1;
+          aoff += (t % 3 == 2) ? 65u : 8u;
+          cnt += 2;
+        }
+        continue;
+      }
       if (variant >= 6) {
         // fully unrolled 3x3: every descriptor = per-chunk base + compile-time offset
 #pragma unroll
@@ -158,7 +170,7 @@ int main() {
   unsigned long long* d;
   cudaMalloc(&d, 32);
   cudaFuncSetAttribute(bench, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-  for (int variant : {0, 6, 8, 9})
+  for (int variant : {0, 6, 10, 11})
     for (int n : {32, 128}) {
       bench<<<148, 128, 140 * 1024>>>(64, 9, n, variant, d);
       bench<<<148, 128, 140 * 1024>>>(64, 9, n, variant, d);
