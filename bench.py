@@ -533,6 +533,7 @@ def main():
             "frac": achieved / peak_t if peak_t else None, "traffic": traffic,
             "launches_per_step": len(conv_ids),
             "flops_per_launch": conv_flops / max(len(conv_ids), 1),
+            "algorithmic_bytes_per_launch": float(B[conv_ids].sum()) / max(len(conv_ids), 1),
             "avg_launch_us": conv_s / max(len(conv_ids), 1) * 1e6,
             "share_of_step": conv_s * 1e3 / step_r if step_r > 0 else None,
             "best_launch": None if best is None else {
