@@ -283,8 +283,15 @@ __global__ void __launch_bounds__(kThreads, 1)
   float* s_scale = reinterpret_cast<float*>(bars + 2 * ST + kBarX + 2);  // [kScaleRes]
   float* s_shift = s_scale + kScaleRes;                            // [kScaleRes]
 
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const uint32_t ncols = tmem_cols(2 * a.n_tile);
+  // warp index via a shuffle from lane 0: provably warp-uniform for ptxas, so
+  // role-derived values (MMA sub-tile, TMEM column, B descriptor) stay in
+  // uniform registers (CUTLASS canonical_warp_idx_sync)
+  const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0), lane = threadIdx.x & 31;
+  // the whole TMEM (512 columns): one conv CTA per SM (164 registers x 384
+  // threads), so the allocation is always column 0 -- a compile-time TMEM
+  // base keeps the MMA issue loop's accumulator address in uniform registers
+  // (measured: a loaded base was re-broadcast with R2UR per MMA)
+  const uint32_t ncols = 512;
   const int RS = a.R * a.S;
   const int tiles_mn = a.tiles_m * a.tiles_n;
   const int tiles = tiles_mn * a.ksplit;  // split-K: each split owns a chunk range
@@ -322,7 +329,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
+  if (*tmem_slot != 0u) __trap();  // cannot happen with one CTA per SM
+  const uint32_t tmem = 0u;
   if (threadIdx.x == 0) TRACE(1);
   // Programmatic dependent launch: the set-up above (barriers, TMEM,
   // descriptor prefetch) overlapped the previous kernel's tail; inputs are
@@ -451,7 +459,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t on = elect_one() ? 1u : 0u;
         const uint32_t ST_ = (uint32_t)ST;
         const uint64_t row_r16 = row_r >> 4, row_s16 = row_s >> 4, b16 = B_BYTES >> 4, bst16 = B_STAGE >> 4;
-        const uint64_t bres0 = umma_desc_sw128(sB0);
+        const uint64_t bres0 = umma_desc_sw128(sB0), bD0h = bres0;
         for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
           mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
           tc_fence_after();
@@ -471,7 +479,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               if (!bres) {
                 mbar_wait(full0 + 8 * st, ph);
                 tc_fence_after();
-                b0 = umma_desc_sw128(sB0 + st * B_STAGE);
+                b0 = bD0h + (uint64_t)st * bst16;
               } else {
                 b0 = bres0 + (uint64_t)(cc * RS + t) * b16;
               }

@@ -393,7 +393,9 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   const size_t stage_out = 128 * ((size_t)c.n_tile * 2 + 16);
   // epilogue: two staging tiles for N tiles <= 128 (the stores of tile i
   // drain while tile i+1 is staged), folded BN resident when K is small
-  c.occ = (getenv("HIOS_OCC") ? atoi(getenv("HIOS_OCC")) : 1) == 2 && c.n_tile <= 128 ? 2 : 1;
+  // one CTA per SM: 164 registers x 384 threads (the kernel also takes the
+  // whole TMEM on that basis)
+  c.occ = 1;
   // epilogue mode (HIOS_EPI overrides): direct register stores for N tiles
   // <= 128 (no staging tile), TMA bulk-tensor stores for wider tiles
   c.epi = getenv("HIOS_EPI") ? atoi(getenv("HIOS_EPI")) : (c.n_tile <= 128 ? 2 : 1);
