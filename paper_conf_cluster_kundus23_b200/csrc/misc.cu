@@ -508,6 +508,148 @@ __global__ void __launch_bounds__(256) dw_tiled_kernel(const DwArgs<T> a) {
   }
 }
 
+// Register-blocked depthwise for bf16 (KS x KS, stride SS): the CTA stages
+// the same bf16 input window as dw_tiled_kernel (TP = 4 * KR output rows x 32
+// columns x 16 channels) plus the weights rounded to bf16; a thread owns KR
+// vertically adjacent output rows of one column and 8 channels.  For each
+// kernel column s it holds the KS weight vectors of that column in registers
+// and walks the (KR - 1) * SS + KS input rows its outputs touch, loading each
+// staged vector once and feeding it to every output row that uses it (the
+// tiled kernel re-read it per output and per tap: shared-memory bound).
+// fma.rn.f32.bf16 (FHFMA.BF16, sm_100) multiplies the bf16 halves directly
+// into fp32 accumulators: no conversions in the inner loop.
+__device__ __forceinline__ float fma_bf16_lo(uint32_t x, uint32_t w, float c) {
+  float d;
+  asm("{\n.reg .b16 xl, xh, wl, wh;\nmov.b32 {xl, xh}, %1;\nmov.b32 {wl, wh}, %2;\n"
+      "fma.rn.f32.bf16 %0, xl, wl, %3;\n}\n" : "=f"(d) : "r"(x), "r"(w), "f"(c));
+  return d;
+}
+__device__ __forceinline__ float fma_bf16_hi(uint32_t x, uint32_t w, float c) {
+  float d;
+  asm("{\n.reg .b16 xl, xh, wl, wh;\nmov.b32 {xl, xh}, %1;\nmov.b32 {wl, wh}, %2;\n"
+      "fma.rn.f32.bf16 %0, xh, wh, %3;\n}\n" : "=f"(d) : "r"(x), "r"(w), "f"(c));
+  return d;
+}
+
+template <int KS, int SS, int KR>
+__global__ void __launch_bounds__(256) dw_reg_kernel(const DwArgs<bf16> a) {
+  extern __shared__ __align__(16) uint8_t dsm[];
+  constexpr int TP = 4 * KR, N = 8, VB = 16;
+  constexpr int IH = (TP - 1) * SS + KS, IW = (kDwTQ - 1) * SS + KS;
+  constexpr int HALF = (IW + 1) / 2;
+  constexpr int NH = (KR - 1) * SS + KS;  // input rows one thread touches
+  const int q0 = blockIdx.y * kDwTQ, p0 = blockIdx.z * TP, c0 = blockIdx.x * 16;
+  uint8_t* swb = dsm;                                   // [KS*KS][16] bf16 weights
+  uint8_t* tile = dsm + (size_t)KS * KS * 32;           // [2][IH][IW] bf16 vectors
+  for (int i = threadIdx.x; i < KS * KS * 16; i += blockDim.x) {
+    const int rs = i >> 4, j = i & 15;
+    reinterpret_cast<bf16*>(swb)[i] =
+        __float2bfloat16_rn((c0 + j < a.C) ? __ldg(a.w + (size_t)rs * a.C + c0 + j) : 0.f);
+  }
+  pdl_enter();
+  const int hb = p0 * SS - a.ph, wb = q0 * SS - a.pw;
+  for (int e = threadIdx.x; e < 2 * IH * IW; e += blockDim.x) {
+    const int cv = e & 1, pix = e >> 1;
+    const int row = pix / IW, col = pix - row * IW;
+    const int h = hb + row, w = wb + col, c = c0 + cv * N;
+    float u[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) u[j] = 0.f;
+    if (h >= 0 && h < a.H && w >= 0 && w < a.W && c < a.C) {
+      const size_t off = (size_t)h * a.W + w;
+      for (int i = 0; i < a.n_in; ++i) {
+        float v[N];
+        load8(a.x[i] + off * a.ldx[i] + c, c, a.C, v);
+#pragma unroll
+        for (int j = 0; j < N; ++j) u[j] += a.agg[i] * v[j];
+      }
+      if (a.pre_relu) {
+#pragma unroll
+        for (int j = 0; j < N; ++j) u[j] = fmaxf(u[j], 0.f);
+      }
+    }
+    const int pos = SS == 2 ? ((col & 1) * HALF + (col >> 1)) : col;
+    uint4 pk;
+    __nv_bfloat162* b2 = reinterpret_cast<__nv_bfloat162*>(&pk);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) b2[j] = __floats2bfloat162_rn(u[2 * j], u[2 * j + 1]);
+    *reinterpret_cast<uint4*>(tile + ((size_t)(cv * IH + row) * IW + pos) * VB) = pk;
+  }
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int cv = warp & 1, pr0 = warp >> 1;
+  const uint8_t* plane = tile + (size_t)cv * IH * IW * VB + (size_t)(pr0 * KR * SS) * IW * VB;
+  float acc[KR][N];
+#pragma unroll
+  for (int k = 0; k < KR; ++k)
+#pragma unroll
+    for (int j = 0; j < N; ++j) acc[k][j] = 0.f;
+#pragma unroll 1
+  for (int s = 0; s < KS; ++s) {
+    uint4 wr[KS];
+#pragma unroll
+    for (int r = 0; r < KS; ++r) wr[r] = *reinterpret_cast<const uint4*>(swb + (size_t)(r * KS + s) * 32 + cv * 16);
+    const int col = lane * SS + s;
+    const int pos = SS == 2 ? ((col & 1) * HALF + (col >> 1)) : col;
+    const uint8_t* src = plane + (size_t)pos * VB;
+#pragma unroll
+    for (int hh = 0; hh < NH; ++hh) {
+      const uint4 x = *reinterpret_cast<const uint4*>(src + (size_t)hh * IW * VB);
+#pragma unroll
+      for (int k = 0; k < KR; ++k) {
+        const int r = hh - k * SS;
+        if (r < 0 || r >= KS) continue;
+        acc[k][0] = fma_bf16_lo(x.x, wr[r].x, acc[k][0]); acc[k][1] = fma_bf16_hi(x.x, wr[r].x, acc[k][1]);
+        acc[k][2] = fma_bf16_lo(x.y, wr[r].y, acc[k][2]); acc[k][3] = fma_bf16_hi(x.y, wr[r].y, acc[k][3]);
+        acc[k][4] = fma_bf16_lo(x.z, wr[r].z, acc[k][4]); acc[k][5] = fma_bf16_hi(x.z, wr[r].z, acc[k][5]);
+        acc[k][6] = fma_bf16_lo(x.w, wr[r].w, acc[k][6]); acc[k][7] = fma_bf16_hi(x.w, wr[r].w, acc[k][7]);
+      }
+    }
+  }
+  const int q = q0 + lane, c = c0 + cv * N;
+  if (q >= a.Q || c >= a.C) return;
+#pragma unroll
+  for (int k = 0; k < KR; ++k) {
+    const int p = p0 + pr0 * KR + k;
+    if (p < a.P) store8(a.out + ((size_t)p * a.Q + q) * a.ldo + c, c, a.C, acc[k]);
+  }
+}
+
+template <int KS, int SS, int KR>
+static void launch_dw_reg(const DwArgs<bf16>& a, cudaStream_t st) {
+  constexpr int TP = 4 * KR;
+  constexpr size_t smem = (size_t)KS * KS * 32 + (size_t)2 * ((TP - 1) * SS + KS) * ((kDwTQ - 1) * SS + KS) * 16;
+  static bool attr_set[64] = {false};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 64 && !attr_set[dev]) {
+    cudaFuncSetAttribute(dw_reg_kernel<KS, SS, KR>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    attr_set[dev] = true;
+  }
+  dim3 grid((a.C + 15) / 16, (a.Q + kDwTQ - 1) / kDwTQ, (a.P + TP - 1) / TP);
+  launch_pdl(dw_reg_kernel<KS, SS, KR>, grid, dim3(256), smem, st, a);
+}
+
+// bf16, square 3/5/7 kernels, stride 1 or 2: the register-blocked kernel
+// (4 rows per thread at stride 1, 2 at stride 2)
+template <typename T>
+static bool try_dw_reg(const DwArgs<T>&, cudaStream_t) { return false; }
+template <>
+bool try_dw_reg<bf16>(const DwArgs<bf16>& a, cudaStream_t st) {
+  static const bool off = getenv("HIOS_DW_NOREG") != nullptr;
+  if (off || a.R != a.S || a.sh != a.sw || (a.sh != 1 && a.sh != 2)) return false;
+  if (a.sh == 1) {
+    if (a.R == 3) { launch_dw_reg<3, 1, 4>(a, st); return true; }
+    if (a.R == 5) { launch_dw_reg<5, 1, 4>(a, st); return true; }
+    if (a.R == 7) { launch_dw_reg<7, 1, 4>(a, st); return true; }
+  } else {
+    if (a.R == 3) { launch_dw_reg<3, 2, 2>(a, st); return true; }
+    if (a.R == 5) { launch_dw_reg<5, 2, 2>(a, st); return true; }
+    if (a.R == 7) { launch_dw_reg<7, 2, 2>(a, st); return true; }
+  }
+  return false;
+}
+
 template <typename T, int KS>
 static void launch_dw_tiled(const DwArgs<T>& a, size_t smem, cudaStream_t st) {
   static bool attr_set[64] = {false};
@@ -526,6 +668,7 @@ void launch_dw(const DwArgs<T>& a, cudaStream_t st) {
   constexpr int N = Vec<T>::N;
   const size_t smem = (size_t)a.R * a.S * 16 * sizeof(float) +
                       (size_t)2 * dw_tile_rows(a.R, a.sh) * dw_tile_cols(a.S, a.sw) * 8 * sizeof(T);
+  if (try_dw_reg(a, st)) return;
   if ((a.sw == 1 || a.sw == 2) && smem <= 200 * 1024 && !getenv("HIOS_DW_OLD")) {
     if (a.R == 3 && a.S == 3) return launch_dw_tiled<T, 3>(a, smem, st);
     if (a.R == 5 && a.S == 5) return launch_dw_tiled<T, 5>(a, smem, st);
