@@ -62,6 +62,32 @@ __device__ __forceinline__ void store8(T* p, int c, int C, const float* v) {
     if (c + h < C) store_vec(p + h, c + h, C, v + h);
 }
 
+// mixed-precision bf16 x fp32 arithmetic (sm_100: FHFMA.BF16 / FHADD.BF16 read
+// either bf16 half of a register directly -- no conversions)
+__device__ __forceinline__ float fma_bf16_lo(uint32_t x, uint32_t w, float c) {
+  float d;
+  asm("{\n.reg .b16 xl, xh, wl, wh;\nmov.b32 {xl, xh}, %1;\nmov.b32 {wl, wh}, %2;\n"
+      "fma.rn.f32.bf16 %0, xl, wl, %3;\n}\n" : "=f"(d) : "r"(x), "r"(w), "f"(c));
+  return d;
+}
+__device__ __forceinline__ float fma_bf16_hi(uint32_t x, uint32_t w, float c) {
+  float d;
+  asm("{\n.reg .b16 xl, xh, wl, wh;\nmov.b32 {xl, xh}, %1;\nmov.b32 {wl, wh}, %2;\n"
+      "fma.rn.f32.bf16 %0, xh, wh, %3;\n}\n" : "=f"(d) : "r"(x), "r"(w), "f"(c));
+  return d;
+}
+
+__device__ __forceinline__ float add_bf16_lo(uint32_t x, float c) {
+  float d;
+  asm("{\n.reg .b16 xl, xh;\nmov.b32 {xl, xh}, %1;\nadd.rn.f32.bf16 %0, xl, %2;\n}\n" : "=f"(d) : "r"(x), "f"(c));
+  return d;
+}
+__device__ __forceinline__ float add_bf16_hi(uint32_t x, float c) {
+  float d;
+  asm("{\n.reg .b16 xl, xh;\nmov.b32 {xl, xh}, %1;\nadd.rn.f32.bf16 %0, xh, %2;\n}\n" : "=f"(d) : "r"(x), "f"(c));
+  return d;
+}
+
 static inline unsigned grid_for(long long n, int block) {
   long long g = (n + block - 1) / block;
   return (unsigned)(g < 1 ? 1 : g);
@@ -203,6 +229,42 @@ __global__ void __launch_bounds__(256) pool_tiled_kernel(const PoolArgs<T> a) {
             if (a.out2) a.out2[pix * a.ldo2 + c + j] = e[j];
           }
         }
+      }
+      return;
+    }
+    {
+      // average: FHADD.BF16 straight from the staged bf16 pairs into fp32
+#pragma unroll
+      for (int k = 0; k < 2; ++k) {
+        const int pl = pr0 + 4 * k, p = p0 + pl;
+        if (p >= a.P) break;
+        float acc[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[j] = 0.f;
+#pragma unroll
+        for (int r = 0; r < KS; ++r) {
+          const int row = pl * a.sh + r;
+#pragma unroll
+          for (int s2 = 0; s2 < KS; ++s2) {
+            const int col = lane * a.sw + s2;
+            const int pos = a.sw == 2 ? ((col & 1) * half + (col >> 1)) : col;
+            const uint4 u = *reinterpret_cast<const uint4*>(plane + ((size_t)row * IW + pos) * VB);
+            acc[0] = add_bf16_lo(u.x, acc[0]); acc[1] = add_bf16_hi(u.x, acc[1]);
+            acc[2] = add_bf16_lo(u.y, acc[2]); acc[3] = add_bf16_hi(u.y, acc[3]);
+            acc[4] = add_bf16_lo(u.z, acc[4]); acc[5] = add_bf16_hi(u.z, acc[5]);
+            acc[6] = add_bf16_lo(u.w, acc[6]); acc[7] = add_bf16_hi(u.w, acc[7]);
+          }
+        }
+        const int h0 = p * a.sh - a.ph, w0 = q * a.sw - a.pw;
+        int div;
+        if (a.cip) div = (min(h0 + kh, a.H + a.ph) - h0) * (min(w0 + kw, a.W + a.pw) - w0);
+        else div = (min(h0 + kh, a.H) - max(h0, 0)) * (min(w0 + kw, a.W) - max(w0, 0));
+        const float inv = 1.f / (float)div;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[j] *= inv;
+        const size_t pix = (size_t)p * a.Q + q;
+        store8(a.out + pix * a.ldo + c, c, a.C, acc);
+        if (a.out2) store8(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
       }
       return;
     }
@@ -518,19 +580,6 @@ __global__ void __launch_bounds__(256) dw_tiled_kernel(const DwArgs<T> a) {
 // tiled kernel re-read it per output and per tap: shared-memory bound).
 // fma.rn.f32.bf16 (FHFMA.BF16, sm_100) multiplies the bf16 halves directly
 // into fp32 accumulators: no conversions in the inner loop.
-__device__ __forceinline__ float fma_bf16_lo(uint32_t x, uint32_t w, float c) {
-  float d;
-  asm("{\n.reg .b16 xl, xh, wl, wh;\nmov.b32 {xl, xh}, %1;\nmov.b32 {wl, wh}, %2;\n"
-      "fma.rn.f32.bf16 %0, xl, wl, %3;\n}\n" : "=f"(d) : "r"(x), "r"(w), "f"(c));
-  return d;
-}
-__device__ __forceinline__ float fma_bf16_hi(uint32_t x, uint32_t w, float c) {
-  float d;
-  asm("{\n.reg .b16 xl, xh, wl, wh;\nmov.b32 {xl, xh}, %1;\nmov.b32 {wl, wh}, %2;\n"
-      "fma.rn.f32.bf16 %0, xh, wh, %3;\n}\n" : "=f"(d) : "r"(x), "r"(w), "f"(c));
-  return d;
-}
-
 template <int KS, int SS, int KR>
 __global__ void __launch_bounds__(256) dw_reg_kernel(const DwArgs<bf16> a) {
   extern __shared__ __align__(16) uint8_t dsm[];
