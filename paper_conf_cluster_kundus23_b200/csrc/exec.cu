@@ -138,7 +138,7 @@ void Executor::plan() {
     if (o.kind == HIOS_OP_CONV && g.dtype == HIOS_BF16 && s2d_conv(o)) {
       OpExec& x = ox[v];
       x.s2d_ldc = rup(4 * o.in_c, 8);
-      x.s2dbuf = alloc(l, (int64_t)(o.H + (o.kh + 1) / 2 - 1) * (o.W + (o.kw + 1) / 2 - 1) * x.s2d_ldc * esz);
+      x.s2dbuf = alloc(l, ((int64_t)(o.H + (o.kh + 1) / 2 - 1) * (o.W + (o.kw + 1) / 2 - 1) + 4) * x.s2d_ldc * esz);
     }
     if (o.kind == HIOS_OP_SEPCONV) {
       OpExec& x = ox[v];
@@ -229,6 +229,17 @@ static void upload_weights_T(Executor& ex, int v) {
                     to_dev_t<T>(o.weight[(((size_t)k * C + c) * o.kh + r) * o.kw + s2]);
               }
         x.w = upload(L, w2);
+        if (Cp2 == 16 && S2 <= 4) {
+          // packed taps: one 64-element K row per r' = S2 taps x 16 channels
+          // (zero weights for the taps s' >= S2 the 4-pixel window also covers)
+          std::vector<T> w3((size_t)o.out_c * R2 * 64, to_dev_t<T>(0.f));
+          for (int k = 0; k < o.out_c; ++k)
+            for (int r2 = 0; r2 < R2; ++r2)
+              for (int s2 = 0; s2 < S2; ++s2)
+                for (int ch = 0; ch < 16; ++ch)
+                  w3[((size_t)k * R2 + r2) * 64 + s2 * 16 + ch] = w2[((size_t)k * R2 * S2 + r2 * S2 + s2) * Cp2 + ch];
+          x.w_pack = upload(L, w3);
+        }
         x.scale.push_back((float*)upload(L, o.scale));
         x.shift.push_back((float*)upload(L, o.shift));
         break;
@@ -469,6 +480,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
 struct View {
   char* p;
   int ldc;
+  int row_px = 0;  // pixels per row for the row pitch (0: the conv's W)
 };
 
 template <typename T>
@@ -493,10 +505,10 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   CUtensorMap mx, mw;
   bool ok;
   if (a.halo)  // R input rows (stride dh) x halo_w pixels per channel chunk
-    ok = make_tmap_3d(&mx, in.p, C, W, H, (uint64_t)in.ldc * 2, (uint64_t)W * in.ldc * 2, 64, a.halo_w, R * dh, 1,
+    ok = make_tmap_3d(&mx, in.p, C, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w, R * dh, 1,
                       dh);
   else         // th x tw output positions of one (r, s) tap, conv stride as traversal stride
-    ok = make_tmap_3d(&mx, in.p, C, W, H, (uint64_t)in.ldc * 2, (uint64_t)W * in.ldc * 2, 64, a.tw * sw, a.th * sh,
+    ok = make_tmap_3d(&mx, in.p, C, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.tw * sw, a.th * sh,
                       sw, sh);
   if (!ok) fail(HIOS_E_CUDA, "tensor map (activation)");
   const int Cp = rup(C, 8);
@@ -593,8 +605,17 @@ static void build_op(Executor& ex, int v) {
         S2dArgs<T> d{(const T*)iv.p, xi.H, xi.W, xi.C, iv.ldc, o.ph, o.pw, (T*)sv.p, H2, W2, sv.ldc};
         fns.push_back([d](cudaStream_t st) { launch_s2d<T>(d, st); });
         ++nk;
-        fns.push_back(conv_closure<T>(ex, sv, H2, W2, 4 * xi.C, x.w, x.scale[0], x.shift[0], o.out_c, R2, S2, 1, 1,
-                                      0, 0, 1, 1, o.H, o.W, o.relu, out, out2, nk));
+        static const bool nopack = getenv("HIOS_NOPACK") != nullptr;
+        if (x.w_pack && !nopack) {
+          // packed taps: a virtual 64-channel input whose pixel j is the
+          // 4-pixel window j..j+3 of the s2d tensor (pixel stride 32 B)
+          View pv{sv.p, sv.ldc, W2};
+          fns.push_back(conv_closure<T>(ex, pv, H2, o.W, 64, x.w_pack, x.scale[0], x.shift[0], o.out_c, R2, 1, 1, 1,
+                                        0, 0, 1, 1, o.H, o.W, o.relu, out, out2, nk));
+        } else {
+          fns.push_back(conv_closure<T>(ex, sv, H2, W2, 4 * xi.C, x.w, x.scale[0], x.shift[0], o.out_c, R2, S2, 1, 1,
+                                        0, 0, 1, 1, o.H, o.W, o.relu, out, out2, nk));
+        }
         break;
       }
       if (small_c_conv(o)) {

@@ -28,6 +28,9 @@ struct OpExec {
   // stride-2 small-C stem (bf16): space-to-depth copy of the input (arena offset)
   int64_t s2dbuf = -1;
   int s2d_ldc = 0;
+  // s2d stem with its S' taps packed into one 64-element K row (overlapping
+  // 4-pixel windows of the s2d tensor; weights W''[k][r'][s'*16 + ch])
+  void* w_pack = nullptr;
   // remote deliveries of this op's output: (consumer lgpu, fused-into-epilogue?)
   std::vector<std::pair<int, bool>> remote;
   std::function<void(cudaStream_t)> run;  // enqueue the op's kernels (incl. fused out2)

@@ -936,13 +936,16 @@ template <typename T>
 __global__ void s2d_kernel(const S2dArgs<T> a) {
   pdl_enter();
   const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= (long long)a.P2 * a.Q2) return;
+  // 4 zero pixels of slack past the end (packed-tap windows of the last row)
+  if (idx >= (long long)a.P2 * a.Q2 + 4) return;
+  const bool tail = idx >= (long long)a.P2 * a.Q2;
   const int i = (int)(idx / a.Q2), j = (int)(idx - (long long)i * a.Q2);
   T v[16];
 #pragma unroll
   for (int e = 0; e < 16; ++e) v[e] = from_f<T>(0.f);
 #pragma unroll
   for (int ab = 0; ab < 4; ++ab) {
+    if (tail) break;
     const int h = 2 * i + (ab >> 1) - a.ph, w = 2 * j + (ab & 1) - a.pw;
     if (h < 0 || h >= a.H || w < 0 || w >= a.W) continue;
     const T* src = a.x + ((size_t)h * a.W + w) * a.ldx;
@@ -958,7 +961,7 @@ __global__ void s2d_kernel(const S2dArgs<T> a) {
 
 template <typename T>
 void launch_s2d(const S2dArgs<T>& a, cudaStream_t st) {
-  launch_pdl(s2d_kernel<T>, dim3(grid_for((long long)a.P2 * a.Q2, 256)), dim3(256), 0, st, a);
+  launch_pdl(s2d_kernel<T>, dim3(grid_for((long long)a.P2 * a.Q2 + 4, 256)), dim3(256), 0, st, a);
 }
 
 // explicit instantiations

@@ -85,6 +85,8 @@ CONV_CASES = [
     (3, 96, 45, 260, 3, 3, 2, 1, 1),      # NASNet-like conv0 with padding
     (3, 39, 33, 37, 3, 3, 2, 1, 1),       # RandWire conv1: K = 39 (ragged N), tap mode
     (2, 24, 30, 31, 5, 5, 2, 2, 2),       # C = 2, 5x5 (taps past R, S in W')
+    (4, 32, 41, 300, 3, 3, 2, 0, 0),      # C = 4: packed taps (S' = 2 < 4), halo mode
+    (3, 64, 300, 35, 5, 5, 2, 2, 2),      # packed taps (S' = 3), tap mode (narrow output)
     # halo mode with resident weights (one N tile, > 148 output tiles per CTA wave)
     (32, 32, 160, 200, 3, 3, 1, 1, 1),
     (64, 80, 150, 130, 1, 1, 1, 0, 0),

@@ -26,6 +26,9 @@ SHAPES = [
     ("nas_sep5_cell0", "sepconv", 168, 256, 256, dict(k=5, s=1, K=168, reps=2)),
     ("nas_sep7s2_red0", "sepconv", 336, 256, 256, dict(k=7, s=2, K=336, reps=2)),
     ("rw_sep3_n5", "sepconv", 78, 256, 256, dict(k=3, s=1, K=78, reps=1, n_in=4)),
+    ("sq_conv1", "conv", 3, 2048, 2048, dict(K=96, k=7, s=2, p=0)),
+    ("rw_conv1", "conv", 3, 2048, 2048, dict(K=39, k=3, s=2, p=1)),
+    ("rw_conv2", "conv", 39, 1024, 1024, dict(K=78, k=3, s=2, p=1)),
     ("i4096_conv1a", "conv", 3, 4096, 4096, dict(K=32, k=3, s=2, p=0)),
     ("i4096_conv5d1x1", "conv", 288, 509, 509, dict(K=64, k=1, s=1, p=0)),
     ("i4096_conv7c1x1", "conv", 2048, 126, 126, dict(K=384, k=1, s=1, p=0)),
