@@ -100,7 +100,9 @@ void Executor::plan() {
   std::vector<int64_t> cursor(M, 0);
   auto alloc = [&](int l, int64_t bytes) {
     int64_t off = cursor[l];
-    cursor[l] += rup64(std::max<int64_t>(bytes, 16), 256);
+    // +128 B of (zeroed) slack: a conv whose C is not a multiple of 64 reads
+    // its last chunk as overlapping 64-channel windows (see conv_closure)
+    cursor[l] += rup64(std::max<int64_t>(bytes, 16) + 128, 256);
     return off;
   };
   // reverse topological order: a concat consumer's buffer exists before its producers are placed
@@ -215,10 +217,10 @@ static void upload_weights_T(Executor& ex, int v) {
   const bool tc = ex.g.dtype == HIOS_BF16;
   switch (o.kind) {
     case HIOS_OP_CONV: {
-      const int Cp = tc ? rup(o.in_c, 8) : o.in_c;
+      const int Cp = tc ? rup(o.in_c, 64) : o.in_c;  // bf16: whole 64-channel chunks (zero-padded)
       if (tc && s2d_conv(o)) {
         // W'[k][r'*S'+s'][(a*2+b)*C + c] (see s2d_conv)
-        const int R2 = (o.kh + 1) / 2, S2 = (o.kw + 1) / 2, C = o.in_c, Cp2 = rup(4 * C, 8);
+        const int R2 = (o.kh + 1) / 2, S2 = (o.kw + 1) / 2, C = o.in_c, Cp2 = rup(4 * C, 64);
         std::vector<T> w2((size_t)o.out_c * R2 * S2 * Cp2, to_dev_t<T>(0.f));
         for (int k = 0; k < o.out_c; ++k)
           for (int c = 0; c < C; ++c)
@@ -229,7 +231,7 @@ static void upload_weights_T(Executor& ex, int v) {
                     to_dev_t<T>(o.weight[(((size_t)k * C + c) * o.kh + r) * o.kw + s2]);
               }
         x.w = upload(L, w2);
-        if (Cp2 == 16 && S2 <= 4) {
+        if (rup(4 * C, 8) == 16 && S2 <= 4) {
           // packed taps: one 64-element K row per r' = S2 taps x 16 channels
           // (zero weights for the taps s' >= S2 the 4-pixel window also covers)
           std::vector<T> w3((size_t)o.out_c * R2 * 64, to_dev_t<T>(0.f));
@@ -260,7 +262,7 @@ static void upload_weights_T(Executor& ex, int v) {
           for (int rs = 0; rs < RS; ++rs) dw[(size_t)rs * c + ch] = o.weight[off + (size_t)ch * RS + rs];
         off += (size_t)c * RS;
         x.dw.push_back((float*)upload(L, dw));
-        const int Cp = tc ? rup(c, 8) : c;
+        const int Cp = tc ? rup(c, 64) : c;
         x.pw.push_back(upload(L, conv_layout<T>(o.weight.data() + off, o.out_c, c, 1, 1, Cp)));
         off += (size_t)o.out_c * c;
         std::vector<float> sc(o.scale.begin() + (size_t)r * o.out_c, o.scale.begin() + (size_t)(r + 1) * o.out_c);
@@ -504,14 +506,24 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   }
   CUtensorMap mx, mw;
   bool ok;
+  // C % 64 != 0: the tensor map's channel extent is rounded up to whole
+  // 64-channel chunks, so the last chunk's box reads past C into the pixel's
+  // pad / the next pixel (finite data -- the arena is zeroed and every buffer
+  // has 128 B of slack) instead of being zero-filled by TMA: measured
+  // (tools/tma_bench.cu) a box with channel out-of-bounds fill streams at
+  // ~16 B/cycle/SM whatever the number of issuing warps, 2-7x slower than an
+  // in-bounds box.  Those channels meet zero weights (pitch rup(C, 64)) or are
+  // skipped (K=16 slices past C are not issued).
+  static const bool nopad = getenv("HIOS_NOCHANPAD") != nullptr;
+  const int Cm = (C % 64 && !nopad) ? rup(C, 64) : C;
   if (a.halo)  // R input rows (stride dh) x halo_w pixels per channel chunk
-    ok = make_tmap_3d(&mx, in.p, C, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w, R * dh, 1,
+    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w, R * dh, 1,
                       dh);
   else         // th x tw output positions of one (r, s) tap, conv stride as traversal stride
-    ok = make_tmap_3d(&mx, in.p, C, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.tw * sw, a.th * sh,
+    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.tw * sw, a.th * sh,
                       sw, sh);
   if (!ok) fail(HIOS_E_CUDA, "tensor map (activation)");
-  const int Cp = rup(C, 8);
+  const int Cp = rup(C, 64);  // weight pitch: whole zero-padded 64-channel chunks (no TMA OOB fill)
   if (!make_tmap_3d(&mw, w, Cp, R * S, K, (uint64_t)Cp * 2, (uint64_t)R * S * Cp * 2, 64, 1, a.n_tile, 1, 1))
     fail(HIOS_E_CUDA, "tensor map (weights)");
   a.P = P; a.Q = Q; a.K = K; a.C = C; a.R = R; a.S = S; a.sh = sh; a.sw = sw; a.ph = ph; a.pw = pw;

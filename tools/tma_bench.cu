@@ -72,33 +72,36 @@ int main() {
   cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q);
   PFN_encodeTiled enc = (PFN_encodeTiled)p;
   // 2048 channels x 64 x 64 pixels bf16 activation (like a deep NHWC layer), 16 MB
-  const int C = 2048, W = 64, H = 64;
+  const int C = 2048, W = 512, H = 64;
   void* buf;
   cudaMalloc(&buf, (size_t)C * W * H * 2);
   cudaMemset(buf, 0, (size_t)C * W * H * 2);
   unsigned long long* cyc;
   cudaMalloc(&cyc, 148 * 8);
   cudaFuncSetAttribute(tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
-  struct Cfg { const char* name; int b1, b2; uint32_t C_dim; };
+  struct Cfg { const char* name; int b1, b2; uint32_t C_dim; int es1 = 1; };
   std::vector<Cfg> cfgs = {{"box {64,128,1} 16KB", 128, 1, (uint32_t)C},
                            {"box {64,32,1} 4KB", 32, 1, (uint32_t)C},
                            {"box {64,64,2} 16KB", 64, 2, (uint32_t)C},
                            {"box {64,128,2} 32KB", 128, 2, (uint32_t)C},
+                           {"box {64,128,1} 16KB C=40", 128, 1, 40u},
+                           {"box {64,256/2,1} 16KB es2", 256, 1, (uint32_t)C, 2},
+                           {"box {64,256/2,1} es2 C=40", 256, 1, 40u, 2},
                            {"box {64,64,8} 64KB", 64, 8, (uint32_t)C}};
   for (auto& c : cfgs) {
-    for (int depth : {3, 8}) for (int lm : {0, 1}) for (int issuers : {1, 2, 4, 8}) {
+    for (int depth : {8}) for (int lm : {0}) for (int issuers : {1, 2, 4}) {
       if (issuers > depth) continue;
       if (!lm && issuers > 4) continue;
       CUtensorMap m;
       cuuint64_t dims[3] = {c.C_dim, (cuuint64_t)W, (cuuint64_t)H};
       cuuint64_t strides[2] = {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2};
       cuuint32_t box[3] = {64, (cuuint32_t)c.b1, (cuuint32_t)c.b2};
-      cuuint32_t es[3] = {1, 1, 1};
+      cuuint32_t es[3] = {1, (cuuint32_t)c.es1, 1};
       CUresult r = enc(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, buf, dims, strides, box, es,
                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
       if (r != CUDA_SUCCESS) { printf("encode failed %d\n", r); continue; }
-      uint32_t bytes = 128u * c.b1 * c.b2;
+      uint32_t bytes = 128u * (c.b1 / c.es1) * c.b2;
       if ((size_t)depth * bytes > 200 * 1024) continue;
       size_t smem = 1024 + depth * bytes + depth * 8;
       int iters = 400;
