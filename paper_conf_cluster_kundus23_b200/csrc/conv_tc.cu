@@ -176,6 +176,23 @@ __device__ __forceinline__ void mma_commit(uint32_t bar) {
                : "memory");
 }
 
+// halo mode, resident weights: one chunk's R_ x S_ taps (kv K=16 slices
+// each) with compile-time window offsets r * row_r16 + s * row_s16
+template <int R_, int S_>
+__device__ __forceinline__ void halo_taps_bres(uint32_t d, uint64_t a0, uint64_t b0, uint32_t idesc, int kv,
+                                               uint32_t on, uint64_t row_r16, uint64_t row_s16, uint64_t b16,
+                                               uint32_t accum) {
+#pragma unroll
+  for (int t = 0; t < R_ * S_; ++t) {
+    const uint64_t ad = a0 + (uint64_t)(t / S_) * row_r16 + (uint64_t)(t % S_) * row_s16;
+    const uint64_t bd = b0 + (uint64_t)t * b16;
+    mma_bf16_on(d, ad, bd, idesc, t == 0 ? accum : 1u, on);
+    if (kv > 1) mma_bf16_on(d, ad + 2, bd + 2, idesc, 1u, on);
+    if (kv > 2) mma_bf16_on(d, ad + 4, bd + 4, idesc, 1u, on);
+    if (kv > 3) mma_bf16_on(d, ad + 6, bd + 6, idesc, 1u, on);
+  }
+}
+
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
@@ -383,8 +400,12 @@ __global__ void __launch_bounds__(kThreads, 1)
             mbar_wait(aempty0 + 8 * ab, aph ^ 1u);
             if (elect_one()) {
               if (a.bres) TRACE2(0, hcount);
-              mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.R * a.halo_w * 128u);
-              tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, cc * 64, x0, y0);
+              if (a.dbg & 4) {  // timing experiment: no halo loads (stale smem)
+                mbar_arrive(afull0 + 8 * ab);
+              } else {
+                mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.R * a.halo_w * 128u);
+                tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, cc * 64, x0, y0);
+              }
             }
             __syncwarp();
           }
@@ -460,6 +481,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t ST_ = (uint32_t)ST;
         const uint64_t row_r16 = row_r >> 4, row_s16 = row_s >> 4, b16 = B_BYTES >> 4, bst16 = B_STAGE >> 4;
         const uint64_t bres0 = umma_desc_sw128(sB0), bD0h = bres0;
+        const bool fixed_rs = !(a.dbg & 32) && ((a.R == 3 && a.S == 3) || (a.R == 1 && a.S == 1) ||
+                                                (a.R == 2 && a.S == 1) || (a.R == 4 && a.S == 1) ||
+                                                (a.R == 5 && a.S == 5));
         for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
           mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
           tc_fence_after();
@@ -471,6 +495,21 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (bres && lane == 0 && j == 0) TRACE2(1, tcount);
             const uint64_t a0 = umma_desc_sw128(sA0 + ab * H_BYTES);
             const int kv = min(4, (C - cc * 64 + 15) >> 4);
+            if (bres && fixed_rs) {
+              // resident weights, common kernel shapes: the chunk's taps fully
+              // unrolled with compile-time window offsets (descriptor adds on
+              // the uniform datapath, no loop-carried offsets)
+              const uint64_t bc = bres0 + (uint64_t)(cc * RS) * b16;
+              if (a.R == 3 && S_ == 3) halo_taps_bres<3, 3>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
+              else if (a.R == 1 && S_ == 1) halo_taps_bres<1, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
+              else if (a.R == 2 && S_ == 1) halo_taps_bres<2, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
+              else if (a.R == 4 && S_ == 1) halo_taps_bres<4, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
+              else halo_taps_bres<5, 5>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
+              accum = 1;
+              mma_commit_on(aempty0 + 8 * ab, on);
+              if (++ab == (uint32_t)abufs) { ab = 0; aph ^= 1u; }
+              continue;
+            }
             uint64_t aoff_r = 0, aoff = 0;
             int s_ = 0;
             for (int t = 0; t < RS;) {
@@ -651,6 +690,14 @@ __global__ void __launch_bounds__(kThreads, 1)
       TRACE5(0, tcount);
       if (tcount == 0 && warp == kEpiWarp0 && lane == 0) TRACE(5);
       const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)a.n_tile;
+      if (a.dbg & 16) {  // timing experiment: accumulator released unread
+        tc_fence_before();
+        mbar_arrive(tempty0 + 8 * acc);
+        TRACE5(1, tcount);
+        acc ^= 1u;
+        if (acc == 0) tph ^= 1u;
+        continue;
+      }
       if (a.epi == 2) {
         // direct stores: each thread owns one output pixel (its TMEM lane)
         // and writes its n_valid channels as 16-byte vectors straight from
