@@ -35,6 +35,10 @@ struct OpExec {
   std::vector<std::pair<int, bool>> remote;
   std::function<void(cudaStream_t)> run;  // enqueue the op's kernels (incl. fused out2)
   int n_kernels = 0;
+  // the same op configured to run alone (a singleton stage / t(v) profiling):
+  // tap-mode convs take narrower N tiles there (more CTAs); empty = run
+  std::function<void(cudaStream_t)> run_solo;
+  int n_kernels_solo = 0;
 };
 
 struct LGpu {

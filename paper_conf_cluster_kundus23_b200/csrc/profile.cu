@@ -126,7 +126,7 @@ std::shared_ptr<Profiler> run_profile(std::shared_ptr<Graph> G, const int32_t* d
   }
   for (int v : g.topo) {
     if (v == g.input_op) continue;
-    g.ops[v].cost = impl->time_ns(E.ox[v].run, st);
+    g.ops[v].cost = impl->time_ns(E.ox[v].run_solo ? E.ox[v].run_solo : E.ox[v].run, st);
   }
   // t(u, v): push of u's output into a buffer on the peer device (or a second buffer here)
   const int peer = n_devices > 1 ? devices[1] : dev0;

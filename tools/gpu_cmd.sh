@@ -1,4 +1,5 @@
 cd $GRAFT_REPO_ROOT
-timeout 900 python -m pytest tests -x -q -m gpu -k "conv or end_to_end or bench_config" 2>&1 | tail -2
-for d in 32 0; do echo "== DBG $d"; HIOS_DBG=$d timeout 300 python tools/op_micro.py i4096_conv sq_conv1 rw_conv1 2>&1 | cut -c1-60; HIOS_DBG=$d timeout 300 python tools/conv_trace2.py i4096_conv2a 2>&1 | sed -n 2,6p; done
-timeout 900 python bench.py --steps 20 --no-cpu-baseline 2>/dev/null > gpurun_out/b.json; python -c "import json; d=json.loads(open('gpurun_out/b.json').read()); print('bench', round(d['value'],4), {k: (round(v['hios_lp_ms'],3), round(v['cp_frac'],3)) for k,v in d['size_sweep'].items()})"
+for v in cur head cur; do
+  if [ $v = head ]; then export HIOS_LIB=$PWD/ab/libhios_head.so; else unset HIOS_LIB; fi
+  timeout 900 python bench.py --steps 30 --no-cpu-baseline --sweep "4096,nasnet_a_large@2048,randwire_ws@2048,squeezenet@2048" 2>/dev/null > gpurun_out/b.json; python -c "import json; d=json.loads(open('gpurun_out/b.json').read()); print('$v bench', round(d['value'],4), 'seq', round(d['single_gpu_refs']['sequential']['ms'],4), 'ios', round(d['single_gpu_refs']['ios']['ms'],4), {k: (round(v['hios_lp_ms'],3), round(v['cp_frac'],3)) for k,v in d['size_sweep'].items()})"
+done
