@@ -176,6 +176,33 @@ __device__ __forceinline__ void mma_commit(uint32_t bar) {
                : "memory");
 }
 
+// halo mode, B ring: one chunk's R_ x S_ taps, KPS_ taps per ring stage
+template <int R_, int S_, int KPS_>
+__device__ __forceinline__ void halo_taps_ring(uint32_t d, uint64_t a0, uint64_t bD0, uint64_t bst16, uint64_t b16,
+                                               uint32_t idesc, int kv, uint32_t on, uint64_t row_r16,
+                                               uint64_t row_s16, uint32_t accum, uint32_t& st, uint32_t& ph,
+                                               uint32_t ST, uint32_t full0, uint32_t empty0) {
+  uint64_t b0 = 0;
+#pragma unroll
+  for (int t = 0; t < R_ * S_; ++t) {
+    if (t % KPS_ == 0) {
+      mbar_wait(full0 + 8 * st, ph);
+      tc_fence_after();
+      b0 = bD0 + (uint64_t)st * bst16;
+    }
+    const uint64_t ad = a0 + (uint64_t)(t / S_) * row_r16 + (uint64_t)(t % S_) * row_s16;
+    const uint64_t bd = b0 + (uint64_t)(t % KPS_) * b16;
+    mma_bf16_on(d, ad, bd, idesc, t == 0 ? accum : 1u, on);
+    if (kv > 1) mma_bf16_on(d, ad + 2, bd + 2, idesc, 1u, on);
+    if (kv > 2) mma_bf16_on(d, ad + 4, bd + 4, idesc, 1u, on);
+    if (kv > 3) mma_bf16_on(d, ad + 6, bd + 6, idesc, 1u, on);
+    if (t % KPS_ == KPS_ - 1 || t == R_ * S_ - 1) {
+      mma_commit_on(empty0 + 8 * st, on);
+      if (++st == ST) { st = 0; ph ^= 1u; }
+    }
+  }
+}
+
 // halo mode, resident weights: one chunk's R_ x S_ taps (kv K=16 slices
 // each) with compile-time window offsets r * row_r16 + s * row_s16
 template <int R_, int S_>
@@ -481,6 +508,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t ST_ = (uint32_t)ST;
         const uint64_t row_r16 = row_r >> 4, row_s16 = row_s >> 4, b16 = B_BYTES >> 4, bst16 = B_STAGE >> 4;
         const uint64_t bres0 = umma_desc_sw128(sB0), bD0h = bres0;
+        const bool fixed_ring = !(a.dbg & 32) && ((a.R == 3 && a.S == 3 && KPS >= 2 && KPS <= 4) ||
+                                                  (a.R == 5 && a.S == 5 && KPS == 4) ||
+                                                  (a.R == 1 && a.S == 1 && KPS == 1));
         const bool fixed_rs = !(a.dbg & 32) && ((a.R == 3 && a.S == 3) || (a.R == 1 && a.S == 1) ||
                                                 (a.R == 2 && a.S == 1) || (a.R == 4 && a.S == 1) ||
                                                 (a.R == 5 && a.S == 5));
@@ -505,6 +535,20 @@ __global__ void __launch_bounds__(kThreads, 1)
               else if (a.R == 2 && S_ == 1) halo_taps_bres<2, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
               else if (a.R == 4 && S_ == 1) halo_taps_bres<4, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
               else halo_taps_bres<5, 5>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
+              accum = 1;
+              mma_commit_on(aempty0 + 8 * ab, on);
+              if (++ab == (uint32_t)abufs) { ab = 0; aph ^= 1u; }
+              continue;
+            }
+            if (!bres && fixed_ring) {
+              // B ring, common shapes: the chunk's taps unrolled with
+              // compile-time window offsets; stage waits / releases at
+              // compile-time tap boundaries (kps taps per stage)
+              if (a.R == 3 && kps == 3) halo_taps_ring<3, 3, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 3 && kps == 2) halo_taps_ring<3, 3, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 3 && kps == 4) halo_taps_ring<3, 3, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 5 && kps == 4) halo_taps_ring<5, 5, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else halo_taps_ring<1, 1, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
               accum = 1;
               mma_commit_on(aempty0 + 8 * ab, on);
               if (++ab == (uint32_t)abufs) { ab = 0; aph ^= 1u; }
