@@ -360,7 +360,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--model", default="inception_v3")
     ap.add_argument("--size", type=int, default=1024)
-    ap.add_argument("--window", type=int, default=4)
+    ap.add_argument("--window", type=int, default=5)
     ap.add_argument("--dtype", default="bf16")
     ap.add_argument("--impl", default="hios", choices=["hios", "reference"])
     ap.add_argument("--cpu-budget", type=float, default=15.0)

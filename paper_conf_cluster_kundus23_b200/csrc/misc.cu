@@ -775,8 +775,19 @@ __global__ void copy_kernel(const CopyArgs<T> a) {
   T* dst = a.out + pix * a.ldo + c;
   // concat slices at channel offsets that are not multiples of 8 are not
   // 16-byte aligned: fall back to element copies there
-  if (c + N <= a.C && ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15) == 0) {
+  const uintptr_t al = reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst);
+  if (c + N <= a.C && (al & 15) == 0) {
     *reinterpret_cast<uint4*>(dst) = *reinterpret_cast<const uint4*>(src);
+  } else if (c + N <= a.C && (al & 7) == 0) {
+    const uint2* s2 = reinterpret_cast<const uint2*>(src);
+    uint2* d2 = reinterpret_cast<uint2*>(dst);
+    d2[0] = s2[0]; d2[1] = s2[1];
+  } else if (c + N <= a.C && (al & 3) == 0) {
+    // even channel offsets (e.g. NASNet's 42-channel concat slices): words
+    const uint32_t* s4 = reinterpret_cast<const uint32_t*>(src);
+    uint32_t* d4 = reinterpret_cast<uint32_t*>(dst);
+    const uint32_t w0 = s4[0], w1 = s4[1], w2 = s4[2], w3 = s4[3];
+    d4[0] = w0; d4[1] = w1; d4[2] = w2; d4[3] = w3;
   } else {
     for (int j = 0; j < N && c + j < a.C; ++j) dst[j] = src[j];
   }
