@@ -136,14 +136,18 @@ SEP_CASES = [
     (168, 168, 20, 33, 5, 1, 1, 2),       # NASNet cell: 5x5, several 16-channel slabs
     (20, 24, 19, 37, 4, 2, 2, 1),         # generic kernel size (even), stride 2, aggregation
     (336, 336, 17, 9, 7, 2, 1, 2),        # deep, narrow (tile mostly padding)
+    (84, 84, 37, 41, 5, 2, 1, 2),         # register-blocked dw 5x5/s2 (2 rows per thread)
+    (30, 32, 50, 19, 3, 2, 3, 1),         # 3x3/s2 with aggregation, C % 8 != 0
+    (48, 48, 35, 66, 7, 1, 1, 1),         # 7x7/s1: 16-row CTA tiles, ragged last tile
 ]
 
 
 @pytest.mark.parametrize("dtype", ["bf16", "f32"])
 @pytest.mark.parametrize("case", SEP_CASES)
 def test_sepconv_parity(dtype, case):
-    """Depthwise (smem-tiled kernel) + pointwise per repetition, per-op check
-    and end to end."""
+    """Depthwise (bf16: register-blocked FHFMA kernel for square 3/5/7 and
+    stride 1/2, else smem-tiled; fp32: smem-tiled) + pointwise per
+    repetition, per-op check and end to end."""
     C, K, H, Wd, k, s, n_in, reps = case
     g = graphs.GraphSpec("sep", C, H, Wd)
     x0 = g.input()
