@@ -108,6 +108,36 @@ __global__ void pool_kernel(const PoolArgs<T> a) {
   const int q = idx / CG, cg = idx - q * CG;
   const int c = cg * N;
   const int h0 = p * a.sh - a.ph, w0 = q * a.sw - a.pw;
+  if constexpr (std::is_same<T, bf16>::value && KH == 3 && KW == 3) {
+    if (a.is_max && c + 8 <= a.C) {
+      // bf16 3x3 max, whole vector: all in-bounds taps' loads issued first,
+      // then packed __hmax2 (exact in bf16; no conversions)
+      uint4 u[9];
+      bool ok[9];
+#pragma unroll
+      for (int t = 0; t < 9; ++t) {
+        const int h = h0 + t / 3, w = w0 + t % 3;
+        ok[t] = h >= 0 && h < a.H && w >= 0 && w < a.W;
+        if (ok[t]) u[t] = __ldg(reinterpret_cast<const uint4*>(a.x + ((size_t)h * a.W + w) * a.ldx + c));
+      }
+      __nv_bfloat162 m[4];
+      const __nv_bfloat162 ninf = __floats2bfloat162_rn(-INFINITY, -INFINITY);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) m[j] = ninf;
+#pragma unroll
+      for (int t = 0; t < 9; ++t) {
+        if (!ok[t]) continue;
+        const __nv_bfloat162* b = reinterpret_cast<const __nv_bfloat162*>(&u[t]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) m[j] = __hmax2(m[j], b[j]);
+      }
+      const size_t pix = (size_t)p * a.Q + q;
+      const uint4 o = *reinterpret_cast<const uint4*>(m);
+      *reinterpret_cast<uint4*>(a.out + pix * a.ldo + c) = o;
+      if (a.out2) *reinterpret_cast<uint4*>(a.out2 + pix * a.ldo2 + c) = o;
+      return;
+    }
+  }
   float acc[N], v[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) acc[j] = a.is_max ? -INFINITY : 0.f;
