@@ -137,6 +137,38 @@ __global__ void pool_kernel(const PoolArgs<T> a) {
       if (a.out2) *reinterpret_cast<uint4*>(a.out2 + pix * a.ldo2 + c) = o;
       return;
     }
+    if (!a.is_max && c + 8 <= a.C) {
+      // bf16 3x3 average: loads first, then FHADD.BF16 into fp32
+      uint4 u[9];
+      bool ok[9];
+#pragma unroll
+      for (int t = 0; t < 9; ++t) {
+        const int h = h0 + t / 3, w = w0 + t % 3;
+        ok[t] = h >= 0 && h < a.H && w >= 0 && w < a.W;
+        if (ok[t]) u[t] = __ldg(reinterpret_cast<const uint4*>(a.x + ((size_t)h * a.W + w) * a.ldx + c));
+      }
+      float acc[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) acc[j] = 0.f;
+#pragma unroll
+      for (int t = 0; t < 9; ++t) {
+        if (!ok[t]) continue;
+        acc[0] = add_bf16_lo(u[t].x, acc[0]); acc[1] = add_bf16_hi(u[t].x, acc[1]);
+        acc[2] = add_bf16_lo(u[t].y, acc[2]); acc[3] = add_bf16_hi(u[t].y, acc[3]);
+        acc[4] = add_bf16_lo(u[t].z, acc[4]); acc[5] = add_bf16_hi(u[t].z, acc[5]);
+        acc[6] = add_bf16_lo(u[t].w, acc[6]); acc[7] = add_bf16_hi(u[t].w, acc[7]);
+      }
+      int div;
+      if (a.cip) div = (min(h0 + 3, a.H + a.ph) - h0) * (min(w0 + 3, a.W + a.pw) - w0);
+      else div = (min(h0 + 3, a.H) - max(h0, 0)) * (min(w0 + 3, a.W) - max(w0, 0));
+      const float inv = 1.f / (float)div;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) acc[j] *= inv;
+      const size_t pix = (size_t)p * a.Q + q;
+      store8(a.out + pix * a.ldo + c, c, a.C, acc);
+      if (a.out2) store8(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+      return;
+    }
   }
   float acc[N], v[N];
 #pragma unroll
@@ -438,6 +470,18 @@ void launch_pool(const PoolArgs<T>& a, cudaStream_t st) {
   const size_t smem = (size_t)2 * ((kPoolTP - 1) * a.sh + a.kh) * ((kPoolTQ - 1) * a.sw + a.kw) * 8 * sizeof(T);
   // measured (tools/op_micro.py, B200): tiled 3x3/s1 avgpool 139 us vs 187 us
   // direct; 3x3/s2 maxpool 297 us vs 205 us direct -- stride 1 only
+  // bf16 3x3: the direct kernel with all tap loads in flight (measured faster
+  // than the smem-tiled kernel; HIOS_POOL_TILED3 keeps the tiled one)
+  // measured: direct wins for stride 2 and for small stride-1 pools (Mixed_6/7
+  // at 1024^2), the tiled kernel for large stride-1 average pools
+  static const bool tiled3 = getenv("HIOS_POOL_TILED3") != nullptr;
+  const bool big_s1 = a.sh == 1 && (long long)a.P * a.Q * a.C >= (4LL << 20);
+  if (std::is_same<T, bf16>::value && a.kh == 3 && a.kw == 3 && !tiled3 && !big_s1) {
+    const int per_row = a.Q * ((a.C + N - 1) / N);
+    dim3 grid((per_row + 255) / 256, a.P);
+    launch_pdl(pool_kernel<T, 3, 3>, grid, dim3(256), 0, st, a);
+    return;
+  }
   static const bool s2_tiled = getenv("HIOS_POOL_S2TILED") != nullptr;
   if (((a.sw == 1 && a.sh == 1) || (s2_tiled && a.sw == 2 && a.sh == 2)) && a.kh * a.kw > 1 && smem <= 200 * 1024 &&
       !getenv("HIOS_POOL_OLD")) {
