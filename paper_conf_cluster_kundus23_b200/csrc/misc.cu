@@ -671,7 +671,42 @@ __global__ void __launch_bounds__(256) dw_reg_kernel(const DwArgs<bf16> a) {
   }
   pdl_enter();
   const int hb = p0 * SS - a.ph, wb = q0 * SS - a.pw;
-  for (int e = threadIdx.x; e < 2 * IH * IW; e += blockDim.x) {
+  // single input, both 8-channel vectors in bounds: the staging loads of four
+  // rounds are issued before any is used (latency overlap), values kept in
+  // bf16 (scale 1: exact; ReLU as packed max)
+  const bool fast = a.n_in == 1 && c0 + 16 <= a.C && a.agg[0] == 1.f;
+  constexpr int NEL = 2 * IH * IW, NB = 4;
+  for (int e0 = fast ? (int)threadIdx.x : NEL; e0 < NEL; e0 += NB * 256) {
+    uint4 raw[NB];
+    int dst[NB];
+#pragma unroll
+    for (int b = 0; b < NB; ++b) {
+      const int e = e0 + b * 256;
+      dst[b] = -1;
+      raw[b] = make_uint4(0u, 0u, 0u, 0u);
+      if (e >= NEL) continue;
+      const int cv = e & 1, pix = e >> 1;
+      const int row = pix / IW, col = pix - row * IW;
+      const int h = hb + row, w = wb + col;
+      const int pos = SS == 2 ? ((col & 1) * HALF + (col >> 1)) : col;
+      dst[b] = (cv * IH + row) * IW + pos;
+      if (h >= 0 && h < a.H && w >= 0 && w < a.W)
+        raw[b] = __ldg(reinterpret_cast<const uint4*>(a.x[0] + ((size_t)h * a.W + w) * a.ldx[0] + c0 + cv * N));
+    }
+#pragma unroll
+    for (int b = 0; b < NB; ++b) {
+      if (dst[b] < 0) continue;
+      uint4 v = raw[b];
+      if (a.pre_relu) {
+        __nv_bfloat162* p2 = reinterpret_cast<__nv_bfloat162*>(&v);
+        const __nv_bfloat162 z = __floats2bfloat162_rn(0.f, 0.f);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) p2[j] = __hmax2(p2[j], z);
+      }
+      *reinterpret_cast<uint4*>(tile + (size_t)dst[b] * VB) = v;
+    }
+  }
+  for (int e = fast ? NEL : (int)threadIdx.x; e < NEL; e += blockDim.x) {
     const int cv = e & 1, pix = e >> 1;
     const int row = pix / IW, col = pix - row * IW;
     const int h = hb + row, w = wb + col, c = c0 + cv * N;
