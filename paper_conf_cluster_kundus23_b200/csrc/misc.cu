@@ -850,6 +850,33 @@ __global__ void add_kernel(const AddArgs<T> a) {
   float acc[N], v[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) acc[j] = 0.f;
+  if constexpr (std::is_same<T, bf16>::value) {
+    if (a.n_in <= 4 && c + 8 <= a.C) {
+      // whole vectors, <= 4 inputs: all loads in flight first
+      uint4 raw[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+        if (i < a.n_in) raw[i] = __ldg(reinterpret_cast<const uint4*>(a.x[i] + pix * a.ldx[i] + c));
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        if (i >= a.n_in) break;
+        const __nv_bfloat162* p2 = reinterpret_cast<const __nv_bfloat162*>(&raw[i]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const float2 f = __bfloat1622float2(p2[j]);
+          acc[2 * j] += a.agg[i] * f.x;
+          acc[2 * j + 1] += a.agg[i] * f.y;
+        }
+      }
+      if (a.relu) {
+#pragma unroll
+        for (int j = 0; j < N; ++j) acc[j] = fmaxf(acc[j], 0.f);
+      }
+      store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
+      if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+      return;
+    }
+  }
   for (int i = 0; i < a.n_in; ++i) {
     load_vec(a.x[i] + pix * a.ldx[i] + c, c, a.C, v);
 #pragma unroll
