@@ -490,7 +490,10 @@ def main():
         t0 = time.perf_counter()
         y = h.hios_run(S, xin if (world == 1 or int(op_gpu[0]) % world == rank or True) else None)
         e2e.append((time.perf_counter() - t0) * 1e3)
-    e2e_ms = max_over_ranks(dist, float(np.mean(e2e[args.warmup:])), world)
+    # median: host-side copies see occasional OS / PCIe stalls (measured: the
+    # mean moved 1.06 -> 1.58 ms between two boxes with the same device time)
+    e2e_ms = max_over_ranks(dist, float(np.median(e2e[args.warmup:])), world)
+    e2e_mean = float(np.mean(e2e[args.warmup:]))
 
     # ---------------- dominant-kernel roofline: per-op device times from the
     # instrumented graph (CUDA events recorded as graph nodes on the launching
@@ -527,6 +530,18 @@ def main():
             traffic = json.load(open(tp)).get("bytes_per_launch")
         except Exception:
             traffic = None
+    # the same convs timed as hios_profile's t(v): median of back-to-back
+    # in-graph replays of the op's kernels (warm L2, no per-op event nodes;
+    # the instrumented graph above records two events around every op)
+    prof = None
+    if rank == 0:
+        tv, _ = h.hios_get_costs(G)
+        conv_tv = np.array([tv[v] for v in conv_ids], dtype=np.float64) * 1e-9
+        if conv_tv.sum() > 0:
+            prof = {"achieved": conv_flops / conv_tv.sum() / 1e12,
+                    "frac": conv_flops / conv_tv.sum() / 1e12 / pk["bf16_tflops_sustained"],
+                    "avg_launch_us": float(conv_tv.mean() * 1e6),
+                    "measured_on": "hios_profile t(v): median of back-to-back in-graph replays (warm L2)"}
     best = max(conv_ids, key=lambda v: F[v] / max(op_ms[v], 1e-9)) if conv_ids else None
     roof = {"bound": "tensor", "kernel": "conv_tc_kernel (tcgen05 implicit GEMM)",
             "achieved": achieved, "peak": peak_t, "unit": "TFLOP/s",
@@ -540,6 +555,7 @@ def main():
                 "op": g.ops[best].name, "us": float(op_ms[best] * 1e3),
                 "tflops": float(F[best] / (op_ms[best] * 1e-3) / 1e12)},
             "measured_on": "sequential schedule, instrumented CUDA graph" if world == 1 else "timed schedule",
+            "profiled": prof,
             "peak_src": f"{pk['src']} bf16 sustained (kernel inside a long step)"}
 
     cp_s = critical_path_bound(g, F, B, op_gpu, op_stage, M, pk, esz, shapes)
@@ -604,7 +620,7 @@ def main():
             "critical_path": {"bound_ms": cp_s * 1e3, "frac": (cp_s * 1e3) / ms if ms > 0 else None,
                               "form": "overlap-edge lower bound, bf16 burst + HBM measured peaks"},
             "cpu_baseline": cpu,
-            "e2e": {"value": e2e_ms, "unit": "ms", "h2d_bytes_per_step": int(x.nbytes),
+            "e2e": {"value": e2e_ms, "stat": "median", "mean": e2e_mean, "unit": "ms", "h2d_bytes_per_step": int(x.nbytes),
                     "d2h_bytes_per_step": int(n_out * 4), "api": "hios_run (pinned host buffers)"},
             "gpu_launches": int(h.hios_kernel_count(S)) * args.steps,
             "clocks": clocks,
