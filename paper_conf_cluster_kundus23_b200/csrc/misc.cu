@@ -370,6 +370,70 @@ __global__ void __launch_bounds__(256) pool_tiled_kernel(const PoolArgs<T> a) {
   }
 }
 
+// 3x3 stride-1 average pool (bf16), 64-channel CTAs: a CTA stages the
+// 10 x 18 input window of 8 x 16 output pixels x 64 channels (128 contiguous
+// bytes per pixel: whole cache lines per load, vs 32-byte pieces in
+// pool_tiled_kernel) and each thread reduces four outputs (columns lane/8 +
+// 4j of row warp, channel vector lane%8) with FHADD.BF16 from smem.
+constexpr int kP64TP = 8, kP64TQ = 16;
+__global__ void __launch_bounds__(256) pool_avg64_kernel(const PoolArgs<bf16> a) {
+  __shared__ __align__(16) uint4 tile[(kP64TP + 2) * (kP64TQ + 2) * 8];
+  const int c0 = blockIdx.x * 64, q0 = blockIdx.y * kP64TQ, p0 = blockIdx.z * kP64TP;
+  pdl_enter();
+  const int hb = p0 - a.ph, wb = q0 - a.pw;
+  constexpr int NEL = (kP64TP + 2) * (kP64TQ + 2) * 8;
+  uint4 raw[6];
+#pragma unroll
+  for (int b = 0; b < 6; ++b) {
+    const int e = threadIdx.x + b * 256;
+    raw[b] = make_uint4(0u, 0u, 0u, 0u);
+    if (e >= NEL) continue;
+    const int cv = e & 7, pix = e >> 3;
+    const int row = pix / (kP64TQ + 2), col = pix - row * (kP64TQ + 2);
+    const int h = hb + row, w = wb + col, c = c0 + cv * 8;
+    if (h >= 0 && h < a.H && w >= 0 && w < a.W && c + 8 <= a.C)
+      raw[b] = __ldg(reinterpret_cast<const uint4*>(a.x + ((size_t)h * a.W + w) * a.ldx + c));
+  }
+#pragma unroll
+  for (int b = 0; b < 6; ++b) {
+    const int e = threadIdx.x + b * 256;
+    if (e < NEL) tile[e] = raw[b];
+  }
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int cv = lane & 7, qq = lane >> 3;
+  const int p = p0 + warp, c = c0 + cv * 8;
+  if (p >= a.P || c >= a.C) return;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const int ql = qq + 4 * j, q = q0 + ql;
+    if (q >= a.Q) break;
+    float acc[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) acc[k] = 0.f;
+#pragma unroll
+    for (int r = 0; r < 3; ++r)
+#pragma unroll
+      for (int s2 = 0; s2 < 3; ++s2) {
+        const uint4 u = tile[((warp + r) * (kP64TQ + 2) + ql + s2) * 8 + cv];
+        acc[0] = add_bf16_lo(u.x, acc[0]); acc[1] = add_bf16_hi(u.x, acc[1]);
+        acc[2] = add_bf16_lo(u.y, acc[2]); acc[3] = add_bf16_hi(u.y, acc[3]);
+        acc[4] = add_bf16_lo(u.z, acc[4]); acc[5] = add_bf16_hi(u.z, acc[5]);
+        acc[6] = add_bf16_lo(u.w, acc[6]); acc[7] = add_bf16_hi(u.w, acc[7]);
+      }
+    const int h0 = p - a.ph, w0 = q - a.pw;
+    int div;
+    if (a.cip) div = (min(h0 + 3, a.H + a.ph) - h0) * (min(w0 + 3, a.W + a.pw) - w0);
+    else div = (min(h0 + 3, a.H) - max(h0, 0)) * (min(w0 + 3, a.W) - max(w0, 0));
+    const float inv = 1.f / (float)div;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) acc[k] *= inv;
+    const size_t pix = (size_t)p * a.Q + q;
+    store8(a.out + pix * a.ldo + c, c, a.C, acc);
+    if (a.out2) store8(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+  }
+}
+
 template <typename T, int KS>
 static void launch_pool_tiled(const PoolArgs<T>& a, size_t smem, cudaStream_t st) {
   static bool attr_set[64] = {false};
@@ -476,6 +540,15 @@ void launch_pool(const PoolArgs<T>& a, cudaStream_t st) {
   // at 1024^2), the tiled kernel for large stride-1 average pools
   static const bool tiled3 = getenv("HIOS_POOL_TILED3") != nullptr;
   const bool big_s1 = a.sh == 1 && (long long)a.P * a.Q * a.C >= (4LL << 20);
+  static const bool no64 = getenv("HIOS_POOL_NO64") != nullptr;
+  if constexpr (std::is_same<T, bf16>::value) {
+    // large stride-1 3x3 average pools with whole 8-channel vectors: 64-channel CTAs
+    if (big_s1 && !a.is_max && a.kh == 3 && a.kw == 3 && a.sw == 1 && a.C % 8 == 0 && !no64 && !tiled3) {
+      dim3 grid((a.C + 63) / 64, (a.Q + kP64TQ - 1) / kP64TQ, (a.P + kP64TP - 1) / kP64TP);
+      launch_pdl(pool_avg64_kernel, grid, dim3(256), 0, st, a);
+      return;
+    }
+  }
   if (std::is_same<T, bf16>::value && a.kh == 3 && a.kw == 3 && !tiled3 && !big_s1) {
     const int per_row = a.Q * ((a.C + N - 1) / N);
     dim3 grid((per_row + 255) / 256, a.P);

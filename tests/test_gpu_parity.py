@@ -169,7 +169,8 @@ POOL_CASES = [
     ("max", 40, 20, 70, 3, 2, 1, 0, 0),     # padded max
     ("avg", 24, 17, 40, 2, 2, 0, 1, 1),     # generic k (even), ceil + count_include_pad
     ("avg", 42, 31, 37, 3, 1, 1, 0, 0),     # row-streaming s1: channel tail, in-bounds divisor
-    ("avg", 128, 400, 400, 3, 1, 1, 0, 1),  # row-streaming s1, several rows per strip
+    ("avg", 128, 400, 400, 3, 1, 1, 0, 1),  # large s1 average: 64-channel CTAs
+    ("avg", 168, 200, 203, 3, 1, 1, 0, 0),  # large s1 average, partial last 64-channel group, in-bounds divisor
     ("max", 64, 801, 803, 3, 2, 0, 1, 0),   # row-streaming s2, ceil mode, several rows per strip
     ("max", 20, 9, 9, 3, 1, 1, 0, 0),       # row-streaming s1 max, tiny
 ]
