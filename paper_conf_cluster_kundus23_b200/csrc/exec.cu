@@ -31,8 +31,18 @@ namespace hios {
 // Every product of the original sum appears exactly once; K per tap is one
 // K=16 MMA slice (4C <= 16) instead of a 64-channel chunk that is 95 % zero,
 // and stride 1 lets the conv run in halo mode.
+// 3x3 stride-2 stems over 3 channels with <= 40 outputs take the direct
+// CUDA-core kernel (misc.cu conv_stem3_kernel; weights in the parameter bank):
+// measured on B200, Inception Conv2d_1a at 4096^2 s2d + tcgen05 ~331 us,
+// smem-weight CUDA-core kernel ~380 us (tools/stem_micro.py).  HIOS_NOSTEM3=1
+// restores the s2d path.
+static bool stem3_conv(const Op& o) {
+  static const bool off = getenv("HIOS_NOSTEM3") != nullptr;
+  return !off && o.kind == HIOS_OP_CONV && o.in_c == 3 && o.kh == 3 && o.kw == 3 && o.sh == 2 && o.sw == 2 &&
+         o.dh == 1 && o.dw == 1 && o.out_c <= kStem3MaxK;
+}
 static bool s2d_conv(const Op& o) {
-  return o.kind == HIOS_OP_CONV && o.in_c <= 4 && o.sh == 2 && o.sw == 2 && o.dh == 1 && o.dw == 1 &&
+  return o.kind == HIOS_OP_CONV && !stem3_conv(o) && o.in_c <= 4 && o.sh == 2 && o.sw == 2 && o.dh == 1 && o.dw == 1 &&
          o.kh * o.kw >= 4 && !getenv("HIOS_NOS2D");
 }
 
@@ -616,6 +626,28 @@ static void build_op(Executor& ex, int v) {
     case HIOS_OP_CONV: {
       const int u = in_op(0);
       const Op& xi = g.ops[u];
+      if (stem3_conv(o)) {
+        View iv = view_of(u, l);
+        if (iv.ldc < (int)(16 / sizeof(T))) fail(HIOS_E_UNSUPPORTED, "stem input pixel pitch below 16 bytes");
+        ConvStem3Args<T> c{};
+        c.x = (const T*)iv.p; c.H = xi.H; c.W = xi.W; c.ldx = iv.ldc;
+        c.P = o.H; c.Q = o.W; c.K = o.out_c; c.ph = o.ph; c.pw = o.pw; c.relu = o.relu;
+        c.out = (T*)out.p; c.ldo = out.ldc;
+        c.out2 = out2 ? (T*)out2->p : nullptr; c.ldo2 = out2 ? out2->ldc : 0;
+        auto wp = std::make_shared<Stem3W>();
+        std::memset(wp.get(), 0, sizeof(Stem3W));
+        for (int k = 0; k < o.out_c; ++k) {
+          for (int cc = 0; cc < 3; ++cc)
+            for (int r = 0; r < 3; ++r)
+              for (int s2 = 0; s2 < 3; ++s2)
+                wp->w[(r * 3 + s2) * 3 + cc][k] = o.weight[(((size_t)k * 3 + cc) * 3 + r) * 3 + s2];
+          wp->scale[k] = o.scale[k];
+          wp->shift[k] = o.shift[k];
+        }
+        fns.push_back([c, wp](cudaStream_t st) { launch_conv_stem3<T>(c, *wp, st); });
+        ++nk;
+        break;
+      }
       if (x.s2dbuf >= 0) {
         View iv = view_of(u, l);
         const int R2 = (o.kh + 1) / 2, S2 = (o.kw + 1) / 2;

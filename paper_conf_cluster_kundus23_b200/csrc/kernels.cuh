@@ -149,6 +149,23 @@ __host__ __device__ inline uint32_t halo_bytes_of(int R, int halo_w) {
 }
 void launch_conv_simt(const ConvSimtArgs& a, cudaStream_t st);
 template <typename T> void launch_conv_small_c(const ConvSmallArgs<T>& a, cudaStream_t st);
+// 3x3 stride-2 stems over 3 input channels (Inception-v3 Conv2d_1a, RandWire
+// conv1): the 27 x KK folded weights and the BN scale/shift travel in the
+// kernel's parameter bank, so every multiply-add is one FFMA with a constant
+// operand (no shared-memory weight loads); see misc.cu conv_stem3_kernel
+constexpr int kStem3MaxK = 40;
+struct Stem3W {
+  float w[27][kStem3MaxK];  // [(r*3+s)*3+c][k]
+  float scale[kStem3MaxK], shift[kStem3MaxK];
+};
+template <typename T>
+struct ConvStem3Args {
+  const T* x; int H, W, ldx;
+  int P, Q, K, ph, pw, relu;
+  T* out; int ldo; T* out2; int ldo2;
+};
+template <typename T> void launch_conv_stem3(const ConvStem3Args<T>& a, const Stem3W& w, cudaStream_t st);
+
 template <typename T> void launch_dw(const DwArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_pool(const PoolArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_add(const AddArgs<T>& a, cudaStream_t st);

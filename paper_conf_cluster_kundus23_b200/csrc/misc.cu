@@ -1336,5 +1336,97 @@ void launch_conv_small_c(const ConvSmallArgs<T>& a, cudaStream_t st) {
     launch_small<T, 0, 0, 0, 16>(a, st);
 }
 template void launch_conv_small_c<float>(const ConvSmallArgs<float>&, cudaStream_t);
+// 3x3 stride-2 stem over 3 channels (kernels.cuh Stem3W): one thread = PX
+// horizontally adjacent output pixels x all K channels.  The 3 x (2PX+1)
+// input window (one 16-byte load per pixel: pixel pitch >= 8 channels) sits in
+// registers; the weights are read from the parameter bank with compile-time
+// offsets, i.e. as the constant operand of FFMA.  fp32 accumulation in the
+// oracle's (r, s, c) order per output; folded BN + ReLU epilogue.
+template <typename T, int PX>
+__device__ __forceinline__ void stem3_load(const ConvStem3Args<T>& a, int QP, long long it, float (&x)[3][2 * PX + 1][3]) {
+  const int p = (int)(it / QP), q0 = (int)(it - (long long)p * QP) * PX;
+  const int h0 = p * 2 - a.ph, w0 = q0 * 2 - a.pw;
+#pragma unroll
+  for (int r = 0; r < 3; ++r)
+#pragma unroll
+    for (int s = 0; s < 2 * PX + 1; ++s) {
+      const int h = h0 + r, ww = w0 + s;
+      float v[Vec<T>::N];
+      if (h >= 0 && h < a.H && ww >= 0 && ww < a.W) {
+        load_vec(a.x + ((size_t)h * a.W + ww) * a.ldx, 0, Vec<T>::N, v);
+      } else {
+#pragma unroll
+        for (int j = 0; j < Vec<T>::N; ++j) v[j] = 0.f;
+      }
+#pragma unroll
+      for (int c = 0; c < 3; ++c) x[r][s][c] = v[c];
+    }
+}
+
+template <typename T, int KK, int PX>
+__global__ void __launch_bounds__(128) conv_stem3_kernel(const ConvStem3Args<T> a, const Stem3W w) {
+  pdl_enter();
+  const int QP = (a.Q + PX - 1) / PX;
+  const long long it = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (it >= (long long)a.P * QP) return;
+  constexpr int XW = 2 * PX + 1;
+  float x[3][XW][3];
+  stem3_load<T, PX>(a, QP, it, x);
+  float acc[PX][KK];
+#pragma unroll
+  for (int u = 0; u < PX; ++u)
+#pragma unroll
+    for (int k = 0; k < KK; ++k) acc[u][k] = 0.f;
+#pragma unroll
+  for (int r = 0; r < 3; ++r)
+#pragma unroll
+    for (int s = 0; s < 3; ++s)
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        const int i = (r * 3 + s) * 3 + c;
+#pragma unroll
+        for (int k = 0; k < KK; ++k) {
+          const float wv = w.w[i][k];  // uniform-register operand of the FFMA
+#pragma unroll
+          for (int u = 0; u < PX; ++u) acc[u][k] = fmaf(x[r][2 * u + s][c], wv, acc[u][k]);
+        }
+      }
+  const int p = (int)(it / QP), q0 = (int)(it - (long long)p * QP) * PX;
+#pragma unroll
+  for (int u = 0; u < PX; ++u) {
+    if (q0 + u >= a.Q) break;
+#pragma unroll
+    for (int k = 0; k < KK; ++k) {
+      const float y = acc[u][k] * w.scale[k] + w.shift[k];
+      acc[u][k] = a.relu ? fmaxf(y, 0.f) : y;
+    }
+    const size_t pix = (size_t)p * a.Q + q0 + u;
+#pragma unroll
+    for (int c0 = 0; c0 < KK; c0 += Vec<T>::N) {
+      if (c0 >= a.K) break;
+      store_vec(a.out + pix * a.ldo + c0, c0, a.K, acc[u] + c0);
+      if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c0, c0, a.K, acc[u] + c0);
+    }
+  }
+}
+
+// (measured on B200, Inception Conv2d_1a at 4096^2: one item per thread 226 us;
+// a persistent grid-stride variant prefetching the next window 334 us, its
+// 216 registers leave 8 warps per SM)
+template <typename T, int KK>
+static void launch_stem3_k(const ConvStem3Args<T>& a, const Stem3W& w, cudaStream_t st) {
+  constexpr int PX = 2;
+  const long long n = (long long)a.P * ((a.Q + PX - 1) / PX);
+  launch_pdl(conv_stem3_kernel<T, KK, PX>, dim3((unsigned)((n + 127) / 128)), dim3(128), 0, st, a, w);
+}
+
+template <typename T>
+void launch_conv_stem3(const ConvStem3Args<T>& a, const Stem3W& w, cudaStream_t st) {
+  if (a.K <= 32) launch_stem3_k<T, 32>(a, w, st);
+  else launch_stem3_k<T, kStem3MaxK>(a, w, st);
+}
+template void launch_conv_stem3<float>(const ConvStem3Args<float>&, const Stem3W&, cudaStream_t);
+template void launch_conv_stem3<bf16>(const ConvStem3Args<bf16>&, const Stem3W&, cudaStream_t);
+
 template void launch_conv_small_c<bf16>(const ConvSmallArgs<bf16>&, cudaStream_t);
 }  // namespace hios

@@ -87,6 +87,11 @@ CONV_CASES = [
     (2, 24, 30, 31, 5, 5, 2, 2, 2),       # C = 2, 5x5 (taps past R, S in W')
     (4, 32, 41, 300, 3, 3, 2, 0, 0),      # C = 4: packed taps (S' = 2 < 4), halo mode
     (3, 64, 300, 35, 5, 5, 2, 2, 2),      # packed taps (S' = 3), tap mode (narrow output)
+    # 3x3 stride-2 stems over 3 channels, K <= 40: direct CUDA-core kernel with
+    # weights in the parameter bank (odd Q = 2-pixel tail, padding, K < 32, K = 40)
+    (3, 32, 64, 301, 3, 3, 2, 1, 1),
+    (3, 24, 20, 21, 3, 3, 2, 0, 0),
+    (3, 40, 17, 150, 3, 3, 2, 1, 0),
     # halo mode with resident weights (one N tile, > 148 output tiles per CTA wave)
     (32, 32, 160, 200, 3, 3, 1, 1, 1),
     (64, 80, 150, 130, 1, 1, 1, 0, 0),
