@@ -1363,7 +1363,9 @@ __device__ __forceinline__ void stem3_load(const ConvStem3Args<T>& a, int QP, lo
     }
 }
 
-template <typename T, int KK, int PX>
+// KT < KK: blockIdx.y selects which KT-channel slice of the KK outputs this
+// CTA computes (fewer registers per thread, more resident warps)
+template <typename T, int KK, int PX, int KT = KK>
 __global__ void __launch_bounds__(128) conv_stem3_kernel(const ConvStem3Args<T> a, const Stem3W w) {
   pdl_enter();
   const int QP = (a.Q + PX - 1) / PX;
@@ -1372,11 +1374,12 @@ __global__ void __launch_bounds__(128) conv_stem3_kernel(const ConvStem3Args<T> 
   constexpr int XW = 2 * PX + 1;
   float x[3][XW][3];
   stem3_load<T, PX>(a, QP, it, x);
-  float acc[PX][KK];
+  const int kb = KT < KK ? (int)blockIdx.y * KT : 0;
+  float acc[PX][KT];
 #pragma unroll
   for (int u = 0; u < PX; ++u)
 #pragma unroll
-    for (int k = 0; k < KK; ++k) acc[u][k] = 0.f;
+    for (int k = 0; k < KT; ++k) acc[u][k] = 0.f;
 #pragma unroll
   for (int r = 0; r < 3; ++r)
 #pragma unroll
@@ -1385,8 +1388,8 @@ __global__ void __launch_bounds__(128) conv_stem3_kernel(const ConvStem3Args<T> 
       for (int c = 0; c < 3; ++c) {
         const int i = (r * 3 + s) * 3 + c;
 #pragma unroll
-        for (int k = 0; k < KK; ++k) {
-          const float wv = w.w[i][k];  // uniform-register operand of the FFMA
+        for (int k = 0; k < KT; ++k) {
+          const float wv = w.w[i][kb + k];  // uniform-register operand of the FFMA
 #pragma unroll
           for (int u = 0; u < PX; ++u) acc[u][k] = fmaf(x[r][2 * u + s][c], wv, acc[u][k]);
         }
@@ -1396,23 +1399,24 @@ __global__ void __launch_bounds__(128) conv_stem3_kernel(const ConvStem3Args<T> 
   for (int u = 0; u < PX; ++u) {
     if (q0 + u >= a.Q) break;
 #pragma unroll
-    for (int k = 0; k < KK; ++k) {
-      const float y = acc[u][k] * w.scale[k] + w.shift[k];
+    for (int k = 0; k < KT; ++k) {
+      const float y = acc[u][k] * w.scale[kb + k] + w.shift[kb + k];
       acc[u][k] = a.relu ? fmaxf(y, 0.f) : y;
     }
     const size_t pix = (size_t)p * a.Q + q0 + u;
 #pragma unroll
-    for (int c0 = 0; c0 < KK; c0 += Vec<T>::N) {
-      if (c0 >= a.K) break;
-      store_vec(a.out + pix * a.ldo + c0, c0, a.K, acc[u] + c0);
-      if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c0, c0, a.K, acc[u] + c0);
+    for (int c0 = 0; c0 < KT; c0 += Vec<T>::N) {
+      if (kb + c0 >= a.K) break;
+      store_vec(a.out + pix * a.ldo + kb + c0, kb + c0, a.K, acc[u] + c0);
+      if (a.out2) store_vec(a.out2 + pix * a.ldo2 + kb + c0, kb + c0, a.K, acc[u] + c0);
     }
   }
 }
 
 // (measured on B200, Inception Conv2d_1a at 4096^2: one item per thread 226 us;
 // a persistent grid-stride variant prefetching the next window 334 us, its
-// 216 registers leave 8 warps per SM)
+// 216 registers leave 8 warps per SM; 16-channel slices per CTA (blockIdx.y,
+// 80 registers, 24 warps per SM) 248 us)
 template <typename T, int KK>
 static void launch_stem3_k(const ConvStem3Args<T>& a, const Stem3W& w, cudaStream_t st) {
   constexpr int PX = 2;
