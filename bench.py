@@ -517,7 +517,12 @@ def main():
                         "in": [shapes[u] for u in g.preds(o.id)], "k": [o.kh, o.kw, o.sh, o.sw],
                         "ms": float(op_ms[o.id]), "gflop": F[o.id] / 1e9, "mb": B[o.id] / 1e6,
                         "gpu": int(op_gpu[o.id]), "stage": int(op_stage[o.id])} for o in g.ops], f, indent=0)
-    conv_ids = [o.id for o in g.ops if o.kind == "conv" and op_ms[o.id] > 0]
+    # ops of conv_tc_kernel only: 3x3 stride-2 3-channel stems with K <= 40 run
+    # on CUDA cores (csrc/exec.cu stem3_conv, conv_stem3_kernel)
+    def on_tc(o):
+        ci = shapes[g.preds(o.id)[0]][0]
+        return not (ci == 3 and o.kh == 3 and o.kw == 3 and o.sh == 2 and o.sw == 2 and o.out_c <= 40)
+    conv_ids = [o.id for o in g.ops if o.kind == "conv" and op_ms[o.id] > 0 and on_tc(o)]
     conv_flops = float(F[conv_ids].sum())
     conv_s = float(op_ms[conv_ids].sum()) / 1e3
     step_r = float(op_ms[op_ms > 0].sum())
