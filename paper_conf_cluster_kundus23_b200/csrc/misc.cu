@@ -1416,7 +1416,8 @@ __global__ void __launch_bounds__(128) conv_stem3_kernel(const ConvStem3Args<T> 
 // (measured on B200, Inception Conv2d_1a at 4096^2: one item per thread 226 us;
 // a persistent grid-stride variant prefetching the next window 334 us, its
 // 216 registers leave 8 warps per SM; 16-channel slices per CTA (blockIdx.y,
-// 80 registers, 24 warps per SM) 248 us)
+// 80 registers, 24 warps per SM) 248 us; pixels per thread PX = 1/3/4:
+// 1219/243/287 us -- at PX = 1 the uniform weight loads (LDCU) bound it)
 template <typename T, int KK>
 static void launch_stem3_k(const ConvStem3Args<T>& a, const Stem3W& w, cudaStream_t st) {
   constexpr int PX = 2;
