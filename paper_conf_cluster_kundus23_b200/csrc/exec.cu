@@ -632,6 +632,12 @@ static void build_op(Executor& ex, int v) {
         ConvStem3Args<T> c{};
         c.x = (const T*)iv.p; c.H = xi.H; c.W = xi.W; c.ldx = iv.ldc;
         c.P = o.H; c.Q = o.W; c.K = o.out_c; c.ph = o.ph; c.pw = o.pw; c.relu = o.relu;
+        // whole 16-byte vectors (zeros into the pad channels) unless an output
+        // is a concat slice, whose pad channels belong to the next producer
+        bool own = true;
+        for (int e : o.out_edges)
+          if (ex.inplace[e]) own = false;
+        c.kst = own ? rup(o.out_c, 8) : o.out_c;
         c.out = (T*)out.p; c.ldo = out.ldc;
         c.out2 = out2 ? (T*)out2->p : nullptr; c.ldo2 = out2 ? out2->ldc : 0;
         auto wp = std::make_shared<Stem3W>();

@@ -162,6 +162,7 @@ template <typename T>
 struct ConvStem3Args {
   const T* x; int H, W, ldx;
   int P, Q, K, ph, pw, relu;
+  int kst;  // channels stored per pixel: K, or rup(K, 8) when the pad channels are this op's own
   T* out; int ldo; T* out2; int ldo2;
 };
 template <typename T> void launch_conv_stem3(const ConvStem3Args<T>& a, const Stem3W& w, cudaStream_t st);

@@ -1407,8 +1407,9 @@ __global__ void __launch_bounds__(128) conv_stem3_kernel(const ConvStem3Args<T> 
 #pragma unroll
     for (int c0 = 0; c0 < KT; c0 += Vec<T>::N) {
       if (kb + c0 >= a.K) break;
-      store_vec(a.out + pix * a.ldo + kb + c0, kb + c0, a.K, acc[u] + c0);
-      if (a.out2) store_vec(a.out2 + pix * a.ldo2 + kb + c0, kb + c0, a.K, acc[u] + c0);
+      // (pad channels past K, when stored, are exact zeros: zero weights, scale and shift)
+      store_vec(a.out + pix * a.ldo + kb + c0, kb + c0, a.kst, acc[u] + c0);
+      if (a.out2) store_vec(a.out2 + pix * a.ldo2 + kb + c0, kb + c0, a.kst, acc[u] + c0);
     }
   }
 }

@@ -285,3 +285,25 @@ def test_inception_1024_bench_config():
     assert nerr(y, ref) <= TOL["bf16"]
     # repeated runs are deterministic
     assert np.array_equal(y, hios().hios_run(S, x))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_stem3_concat_slice(dtype):
+    """A 3x3 stride-2 3-channel stem with K % 8 != 0 (RandWire conv1-like, K = 39)
+    written in place into slot 0 of a concat: its pad channel belongs to the
+    next producer, so the kernel must store exactly K channels (csrc/exec.cu:
+    kst); next to it the same stem feeding a 1x1 conv from its own buffer."""
+    g = graphs.GraphSpec("stem3cat", 3, 45, 70)
+    x0 = g.input()
+    a = g.conv(x0, 39, 3, s=2, p=1, relu=1)
+    b = g.conv(x0, 9, 3, s=2, p=1, relu=1)
+    d = g.conv(a, 16, 1, relu=1)
+    e = g.conv(x0, 39, 3, s=2, p=1, relu=0)
+    f = g.conv(e, 16, 1, relu=1)
+    g.concat([a, b, d, f])
+    W = gen.make_weights(g)
+    x = gen.make_input(g) - 0.5
+    _, S, y = run_graph_gpu(g, W, x, dtype, profile=False)
+    ref = infer.run_graph(g, W, x)[g.n_ops - 1]
+    assert nerr(y.reshape(ref.shape), ref) <= TOL[dtype] / (4 if dtype == "bf16" else 1)
