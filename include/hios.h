@@ -245,6 +245,16 @@ hios_status hios_read_op_output(hios_schedule s, int32_t op, float* host, int64_
 hios_status hios_run_timed(hios_schedule s, const void* d_in, void* d_out, void* stream,
                            int64_t* op_ns);
 
+/* Uninstrumented device time of each op's kernels as configured in Q (the
+ * stage context decides the conv tile plan), each op timed alone on its
+ * logical GPU's device: per rep the L2 is flushed by writing `flush_bytes`
+ * (0 = no flush), then CUDA events recorded as graph nodes on the launching
+ * stream bracket the op's kernels only; median of `reps` (>= 1) after one
+ * warm-up.  Lowers/captures Q first if needed.  op_ns [n_ops] (caller-owned):
+ * ns, or -1 for ops not executed by this process, the INPUT placeholder and
+ * concats (zero-copy).  Errors: HIOS_E_INVALID, HIOS_E_CUDA, HIOS_E_OOM. */
+hios_status hios_time_ops(hios_schedule s, int32_t reps, int64_t flush_bytes, int64_t* op_ns);
+
 /* Number of kernels one run launches on this process's GPUs (graph nodes
  * that are kernels written in this library). */
 hios_status hios_kernel_count(hios_schedule s, int64_t* n);

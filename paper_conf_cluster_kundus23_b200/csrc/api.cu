@@ -428,6 +428,15 @@ hios_status hios_read_op_output(hios_schedule s, int32_t op, float* host, int64_
   });
 }
 
+hios_status hios_time_ops(hios_schedule s, int32_t reps, int64_t flush_bytes, int64_t* op_ns) {
+  return guard([&] {
+    NEED(s && op_ns && reps >= 1 && flush_bytes >= 0, HIOS_E_INVALID, "bad argument");
+    auto& E = ensure_exec(*s->s);
+    if (!s->s->owner.empty()) check_remote_mapped(E);
+    E.time_ops(reps, flush_bytes, op_ns);
+  });
+}
+
 hios_status hios_kernel_count(hios_schedule s, int64_t* n) {
   return guard([&] {
     NEED(s && n, HIOS_E_INVALID, "NULL argument");

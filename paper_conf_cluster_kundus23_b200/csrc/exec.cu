@@ -1006,6 +1006,65 @@ void Executor::run_device(const void* d_in, void* d_out, cudaStream_t user, bool
   ck(cudaGetLastError(), "run");
 }
 
+// Uninstrumented per-op device time of the schedule's own kernels (bench.py's
+// roofline): for op v, one CUDA graph = [L2 flush (a write of flush_bytes) ->
+// event -> v's kernels as configured in Q (its stage context) -> event],
+// replayed reps + 1 times (the first is a warm-up); median of the event
+// intervals.  Cold L2 per op, like ncu's default --cache-control all.
+void Executor::time_ops(int reps, int64_t flush_bytes, int64_t* op_ns) {
+  if (!lowered) {
+    plan();
+    allocate();
+  }
+  if (!captured) {
+    build_closures();
+    capture();
+  }
+  for (int v = 0; v < g.n; ++v) op_ns[v] = -1;
+  for (int l = 0; l < M; ++l) {
+    LGpu& L = lg[l];
+    if (!L.local) continue;
+    ck(cudaSetDevice(L.dev), "cudaSetDevice");
+    void* fl = nullptr;
+    if (flush_bytes > 0) ck(cudaMalloc(&fl, (size_t)flush_bytes), "cudaMalloc flush");
+    cudaEvent_t a, b;
+    ck(cudaEventCreate(&a), "event");
+    ck(cudaEventCreate(&b), "event");
+    cudaStream_t st = L.streams[0];
+    for (int j = 0; j < (int)s.Q[l].size(); ++j) {
+      const auto& S = s.Q[l][j];
+      for (int v : S) {
+        if (g.ops[v].kind == HIOS_OP_INPUT || g.ops[v].kind == HIOS_OP_CONCAT) continue;
+        const bool solo = S.size() == 1 && ox[v].run_solo;
+        cudaGraph_t graph;
+        ck(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed), "time_ops capture");
+        if (fl) launch_fill(fl, (size_t)flush_bytes, st);
+        ck(cudaEventRecordWithFlags(a, st, cudaEventRecordExternal), "record");
+        (solo ? ox[v].run_solo : ox[v].run)(st);
+        ck(cudaEventRecordWithFlags(b, st, cudaEventRecordExternal), "record");
+        ck(cudaStreamEndCapture(st, &graph), "time_ops capture end");
+        cudaGraphExec_t ge;
+        ck(cudaGraphInstantiate(&ge, graph, 0), "time_ops instantiate");
+        cudaGraphDestroy(graph);
+        std::vector<float> ms;
+        for (int i = 0; i <= std::max(1, reps); ++i) {
+          ck(cudaGraphLaunch(ge, st), "time_ops launch");
+          ck(cudaStreamSynchronize(st), "time_ops sync");
+          float t = 0;
+          ck(cudaEventElapsedTime(&t, a, b), "elapsed");
+          if (i > 0) ms.push_back(t);
+        }
+        cudaGraphExecDestroy(ge);
+        std::sort(ms.begin(), ms.end());
+        op_ns[v] = (int64_t)(ms[ms.size() / 2] * 1e6);
+      }
+    }
+    cudaEventDestroy(a);
+    cudaEventDestroy(b);
+    if (fl) cudaFree(fl);
+  }
+}
+
 void Executor::read_output(int op, float* host, int64_t n) {
   const int l = s.gpu_of[op];
   if (!lg[l].local) fail(HIOS_E_INVALID, "op not executed by this process");

@@ -88,6 +88,8 @@ struct Executor {
   bool is_local(int l) const { return lg[l].local; }
   void read_output(int op, float* host, int64_t n);
   void enqueue_stage_program(int l, bool timed);
+  // each local op's kernels alone, L2 flushed, as configured in Q (hios_time_ops)
+  void time_ops(int reps, int64_t flush_bytes, int64_t* op_ns);
 };
 
 void ck(cudaError_t e, const char* what);

@@ -80,6 +80,7 @@ def load() -> C.CDLL:
         "hios_run_timed": [VP, VP, VP, VP, P(I64)],
         "hios_read_op_output": [VP, I32, P(C.c_float), I64],
         "hios_kernel_count": [VP, P(I64)],
+        "hios_time_ops": [VP, I32, I64, P(I64)],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -336,6 +337,12 @@ def hios_run_timed(s: Schedule, d_in: int, d_out: int, stream: int = 0) -> np.nd
     t = np.zeros(s.graph.n_ops, dtype=np.int64)
     _ck(load().hios_run_timed(s.h, C.c_void_p(d_in), C.c_void_p(d_out), C.c_void_p(stream),
                               t.ctypes.data_as(C.POINTER(C.c_int64))))
+    return t
+
+
+def hios_time_ops(s: Schedule, reps: int = 5, flush_bytes: int = 256 << 20) -> np.ndarray:
+    t = np.zeros(s.graph.n_ops, dtype=np.int64)
+    _ck(load().hios_time_ops(s.h, reps, flush_bytes, t.ctypes.data_as(C.POINTER(C.c_int64))))
     return t
 
 

@@ -189,3 +189,66 @@ def test_all_workloads_run_small():
         out = I.run_graph(g, gen.make_weights(g), gen.make_input(g), keep={g.n_ops - 1})
         y = out[g.n_ops - 1]
         assert np.isfinite(y).all() and np.abs(y).max() > 0
+
+
+def test_add_hand_computed():
+    """add (oracle/infer.py run_op 'add'): y = act(sum_i agg_i x_i), agg_i = 1
+    when the op carries no weights.  Values worked by hand."""
+    g = graphs.GraphSpec("add", 1, 1, 2)
+    x0 = g.input()
+    plain = g.add([x0, x0, x0], relu=0)          # 3 x
+    plain_r = g.add([x0, x0], relu=1)            # relu(2 x)
+    weighted = g.add([x0, x0], relu=0, agg=1)    # (1/2 + 1/2) x = x (gen: agg = 1/n)
+    op = {o.id: o for o in g.ops}
+    x = np.array([[[-1.5, 2.0]]])
+    assert np.array_equal(I.run_op(op[plain], [x, x, x], {}), [[[-4.5, 6.0]]])
+    assert np.array_equal(I.run_op(op[plain_r], [x, x], {}), [[[0.0, 4.0]]])
+    w = {"agg": np.array([0.25, 0.75], dtype=np.float32)}
+    y = I.run_op(op[weighted], [x, 2 * x], w)    # 0.25 x + 1.5 x = 1.75 x
+    assert np.array_equal(y, [[[-2.625, 3.5]]])
+    op[weighted].relu = 1
+    assert np.array_equal(I.run_op(op[weighted], [x, 2 * x], w), [[[0.0, 3.5]]])
+    # a single-input ReLU add and the input order (slot order) of weights
+    one = g.add([x0], relu=1)
+    assert np.array_equal(I.run_op({o.id: o for o in g.ops}[one], [x], {}), [[[0.0, 2.0]]])
+    w2 = {"agg": np.array([1.0, -3.0], dtype=np.float32)}
+    op[weighted].relu = 0
+    assert np.array_equal(I.run_op(op[weighted], [x, 0 * x + 1.0], w2), [[[-4.5, -1.0]]])
+
+
+@pytest.mark.parametrize("n_in,agg,act", [(2, 0, 0), (2, 0, 1), (5, 1, 1), (4, 1, 0)])
+def test_add_vs_torch_in_graph(n_in, agg, act):
+    """The add branch as run_graph reaches it (edge slots, gen's aggregation
+    weights), against torch fp64: relu(sum_i a_i x_i) by torch.stack /
+    tensordot, a_i = gen's agg weights or 1."""
+    g = graphs.GraphSpec("addg", 3, 7, 6)
+    x0 = g.input()
+    ins = [g.conv(x0, 5, 3, p=1, relu=0) for _ in range(n_in)]
+    s = g.add(ins[::-1], relu=act, agg=agg)       # reversed: slot order != id order
+    W = gen.make_weights(g)
+    x = gen.make_input(g)
+    out = I.run_graph(g, W, x)
+    t = torch.stack([torch.from_numpy(out[i]) for i in ins[::-1]])
+    a = torch.from_numpy(W[s]["agg"].astype(np.float64)) if agg else torch.ones(n_in, dtype=torch.float64)
+    ref = torch.tensordot(a, t, dims=([0], [0]))
+    if act:
+        ref = F.relu(ref)
+    np.testing.assert_allclose(out[s], ref.numpy(), rtol=1e-13, atol=1e-13)
+    if agg:  # gen's add weights are 1/n: the aggregation is the mean
+        np.testing.assert_allclose(W[s]["agg"].astype(np.float64).sum(), 1.0, rtol=1e-6)
+
+
+def test_identity_is_a_copy():
+    g = graphs.GraphSpec("id", 4, 5, 5)
+    x0 = g.input()
+    c = g.conv(x0, 6, 3, p=1)
+    i = g.identity(c)
+    g.add([i, c], relu=0)
+    W = gen.make_weights(g)
+    x = gen.make_input(g)
+    out = I.run_graph(g, W, x)
+    assert np.array_equal(out[i], out[c])
+    np.testing.assert_array_equal(out[g.n_ops - 1], 2 * out[c])
+    y = I.run_op(g.ops[i], [out[c]], {})
+    y += 1.0                                       # a copy, not a view of the input
+    assert np.array_equal(out[i], out[c])

@@ -290,8 +290,8 @@ def squeezenet(h: int = 224, w: Optional[int] = None) -> GraphSpec:
 # ============================================================================
 # WS(N=32, K=4, P=0.75) graphs, generated once with
 #   networkx.connected_watts_strogatz_graph(32, 4, 0.75, seed=s), s = 0, 1, 2
-# and oriented low id -> high id.  Frozen in tests/golden/randwire_ws_edges.json
-# (regenerated by tests/golden/make_randwire_edges.py) so a networkx change
+# and oriented low id -> high id.  Frozen in workloads/randwire_ws_edges.json
+# (regenerated by workloads/make_randwire_edges.py) so a networkx change
 # cannot alter the workload.
 def _randwire_edges() -> List[List[Tuple[int, int]]]:
     import json
