@@ -299,6 +299,19 @@ constexpr int kEpi = 4;        // epilogue warps (one TMEM lane quarter each)
 constexpr int kThreads = 32 * (kProducers + kMma + kEpi);
 constexpr int kEpiWarp0 = kProducers + kMma;
 
+// output pixel of accumulator row m of M-tile m_blk (tile origin p0, q0)
+__device__ __forceinline__ void tile_pixel(const ConvTcArgs& a, int m_blk, int p0, int q0, int m, int& p, int& q) {
+  if (a.vgrid) {
+    const int v = m_blk * 128 + m;
+    p = v / a.vgrid;
+    q = v - p * a.vgrid;  // q >= Q: a virtual column, dropped by the caller
+  } else {
+    const int hh = m / a.tw;
+    p = p0 + hh;
+    q = q0 + (m - hh * a.tw);
+  }
+}
+
 __host__ __device__ inline uint32_t stage_pitch(int n_tile) { return (uint32_t)n_tile * 2u + 16u; }
 
 __global__ void __launch_bounds__(kThreads, 1)
@@ -310,7 +323,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int ST = a.stages;
   const uint32_t A_BYTES = 128 * 128;
   const uint32_t B_BYTES = (uint32_t)a.n_tile * 128;
-  const uint32_t H_BYTES = a.halo ? halo_bytes_of(a.R, a.halo_w) : 0u;
+  const uint32_t H_BYTES = a.halo ? halo_bytes_of(a.hrows, a.halo_w) : 0u;
   const uint32_t PITCH = stage_pitch(a.n_tile);
   uint8_t* sA = smem;  // halo: a_bufs x H_BYTES ; tap: ST x kps x A_BYTES
   uint8_t* sB = smem + (a.halo ? a.a_bufs * H_BYTES : ST * a.kps * A_BYTES);
@@ -416,7 +429,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int m_blk = tmn / a.tiles_n, n_blk = tmn - m_blk * a.tiles_n;
         const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
         const int p0 = tp * a.th, q0 = tq * a.tw, n0 = n_blk * a.n_tile;
-        const int x0 = q0 * a.sw - a.pw, y0 = p0 * a.sh - a.ph;
+        // vgrid: the box = whole padded input rows from the tile's first row
+        const int x0 = a.vgrid ? -a.pw : q0 * a.sw - a.pw;
+        const int y0 = a.vgrid ? (m_blk * 128) / a.vgrid - a.ph : p0 * a.sh - a.ph;
         // split-K: this split's K-steps [k_lo, k_hi) (any (chunk, tap) boundary)
         const int k_lo = split * a.kpsplit, k_hi = min(a.c_chunks * RS, k_lo + a.kpsplit);
         int cc = k_lo / RS, rs = k_lo - (k_lo / RS) * RS;
@@ -430,7 +445,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               if (a.dbg & 4) {  // timing experiment: no halo loads (stale smem)
                 mbar_arrive(afull0 + 8 * ab);
               } else {
-                mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.R * a.halo_w * 128u);
+                mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.hrows * a.halo_w * 128u);
                 tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, cc * 64, x0, y0);
               }
             }
@@ -493,7 +508,7 @@ __global__ void __launch_bounds__(kThreads, 1)
                              | ((uint32_t)(128 >> 4) << 24);    // M = 128
       uint32_t st = 0, ph = 0, ab = 0, aph = 0, ks = 0, acc = 0, tph = 0;
       const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB) + (uint32_t)(j * n_sub) * 128u;
-      const uint32_t row_r = (uint32_t)a.halo_w * 128u, row_s = (uint32_t)a.dw * 128u;
+      const uint32_t row_r = (uint32_t)a.hrow_px * 128u, row_s = (uint32_t)a.dw * 128u;
       int tcount = 0;
       if (a.bres) {
         mbar_wait(bres_bar, 0);
@@ -519,11 +534,17 @@ __global__ void __launch_bounds__(kThreads, 1)
           tc_fence_after();
           const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
           uint32_t accum = 0;
+          // vgrid: the tile's window starts v0 mod Wh pixels into the box
+          uint32_t xoff = 0;
+          if (a.vgrid) {
+            const int m0 = ((tile % tiles_mn) / a.tiles_n) * 128;
+            xoff = (uint32_t)(m0 - (m0 / a.vgrid) * a.vgrid) * 128u;
+          }
           for (int cc = 0; cc < nchunks; ++cc) {
             mbar_wait(afull0 + 8 * ab, aph);
             tc_fence_after();
             if (bres && lane == 0 && j == 0) TRACE2(1, tcount);
-            const uint64_t a0 = umma_desc_sw128(sA0 + ab * H_BYTES);
+            const uint64_t a0 = umma_desc_sw128(sA0 + ab * H_BYTES + xoff);
             const int kv = min(4, (C - cc * 64 + 15) >> 4);
             if (bres && fixed_rs) {
               // resident weights, common kernel shapes: the chunk's taps fully
@@ -675,8 +696,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         __syncwarp();
         tc_fence_after();
         const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)a.n_tile;
-        const int hh = m / a.tw, ww = m - hh * a.tw;
-        const int p = p0 + hh, q = q0 + ww;
+        int p, q;
+        tile_pixel(a, m_blk, p0, q0, m, p, q);
         const bool valid = p < a.P && q < a.Q;
         float* wrow = a.ws + (size_t)split * a.ws_split + ((size_t)p * a.Q + q) * a.ws_ld + n0;
         for (int col = 0; col < a.n_tile; col += 16) {
@@ -748,8 +769,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         // registers -- no staging, no proxy fence, no bulk-group waits
         const float* scs = s_scale + (a.sres ? n0 : 0);
         const float* shs = s_shift + (a.sres ? n0 : 0);
-        const int hh = m / a.tw, ww = m - hh * a.tw;
-        const int p = p0 + hh, q = q0 + ww;
+        int p, q;
+        tile_pixel(a, m_blk, p0, q0, m, p, q);
         const bool valid = p < a.P && q < a.Q;
         const size_t pix = (size_t)p * a.Q + q;
         bf16* o1 = a.out + pix * a.ldo + n0;
@@ -922,8 +943,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         for (int u = 0; u < 4; ++u) {
           const int i = i0 + u * 128;
           if (i >= total) break;
-          const int hh = rr[u] / a.tw, ww = rr[u] - hh * a.tw;
-          const int p = p0 + hh, q = q0 + ww;
+          int p, q;
+          tile_pixel(a, m_blk, p0, q0, rr[u], p, q);
           if (p >= a.P || q >= a.Q) continue;
           const size_t pix = (size_t)p * a.Q + q;
           *reinterpret_cast<uint4*>(a.out + pix * a.ldo + n0 + cc4[u] * 8) = v[u];
@@ -934,8 +955,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int tail0 = chunks * 8, nt = n_valid - tail0;
         for (int i = et; i < 128 * nt; i += 128) {
           const int rr1 = i / nt, e = tail0 + (i - rr1 * nt);
-          const int hh = rr1 / a.tw, ww = rr1 - hh * a.tw;
-          const int p = p0 + hh, q = q0 + ww;
+          int p, q;
+          tile_pixel(a, m_blk, p0, q0, rr1, p, q);
           if (p >= a.P || q >= a.Q) continue;
           const size_t pix = (size_t)p * a.Q + q;
           const uint16_t v = lds16(sbase + (uint32_t)rr1 * PITCH + (uint32_t)e * 2u);
@@ -1005,7 +1026,7 @@ void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st) {
 
 size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
   const size_t B = a.bres ? (size_t)a.n_tile * 128 * a.c_chunks * a.R * a.S : (size_t)a.n_tile * 128 * a.kps * a.stages;
-  const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.R, a.halo_w) : (size_t)a.stages * a.kps * 128 * 128;
+  const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.hrows, a.halo_w) : (size_t)a.stages * a.kps * 128 * 128;
   return 1024 + A + B + (size_t)a.out_bufs * 128 * (size_t)stage_pitch(a.n_tile) +
          (2 * a.stages + 2 * kMaxABufs + 6) * 8 +
          2 * kScaleRes * 4;

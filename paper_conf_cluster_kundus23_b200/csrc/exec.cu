@@ -354,12 +354,26 @@ void Executor::allocate() {
 // (waves x per-K-step time, where a K-step costs max(MMA, L2->SM bytes)).
 static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh, int sw, int dh, int dw) {
   ConvTcArgs c{};
-  const int hw = 128 + (S - 1) * dw;
+  int hw = 128 + (S - 1) * dw;
   c.halo = (sw == 1 && Q >= 96 && hw <= 256 && R * dh <= 256 && halo_bytes_of(R, hw) <= 100 * 1024) ? 1 : 0;
+  // virtual-grid halo (narrow stride-1 convs with R*S > 1, see ConvTcArgs):
+  // tap mode would stream the input R*S times through L2->SM; the box of
+  // whole padded rows streams it ~(128 + (R-1) dh Wh + (S-1) dw) / 128 times
+  const int Wh = Q + (S - 1) * dw;
+  const int vrows = (Wh - 1 + 127 + (S - 1) * dw) / Wh + 1 + (R - 1) * dh;
+  static const bool novgrid = getenv("HIOS_NOVGRID") != nullptr;  // A/B switch
+  if (!c.halo && !novgrid && sh == 1 && sw == 1 && dh == 1 && dw == 1 && R * S > 1 && Wh <= 256 && vrows <= 256 &&
+      halo_bytes_of(vrows, Wh) <= 96 * 1024) {
+    c.halo = 1;
+    c.vgrid = Wh;
+    hw = Wh;
+  }
   if (c.halo) {
     c.th = 1;
     c.tw = 128;
     c.halo_w = hw;
+    c.hrows = c.vgrid ? vrows : R;
+    c.hrow_px = c.vgrid ? dh * Wh : hw;
   } else {
     int64_t best = -1;
     for (int tw : {128, 64, 32, 16, 8}) {
@@ -372,6 +386,10 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   }
   c.tiles_q = (Q + c.tw - 1) / c.tw;
   c.tiles_m = ((P + c.th - 1) / c.th) * c.tiles_q;
+  if (c.vgrid) {
+    c.tiles_q = 1;
+    c.tiles_m = (int)(((int64_t)P * c.vgrid + 127) / 128);
+  }
   c.c_chunks = (C + 63) / 64;
   const int KI = R * S * c.c_chunks;
   // cost model (cycles), from the measured issue costs on B200
@@ -385,7 +403,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     const int tn = (K + nt - 1) / nt;
     const int nm = n_mma_of(nt);
     const double mma = std::max(4.0 * nt / 2.0, 4.0 * 100.0 / nm);
-    const double a_bytes = c.halo ? (double)R * (128 + (S - 1) * dw) * 128.0 / (R * S) : 16384.0;
+    const double a_bytes = c.halo ? (double)c.hrows * c.halo_w * 128.0 / (R * S) : 16384.0;
     const double tma = std::max((c.halo ? 1.0 : 2.0) * 500.0 / 4.0, (a_bytes + nt * 128.0) / 64.0);
     const double epi = nt / 16.0 * 80.0 + 128.0 * nt * 2.0 / 64.0;
     const double tile = std::max(KI * std::max(mma, tma), epi) + 300.0;
@@ -441,18 +459,18 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   const size_t b_all = (size_t)c.c_chunks * R * S * B;
   c.bres = 0;
   if (c.halo && c.tiles_n == 1 && c.tiles_m > 148 * c.occ && b_all <= 96 * 1024 && !getenv("HIOS_NOBRES") &&
-      halo_bytes_of(R, hw) + b_all <= budget) {
+      halo_bytes_of(c.hrows, hw) + b_all <= budget) {
     c.bres = 1;
     c.kps = std::min(4, R * S);
     // as many input boxes in flight as fit (measured: the halo TMA latency,
     // ~2 us, bounds a 2-deep ring at small K; tools/conv_trace2.py)
     const int cap = getenv("HIOS_ABUFS") ? std::max(1, std::min(kMaxABufs, atoi(getenv("HIOS_ABUFS")))) : kMaxABufs;
     c.a_bufs = 1;
-    while (c.a_bufs < cap && (c.a_bufs + 1) * halo_bytes_of(R, hw) + b_all <= budget) ++c.a_bufs;
+    while (c.a_bufs < cap && (c.a_bufs + 1) * halo_bytes_of(c.hrows, hw) + b_all <= budget) ++c.a_bufs;
     c.stages = 2;
   }
   if (c.halo && !c.bres) {
-    const size_t H = halo_bytes_of(R, hw);
+    const size_t H = halo_bytes_of(c.hrows, hw);
     if (!c.kps) c.kps = std::min(4, R * S);
     while (c.kps > 1 && H + 2 * c.kps * B > budget) --c.kps;
     c.a_bufs = (2 * H + 2 * c.kps * B <= budget) ? 2 : 1;
@@ -460,7 +478,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
       const int cap = getenv("HIOS_ABUFS") ? std::max(1, std::min(kMaxABufs, atoi(getenv("HIOS_ABUFS")))) : 4;
       while (c.a_bufs < cap && (c.a_bufs + 1) * H + 4 * c.kps * B <= budget) ++c.a_bufs;
     }
-    if (H + 2 * c.kps * B > budget) c.halo = 0;  // does not fit: fall back to tap mode
+    if (H + 2 * c.kps * B > budget) fail(HIOS_E_UNSUPPORTED, "conv halo plan does not fit shared memory");
     else c.stages = (int)std::min<size_t>(8, (budget - c.a_bufs * H) / (c.kps * B));
   }
   if (!c.halo) {
@@ -515,12 +533,6 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
                                                      int ph, int pw, int dh, int dw, int P, int Q, int relu,
                                                      const View& out, const View* out2, int& nk) {
   ConvTcArgs a = plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw);
-  if (getenv("HIOS_NOHALO") && a.halo) {  // debug: force tap mode on the same tiles
-    a.halo = 0;
-    a.bres = 0;
-    a.kps = 1;
-    a.stages = std::max(2, std::min(8, (int)((212 * 1024 - 128 * (a.n_tile * 2 + 16)) / (16384 + a.n_tile * 128))));
-  }
   CUtensorMap mx, mw;
   bool ok;
   // C % 64 != 0: the tensor map's channel extent is rounded up to whole
@@ -533,7 +545,10 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   // skipped (K=16 slices past C are not issued).
   static const bool nopad = getenv("HIOS_NOCHANPAD") != nullptr;
   const int Cm = (C % 64 && !nopad) ? rup(C, 64) : C;
-  if (a.halo)  // R input rows (stride dh) x halo_w pixels per channel chunk
+  if (a.vgrid)  // hrows whole padded input rows (x from -pw) per channel chunk
+    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w,
+                      a.hrows, 1, 1);
+  else if (a.halo)  // R input rows (stride dh) x halo_w pixels per channel chunk
     ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w, R * dh, 1,
                       dh);
   else         // th x tw output positions of one (r, s) tap, conv stride as traversal stride
@@ -555,6 +570,7 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   // destination slice (clips the ragged pixel / channel edges of a tile)
   CUtensorMap mo = mx, mo2 = mx;
   a.out_sw = a.n_tile % 64 == 0 ? 64 : (a.n_tile % 32 == 0 ? 32 : 16);
+  if (a.vgrid && a.epi == 1) a.epi = 0;  // tiles are not rectangular: no TMA-store boxes
   a.tma_out = !getenv("HIOS_NOTMASTORE") && a.ksplit == 1 && a.epi == 1 ? 1 : 0;
   if (a.ksplit > 1 || (a.epi == 1 && !a.tma_out)) a.epi = 0;
   if (a.tma_out) {

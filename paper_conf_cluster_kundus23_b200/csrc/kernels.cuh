@@ -78,6 +78,14 @@ struct ConvTcArgs {
   int out_bufs;        // epilogue staging tiles (2: tile i's stores drain while tile i+1 is staged)
   int sres;            // folded-BN scale/shift of all K channels staged once per CTA (K <= kScaleRes)
   int epi;             // epilogue: 0 smem staging + st.global, 1 TMA bulk-tensor stores, 2 direct register stores
+  // halo box geometry: hrows rows of halo_w pixels per 64-channel chunk; tap
+  // row r starts r * hrow_px pixels into the box (classic halo: hrows = R,
+  // hrow_px = halo_w).  vgrid = Wh > 0: "virtual-grid" halo for narrow
+  // stride-1 convs -- output (p, q) is virtual position v = p * Wh + q with
+  // Wh = Q + (S-1) dw (the padded input row), a tile = 128 consecutive v, the
+  // box = whole padded input rows, tap (r, s) = the window at
+  // v - v0 + r dh Wh + s dw; virtual columns q >= Q are computed and dropped
+  int hrows, hrow_px, vgrid;
 };
 constexpr int kScaleRes = 512;
 constexpr int kMaxABufs = 6;  // halo-mode input boxes in flight

@@ -92,6 +92,15 @@ CONV_CASES = [
     (3, 32, 64, 301, 3, 3, 2, 1, 1),
     (3, 24, 20, 21, 3, 3, 2, 0, 0),
     (3, 40, 17, 150, 3, 3, 2, 1, 0),
+    # virtual-grid halo mode (stride 1, R*S > 1, output width < 96: tiles of 128
+    # consecutive positions of the padded-row grid, virtual columns dropped)
+    (160, 192, 62, 62, 1, 7, 1, 0, 3),    # Inception Mixed_6 1x7 at 1024^2 (Wh = 68)
+    (160, 192, 62, 62, 7, 1, 1, 3, 0),    # 7x1: 10-row box (Wh = 62)
+    (448, 384, 30, 30, 3, 3, 1, 1, 1),    # Mixed_7 3x3, K > 128 (staged epilogue), C tail
+    (384, 384, 30, 30, 1, 3, 1, 0, 1),
+    (40, 24, 13, 90, 3, 3, 1, 1, 1),      # Wh = 92, ragged last tile, small K
+    (72, 200, 11, 7, 5, 5, 1, 2, 2),      # tiny image: one tile spans the whole output
+    (64, 64, 20, 31, 3, 3, 1, 0, 0),      # no padding: Wh = Q + 2
     # halo mode with resident weights (one N tile, > 148 output tiles per CTA wave)
     (32, 32, 160, 200, 3, 3, 1, 1, 1),
     (64, 80, 150, 130, 1, 1, 1, 0, 0),
