@@ -314,13 +314,19 @@ def share_schedule(h, dist, G, g, S, M, window, rank):
     return S
 
 
-def bind_and_exchange(h, dist, S, M, world, rank, dev):
+def bind_and_exchange(h, dist, S, M, world, rank, dev, transport="peer"):
     """Each rank owns its logical GPUs; device buffers and flag words are
     exported as CUDA IPC handles and mapped by every other rank, so producers
-    store straight into consumer buffers (peer memory over NVLink)."""
+    store straight into consumer buffers (peer memory over NVLink).  With the
+    NCCL transport rank 0's ncclUniqueId is broadcast and every rank creates
+    its communicator (the IPC maps then only carry same-process flags)."""
     own = owners(M, world)
     h.hios_schedule_place(S, [dev] * M)
     h.hios_schedule_bind_rank(S, own, rank)
+    if transport == "nccl":
+        uid = [h.hios_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        h.hios_schedule_nccl_init(S, uid[0], world, rank)
     blob = h.hios_ipc_export(S)
     blobs = [None] * world
     dist.all_gather_object(blobs, blob)

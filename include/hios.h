@@ -210,6 +210,43 @@ hios_status hios_schedule_stages(hios_schedule s, int32_t* op_gpu, int32_t* op_s
  * Must precede the first run. */
 hios_status hios_schedule_place(hios_schedule s, const int32_t* devices, int32_t n);
 
+/* Transport of the cross-GPU edges; must precede the
+ * first run.
+ *   HIOS_TRANSPORT_PEER (default): the producer's epilogue stores straight into
+ *     every consumer GPU's buffer (peer memory over NVLink / CUDA IPC), then a
+ *     system-scope release of an epoch flag; the consumer stage waits on the
+ *     flag device-side.
+ *   HIOS_TRANSPORT_COPY: the producer writes locally; a copy-engine transfer
+ *     (cudaMemcpy2DAsync) into the consumer's buffer follows it, then the flag
+ *     -- the paper's launch-after-transfer design (CUDA-aware MPI).
+ *   HIOS_TRANSPORT_NCCL: the producer writes locally; ncclSend / ncclRecv on a
+ *     per-GPU communication stream in one global transfer order (the stage
+ *     DAG's topological order), the consumer stage waits for the receive --
+ *     the fallback baseline P:318 names.  Needs one process per GPU
+ *     (hios_schedule_bind_rank) and hios_schedule_nccl_init; edges between
+ *     logical GPUs of the same process use the copy transport.
+ * Errors: HIOS_E_INVALID (unknown transport), HIOS_E_STATE (already run). */
+typedef enum { HIOS_TRANSPORT_PEER = 0, HIOS_TRANSPORT_COPY = 1, HIOS_TRANSPORT_NCCL = 2 } hios_transport;
+hios_status hios_schedule_transport(hios_schedule s, int32_t transport);
+
+/* NCCL transport set-up.  hios_nccl_unique_id writes a 128-byte ncclUniqueId
+ * (call on one rank, broadcast the bytes); hios_schedule_nccl_init creates
+ * this rank's communicator (nranks processes, this one = rank, on the device
+ * of its logical GPUs) after hios_schedule_bind_rank.  libnccl.so.2 is
+ * loaded at run time (HIOS_NCCL_LIB overrides the path).  Errors: HIOS_E_NCCL
+ * (library missing, init failed), HIOS_E_UNSUPPORTED (this rank owns logical
+ * GPUs on several devices), HIOS_E_STATE (not in rank mode). */
+hios_status hios_nccl_unique_id(void* id128);
+hios_status hios_schedule_nccl_init(hios_schedule s, const void* id128, int32_t nranks, int32_t rank);
+
+/* The global order of the cross-GPU transfers (one per (producer op,
+ * consumer logical GPU) pair) the NCCL transport posts its sends / receives
+ * in: ascending position of the producer's stage in a topological order of the
+ * stage DAG (data edges + per-GPU stage order), ties by producer id, then
+ * consumer GPU.  src_op / dst_gpu [cap] (caller-owned), *n = count (if the
+ * arrays are NULL only *n is written). */
+hios_status hios_schedule_transfers(hios_schedule s, int32_t* src_op, int32_t* dst_gpu, int32_t cap, int32_t* n);
+
 /* Multi-process execution (one process per GPU): this process executes only
  * the logical GPUs i with owner[i] == rank.  Cross-process edges use CUDA IPC
  * peer memory: after hios_ipc_export on every rank, each rank imports every

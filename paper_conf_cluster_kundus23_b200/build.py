@@ -20,7 +20,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
          "--expt-relaxed-constexpr", "-I", os.path.join(HERE, "..", "include")]
 SOURCES = ["graph.cpp", "sched.cpp", "conv_tc.cu", "conv_simt.cu", "misc.cu", "exec.cu",
-           "profile.cu", "api.cu"]
+           "profile.cu", "nccl.cpp", "api.cu"]
 
 
 def _compile(src: str) -> str:

@@ -262,6 +262,62 @@ static hios::Executor& ensure_exec(hios::Schedule& S) {
   return *S.exec;
 }
 
+hios_status hios_schedule_transport(hios_schedule s, int32_t transport) {
+  return guard([&] {
+    NEED(s, HIOS_E_INVALID, "NULL schedule");
+    NEED(transport == HIOS_TRANSPORT_PEER || transport == HIOS_TRANSPORT_COPY || transport == HIOS_TRANSPORT_NCCL,
+         HIOS_E_INVALID, "unknown transport");
+    NEED(!s->s->exec, HIOS_E_STATE, "set the transport before the first run / IPC export");
+    s->s->transport = transport;
+  });
+}
+
+hios_status hios_nccl_unique_id(void* id128) {
+  return guard([&] {
+    NEED(id128, HIOS_E_INVALID, "NULL id");
+    hios::NcclUniqueId id;
+    hios::nccl_unique_id(&id);
+    memcpy(id128, &id, sizeof(id));
+  });
+}
+
+hios_status hios_schedule_nccl_init(hios_schedule s, const void* id128, int32_t nranks, int32_t rank) {
+  return guard([&] {
+    NEED(s && id128 && nranks >= 1 && rank >= 0 && rank < nranks, HIOS_E_INVALID, "bad argument");
+    auto& S = *s->s;
+    NEED(!S.owner.empty(), HIOS_E_STATE, "NCCL transport: bind ranks first (hios_schedule_bind_rank)");
+    NEED(S.rank == rank, HIOS_E_INVALID, "rank differs from hios_schedule_bind_rank's");
+    NEED(S.transport == HIOS_TRANSPORT_NCCL, HIOS_E_STATE, "set HIOS_TRANSPORT_NCCL first");
+    int dev = -1;
+    for (int l = 0; l < S.M; ++l) {
+      if (S.owner[l] != rank) continue;
+      const int d = S.devices.empty() ? 0 : S.devices[l];
+      NEED(dev < 0 || dev == d, HIOS_E_UNSUPPORTED, "NCCL transport: a rank's logical GPUs must share one device");
+      dev = d;
+    }
+    auto& E = ensure_exec(S);
+    NEED(!E.comm, HIOS_E_STATE, "NCCL already initialised");
+    NEED(!E.captured, HIOS_E_STATE, "initialise NCCL before the first run");
+    hios::NcclUniqueId id;
+    memcpy(&id, id128, sizeof(id));
+    E.comm = hios::nccl_comm_init(dev < 0 ? 0 : dev, id, nranks, rank);
+  });
+}
+
+hios_status hios_schedule_transfers(hios_schedule s, int32_t* src_op, int32_t* dst_gpu, int32_t cap, int32_t* n) {
+  return guard([&] {
+    NEED(s && n, HIOS_E_INVALID, "NULL argument");
+    auto t = hios::transfer_order(*s->s);
+    *n = (int32_t)t.size();
+    if (!src_op && !dst_gpu) return;
+    NEED(src_op && dst_gpu && cap >= (int32_t)t.size(), HIOS_E_INVALID, "arrays too small");
+    for (size_t i = 0; i < t.size(); ++i) {
+      src_op[i] = t[i].first;
+      dst_gpu[i] = t[i].second;
+    }
+  });
+}
+
 // blob: [int32 n][n x { int32 lgpu, cudaIpcMemHandle arena, cudaIpcMemHandle sync }]
 hios_status hios_ipc_export(hios_schedule s, void* blob, size_t* len) {
   return guard([&] {

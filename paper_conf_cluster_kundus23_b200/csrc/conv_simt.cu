@@ -97,7 +97,7 @@ __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
       float y = acc[i][j] * a.scale[n] + a.shift[n];
       if (a.relu) y = fmaxf(y, 0.f);
       a.out[(size_t)m * a.ldo + n] = y;
-      if (a.out2) a.out2[(size_t)m * a.ldo2 + n] = y;
+      for (int d_ = 0; d_ < a.out2.n; ++d_) a.out2.p[d_][(size_t)m * a.out2.ld[d_] + n] = y;
     }
   }
 }

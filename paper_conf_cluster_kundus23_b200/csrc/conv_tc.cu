@@ -375,7 +375,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mw)) : "memory");
     if (a.tma_out) {
       asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mo)) : "memory");
-      if (a.out2) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mo2)) : "memory");
+      if (a.out2.n) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mo2)) : "memory");
     }
   }
   if (warp == kProducers) {
@@ -525,7 +525,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint64_t bres0 = umma_desc_sw128(sB0), bD0h = bres0;
         const bool fixed_ring = !(a.dbg & 32) && ((a.R == 3 && a.S == 3 && KPS >= 2 && KPS <= 4) ||
                                                   (a.R == 5 && a.S == 5 && KPS == 4) ||
-                                                  (a.R == 1 && a.S == 1 && KPS == 1));
+                                                  (a.R == 1 && a.S == 1 && KPS == 1) ||
+                                                  (a.R * a.S == 7 && (a.R == 1 || a.S == 1) && KPS == 4) ||
+                                                  (a.R * a.S == 3 && (a.R == 1 || a.S == 1) && KPS == 3));
         const bool fixed_rs = !(a.dbg & 32) && ((a.R == 3 && a.S == 3) || (a.R == 1 && a.S == 1) ||
                                                 (a.R == 2 && a.S == 1) || (a.R == 4 && a.S == 1) ||
                                                 (a.R == 5 && a.S == 5));
@@ -569,6 +571,10 @@ __global__ void __launch_bounds__(kThreads, 1)
               else if (a.R == 3 && kps == 2) halo_taps_ring<3, 3, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
               else if (a.R == 3 && kps == 4) halo_taps_ring<3, 3, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
               else if (a.R == 5 && kps == 4) halo_taps_ring<5, 5, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 1 && S_ == 7) halo_taps_ring<1, 7, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 7) halo_taps_ring<7, 1, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 1 && S_ == 3) halo_taps_ring<1, 3, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 3 && S_ == 1) halo_taps_ring<3, 1, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
               else halo_taps_ring<1, 1, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
               accum = 1;
               mma_commit_on(aempty0 + 8 * ab, on);
@@ -774,7 +780,6 @@ __global__ void __launch_bounds__(kThreads, 1)
         const bool valid = p < a.P && q < a.Q;
         const size_t pix = (size_t)p * a.Q + q;
         bf16* o1 = a.out + pix * a.ldo + n0;
-        bf16* o2 = a.out2 ? a.out2 + pix * a.ldo2 + n0 : nullptr;
         for (int col = 0; col < a.n_tile; col += 32) {
           const bool two = col + 16 < a.n_tile;  // warp-uniform
           uint32_t r0[16], r1[16];
@@ -813,12 +818,14 @@ __global__ void __launch_bounds__(kThreads, 1)
               if (c8 + 8 <= n_valid) {
                 const uint4 v = make_uint4(pk[4 * v8], pk[4 * v8 + 1], pk[4 * v8 + 2], pk[4 * v8 + 3]);
                 *reinterpret_cast<uint4*>(o1 + c8) = v;
-                if (o2) *reinterpret_cast<uint4*>(o2 + c8) = v;
+                for (int d_ = 0; d_ < a.out2.n; ++d_)
+                  *reinterpret_cast<uint4*>(a.out2.p[d_] + pix * a.out2.ld[d_] + n0 + c8) = v;
               } else {
                 for (int e = 0; e < 8 && c8 + e < n_valid; ++e) {
                   const uint16_t hv = (uint16_t)(pk[4 * v8 + (e >> 1)] >> (16 * (e & 1)));
                   reinterpret_cast<uint16_t*>(o1)[c8 + e] = hv;
-                  if (o2) reinterpret_cast<uint16_t*>(o2)[c8 + e] = hv;
+                  for (int d_ = 0; d_ < a.out2.n; ++d_)
+                    reinterpret_cast<uint16_t*>(a.out2.p[d_] + pix * a.out2.ld[d_] + n0)[c8 + e] = hv;
                 }
               }
             }
@@ -909,7 +916,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (c0 >= a.K) break;
             const uint32_t src = sOut_t + sl * 128u * SWB + (uint32_t)mr * SWB;
             tma_store_3d(&mo, src, c0, q0 + ww0, p0 + hh0);
-            if (a.out2) tma_store_3d(&mo2, src, c0, q0 + ww0, p0 + hh0);
+            if (a.out2.n) tma_store_3d(&mo2, src, c0, q0 + ww0, p0 + hh0);
           }
           bulk_commit();
         }
@@ -948,7 +955,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (p >= a.P || q >= a.Q) continue;
           const size_t pix = (size_t)p * a.Q + q;
           *reinterpret_cast<uint4*>(a.out + pix * a.ldo + n0 + cc4[u] * 8) = v[u];
-          if (a.out2) *reinterpret_cast<uint4*>(a.out2 + pix * a.ldo2 + n0 + cc4[u] * 8) = v[u];
+          for (int d_ = 0; d_ < a.out2.n; ++d_) *reinterpret_cast<uint4*>(a.out2.p[d_] + pix * a.out2.ld[d_] + n0 + cc4[u] * 8) = v[u];
         }
       }
       if (n_valid & 7) {  // channel tail (K % 8 != 0): element copies
@@ -961,7 +968,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           const size_t pix = (size_t)p * a.Q + q;
           const uint16_t v = lds16(sbase + (uint32_t)rr1 * PITCH + (uint32_t)e * 2u);
           reinterpret_cast<uint16_t*>(a.out + pix * a.ldo + n0)[e] = v;
-          if (a.out2) reinterpret_cast<uint16_t*>(a.out2 + pix * a.ldo2 + n0)[e] = v;
+          for (int d_ = 0; d_ < a.out2.n; ++d_) reinterpret_cast<uint16_t*>(a.out2.p[d_] + pix * a.out2.ld[d_] + n0)[e] = v;
         }
       }
       if (tcount == 0 && et == 0) TRACE3(1);
@@ -984,7 +991,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 // sum the split-K partials, folded BN + ReLU, bf16, 16-byte stores
 __global__ void conv_splitk_finalize(const float* __restrict__ ws, int ksplit, size_t ws_split, int ws_ld, int PQ,
                                      int K, const float* __restrict__ scale, const float* __restrict__ shift,
-                                     int relu, bf16* out, int ldo, bf16* out2, int ldo2) {
+                                     int relu, bf16* out, int ldo, Dst<bf16> out2) {
   pdl_enter();
   const int KG = (K + 7) / 8;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
@@ -1006,14 +1013,14 @@ __global__ void conv_splitk_finalize(const float* __restrict__ ws, int ksplit, s
     v[j] = __float2bfloat16_rn(relu ? fmaxf(y, 0.f) : y);
   }
   bf16* d = out + (size_t)pix * ldo + n;
-  bf16* d2 = out2 ? out2 + (size_t)pix * ldo2 + n : nullptr;
   if (n + 8 <= K) {
     *reinterpret_cast<uint4*>(d) = *reinterpret_cast<const uint4*>(v);
-    if (d2) *reinterpret_cast<uint4*>(d2) = *reinterpret_cast<const uint4*>(v);
+    for (int d_ = 0; d_ < out2.n; ++d_)
+      *reinterpret_cast<uint4*>(out2.p[d_] + (size_t)pix * out2.ld[d_] + n) = *reinterpret_cast<const uint4*>(v);
   } else {
     for (int j = 0; n + j < K; ++j) {
       d[j] = v[j];
-      if (d2) d2[j] = v[j];
+      for (int d_ = 0; d_ < out2.n; ++d_) out2.p[d_][(size_t)pix * out2.ld[d_] + n + j] = v[j];
     }
   }
 }
@@ -1021,7 +1028,7 @@ __global__ void conv_splitk_finalize(const float* __restrict__ ws, int ksplit, s
 void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st) {
   const int PQ = a.P * a.Q, KG = (a.K + 7) / 8;
   launch_pdl(conv_splitk_finalize, dim3((PQ * KG + 255) / 256), dim3(256), 0, st, (const float*)a.ws, a.ksplit,
-             a.ws_split, a.ws_ld, PQ, a.K, a.scale, a.shift, a.relu, a.out, a.ldo, a.out2, a.ldo2);
+             a.ws_split, a.ws_ld, PQ, a.K, a.scale, a.shift, a.relu, a.out, a.ldo, a.out2);
 }
 
 size_t conv_tc_smem_bytes(const ConvTcArgs& a) {

@@ -60,6 +60,7 @@ static inline int64_t rup64(int64_t x, int64_t m) { return (x + m - 1) / m * m; 
 
 Executor::Executor(Schedule& sch) : s(sch), g(*sch.g), M(sch.M) {
   esz = g.dtype == HIOS_BF16 ? 2 : 4;
+  transport = sch.transport;
   int ndev = 0;
   ck(cudaGetDeviceCount(&ndev), "cudaGetDeviceCount");
   if (ndev <= 0) fail(HIOS_E_CUDA, "no CUDA device");
@@ -95,6 +96,13 @@ Executor::~Executor() {
     if (L.sync) cudaFree(L.sync);
     for (void* p : L.allocs) cudaFree(p);
   }
+  for (auto& x : xfers) {
+    if (x.ev_ready) cudaEventDestroy(x.ev_ready);
+    if (x.ev_recv) cudaEventDestroy(x.ev_recv);
+  }
+  for (auto& L : lg)
+    if (L.comm) cudaStreamDestroy(L.comm);
+  nccl_comm_destroy(comm);
   for (auto e : op_ev0) if (e) cudaEventDestroy(e);
   for (auto e : op_ev1) if (e) cudaEventDestroy(e);
   if (d_in_stage) cudaFree(d_in_stage);
@@ -172,15 +180,44 @@ void Executor::plan() {
   for (int u = 0; u < n; ++u) {
     const int home = s.gpu_of[u];
     const int kind = g.ops[u].kind;
-    const bool can_fuse = kind == HIOS_OP_CONV || kind == HIOS_OP_MAXPOOL || kind == HIOS_OP_AVGPOOL ||
-                          kind == HIOS_OP_ADD;
-    bool fused_used = false;
+    const bool can_fuse = kind == HIOS_OP_CONV || kind == HIOS_OP_SEPCONV || kind == HIOS_OP_MAXPOOL ||
+                          kind == HIOS_OP_AVGPOOL || kind == HIOS_OP_ADD;
     for (int l = 0; l < M; ++l) {
       if (l == home || !need[u][l]) continue;
-      flag_index[u][l] = nflags[l]++;
-      const bool fuse = can_fuse && !fused_used;
-      fused_used = fused_used || fuse;
-      ox[u].remote.push_back({l, fuse});
+      const bool cross_proc = !s.owner.empty() && s.owner[l] != s.owner[home];
+      int mode;
+      if (transport == HIOS_TRANSPORT_NCCL && cross_proc) mode = DM_NCCL;
+      else if (transport == HIOS_TRANSPORT_PEER) mode = can_fuse ? DM_FUSED : DM_PUSH;
+      else mode = DM_COPY;  // copy transport; NCCL between logical GPUs of one process
+      if (mode != DM_NCCL) flag_index[u][l] = nflags[l]++;
+      ox[u].remote.push_back({l, mode});
+    }
+  }
+  // NCCL transfers in the global order; a transfer whose two buffers are not
+  // both whole [H*W][ldc] tensors with the same pitch goes through packed
+  // [H*W][C] staging buffers on both sides
+  xfers.clear();
+  if (transport == HIOS_TRANSPORT_NCCL) {
+    for (auto& pr : transfer_order(s)) {
+      const int u = pr.first, d = pr.second;
+      bool nc = false;
+      for (auto& r : ox[u].remote)
+        if (r.gpu == d && r.mode == DM_NCCL) nc = true;
+      if (!nc) continue;
+      const Op& o = g.ops[u];
+      NcclXfer x;
+      x.u = u;
+      x.src = s.gpu_of[u];
+      x.dst = d;
+      const int lw = rup(o.C, 8);
+      if (loc[u][x.src].ldc == lw && loc[u][d].ldc == lw) {
+        x.bytes = (size_t)o.H * o.W * lw * esz;
+      } else {
+        x.bytes = (size_t)o.H * o.W * o.C * esz;
+        x.send_off = alloc(x.src, (int64_t)x.bytes);
+        x.recv_off = alloc(d, (int64_t)x.bytes);
+      }
+      xfers.push_back(x);
     }
   }
   for (int l = 0; l < M; ++l) {
@@ -338,6 +375,18 @@ void Executor::allocate() {
     ck(cudaEventCreate(&L.ev_start), "event");
     ck(cudaEventCreate(&L.ev_done), "event");
   }
+  for (auto& x : xfers) {
+    for (int side = 0; side < 2; ++side) {
+      const int l = side ? x.dst : x.src;
+      if (!lg[l].local) continue;
+      ck(cudaSetDevice(lg[l].dev), "cudaSetDevice");
+      if (!lg[l].comm) ck(cudaStreamCreateWithFlags(&lg[l].comm, cudaStreamNonBlocking), "comm stream");
+      cudaEvent_t& e = side ? x.ev_recv : x.ev_ready;
+      ck(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
+    }
+  }
+  if (!xfers.empty() && !comm)
+    fail(HIOS_E_STATE, "NCCL transport: call hios_schedule_nccl_init before the first run");
   for (int v = 0; v < g.n; ++v) {
     const int l = s.gpu_of[v];
     if (!lg[l].local) continue;
@@ -410,6 +459,14 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     const double waves = std::ceil((double)c.tiles_m * tn / 148.0);
     const double cost = waves * tile + 1500.0;
     if (cost < best_cost * 0.98) { best_cost = cost; c.n_tile = nt; }
+  }
+  if (c.vgrid && !g_conv_solo) {
+    // virtual-grid halo next to other ops of its stage: the tap-mode rule
+    // (widest N tile <= 128 that splits K evenly) -- fewer CTAs, since the
+    // stage's concurrent ops already fill the SMs (measured: the cost model's
+    // 64-wide tiles made Inception-1024 HIOS-LP 0.74 -> 0.84 ms)
+    const int nb = (K + 127) / 128;
+    c.n_tile = rup((K + nb - 1) / nb, 16);
   }
   if (!c.halo) {
     // tap mode: the per-stage cost is dominated by a fixed handshake
@@ -521,17 +578,29 @@ struct View {
 };
 
 template <typename T>
+static Dst<T> dst_of(const std::vector<View>& v) {
+  if ((int)v.size() > kMaxDst) fail(HIOS_E_UNSUPPORTED, "more remote destinations than kMaxDst");
+  Dst<T> d{};
+  d.n = (int)v.size();
+  for (size_t i = 0; i < v.size(); ++i) {
+    d.p[i] = (T*)v[i].p;
+    d.ld[i] = v[i].ldc;
+  }
+  return d;
+}
+
+template <typename T>
 static std::function<void(cudaStream_t)> conv_closure(Executor& ex, const View& in, int H, int W, int C,
                                                       const void* w, float* scale, float* shift, int K, int R,
                                                       int S, int sh, int sw, int ph, int pw, int dh, int dw,
-                                                      int P, int Q, int relu, const View& out, const View* out2,
-                                                      int& nk);
+                                                      int P, int Q, int relu, const View& out,
+                                                      const std::vector<View>& out2, int& nk);
 
 template <>
 std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& in, int H, int W, int C, const void* w,
                                                      float* scale, float* shift, int K, int R, int S, int sh, int sw,
                                                      int ph, int pw, int dh, int dw, int P, int Q, int relu,
-                                                     const View& out, const View* out2, int& nk) {
+                                                     const View& out, const std::vector<View>& out2, int& nk) {
   ConvTcArgs a = plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw);
   CUtensorMap mx, mw;
   bool ok;
@@ -565,7 +634,7 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   a.spin = getenv("HIOS_SPIN") ? atoi(getenv("HIOS_SPIN")) : 0;
   a.dbg = getenv("HIOS_DBG") ? atoi(getenv("HIOS_DBG")) : 0;
   a.out = (bf16*)out.p; a.ldo = out.ldc;
-  a.out2 = out2 ? (bf16*)out2->p : nullptr; a.ldo2 = out2 ? out2->ldc : 0;
+  a.out2 = dst_of<bf16>(out2);
   // epilogue by TMA bulk-tensor stores: output tensor map {K, Q, P} over the
   // destination slice (clips the ragged pixel / channel edges of a tile)
   CUtensorMap mo = mx, mo2 = mx;
@@ -579,8 +648,9 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
     const uint32_t bw = (uint32_t)std::min(a.tw, 32), bh = 32u / bw;
     a.tma_out = make_tmap_3d(&mo, out.p, K, Q, P, (uint64_t)out.ldc * 2, (uint64_t)Q * out.ldc * 2, a.out_sw, bw, bh,
                              1, 1, sb) &&
-                (!out2 || make_tmap_3d(&mo2, out2->p, K, Q, P, (uint64_t)out2->ldc * 2,
-                                       (uint64_t)Q * out2->ldc * 2, a.out_sw, bw, bh, 1, 1, sb));
+                (out2.empty() || (out2.size() == 1 && make_tmap_3d(&mo2, out2[0].p, K, Q, P, (uint64_t)out2[0].ldc * 2,
+                                                                   (uint64_t)Q * out2[0].ldc * 2, a.out_sw, bw, bh, 1,
+                                                                   1, sb)));
     if (!a.tma_out) a.epi = 0;
   }
   const size_t smem = conv_tc_smem_bytes(a);
@@ -606,13 +676,13 @@ template <>
 std::function<void(cudaStream_t)> conv_closure<float>(Executor&, const View& in, int H, int W, int C, const void* w,
                                                       float* scale, float* shift, int K, int R, int S, int sh,
                                                       int sw, int ph, int pw, int dh, int dw, int P, int Q, int relu,
-                                                      const View& out, const View* out2, int& nk) {
+                                                      const View& out, const std::vector<View>& out2, int& nk) {
   ConvSimtArgs a{};
   a.x = (const float*)in.p; a.H = H; a.W = W; a.C = C; a.ldx = in.ldc;
   a.w = (const float*)w; a.P = P; a.Q = Q; a.K = K; a.R = R; a.S = S; a.sh = sh; a.sw = sw; a.ph = ph;
   a.pw = pw; a.dh = dh; a.dw = dw; a.relu = relu; a.scale = scale; a.shift = shift;
   a.out = (float*)out.p; a.ldo = out.ldc;
-  a.out2 = out2 ? (float*)out2->p : nullptr; a.ldo2 = out2 ? out2->ldc : 0;
+  a.out2 = dst_of<float>(out2);
   nk += 1;
   return [a](cudaStream_t st) { launch_conv_simt(a, st); };
 }
@@ -626,14 +696,11 @@ static void build_op(Executor& ex, int v) {
   auto view_of = [&](int u, int on) { return View{ex.ptr(on, ex.loc[u][on].off), ex.loc[u][on].ldc}; };
   auto in_op = [&](int k) { return g.edges[o.in_edges[k]].src; };
   const View out = view_of(v, l);
-  // fused remote destination (first remote consumer GPU of a fusable op)
-  View out2v{nullptr, 0};
-  const View* out2 = nullptr;
+  // fused remote destinations: every consumer GPU of a fusable op gets the
+  // epilogue's stores directly (peer memory / aliased logical GPU)
+  std::vector<View> out2;
   for (auto& r : x.remote)
-    if (r.second) {
-      out2v = view_of(v, r.first);
-      out2 = &out2v;
-    }
+    if (r.mode == DM_FUSED) out2.push_back(view_of(v, r.gpu));
   std::vector<std::function<void(cudaStream_t)>> fns;
   int nk = 0;
   switch (o.kind) {
@@ -655,7 +722,7 @@ static void build_op(Executor& ex, int v) {
           if (ex.inplace[e]) own = false;
         c.kst = own ? rup(o.out_c, 8) : o.out_c;
         c.out = (T*)out.p; c.ldo = out.ldc;
-        c.out2 = out2 ? (T*)out2->p : nullptr; c.ldo2 = out2 ? out2->ldc : 0;
+        c.out2 = dst_of<T>(out2);
         auto wp = std::make_shared<Stem3W>();
         std::memset(wp.get(), 0, sizeof(Stem3W));
         for (int k = 0; k < o.out_c; ++k) {
@@ -699,7 +766,7 @@ static void build_op(Executor& ex, int v) {
         c.P = o.H; c.Q = o.W; c.K = o.out_c; c.R = o.kh; c.S = o.kw; c.sh = o.sh; c.sw = o.sw;
         c.ph = o.ph; c.pw = o.pw; c.relu = o.relu;
         c.out = (T*)out.p; c.ldo = out.ldc;
-        c.out2 = out2 ? (T*)out2->p : nullptr; c.ldo2 = out2 ? out2->ldc : 0;
+        c.out2 = dst_of<T>(out2);
         fns.push_back([c](cudaStream_t st) { launch_conv_small_c<T>(c, st); });
         ++nk;
         break;
@@ -737,7 +804,7 @@ static void build_op(Executor& ex, int v) {
         const bool last = r == o.reps - 1;
         fns.push_back(conv_closure<T>(ex, dwv, o.H, o.W, c, x.pw[r], x.scale[r], x.shift[r], o.out_c, 1, 1, 1, 1, 0,
                                       0, 1, 1, o.H, o.W, last ? o.relu : 0, last ? out : midv,
-                                      last ? nullptr : nullptr, nk));
+                                      last ? out2 : std::vector<View>(), nk));
       }
       break;
     }
@@ -751,7 +818,7 @@ static void build_op(Executor& ex, int v) {
       p.P = o.H; p.Q = o.W; p.kh = o.kh; p.kw = o.kw; p.sh = o.sh; p.sw = o.sw; p.ph = o.ph; p.pw = o.pw;
       p.is_max = o.kind == HIOS_OP_MAXPOOL; p.cip = o.cip;
       p.out = (T*)out.p; p.ldo = out.ldc;
-      p.out2 = out2 ? (T*)out2->p : nullptr; p.ldo2 = out2 ? out2->ldc : 0;
+      p.out2 = dst_of<T>(out2);
       fns.push_back([p](cudaStream_t st) { launch_pool<T>(p, st); });
       ++nk;
       break;
@@ -803,7 +870,7 @@ static void build_op(Executor& ex, int v) {
       }
       a.n_in = nin; a.HW = o.H * o.W; a.C = o.C; a.relu = o.relu;
       a.out = (T*)out.p; a.ldo = out.ldc;
-      a.out2 = out2 ? (T*)out2->p : nullptr; a.ldo2 = out2 ? out2->ldc : 0;
+      a.out2 = dst_of<T>(out2);
       fns.push_back([a](cudaStream_t st) { launch_add<T>(a, st); });
       ++nk;
       break;
@@ -853,8 +920,38 @@ static int enqueue_deliver(Executor& ex, int u, cudaStream_t st) {
   const Op& o = ex.g.ops[u];
   int nk = 0;
   for (auto& r : ex.ox[u].remote) {
-    const int d = r.first;
-    if (!r.second) {
+    const int d = r.gpu;
+    if (r.mode == DM_NCCL) {
+      // pack into the send staging buffer if needed; the send itself is
+      // posted on the communication stream in the global order
+      for (auto& x : ex.xfers) {
+        if (x.u != u || x.dst != d) continue;
+        if (x.send_off >= 0) {
+          const Loc& src = ex.loc[u][l];
+          if (ex.g.dtype == HIOS_BF16) {
+            CopyArgs<bf16> c{(const bf16*)ex.ptr(l, src.off), src.ldc, o.H * o.W, o.C, (bf16*)ex.ptr(l, x.send_off), o.C};
+            launch_copy<bf16>(c, st);
+          } else {
+            CopyArgs<float> c{(const float*)ex.ptr(l, src.off), src.ldc, o.H * o.W, o.C, (float*)ex.ptr(l, x.send_off),
+                              o.C};
+            launch_copy<float>(c, st);
+          }
+          ++nk;
+        }
+        ck(cudaEventRecord(x.ev_ready, st), "record send-ready");
+      }
+      continue;
+    }
+    if (r.mode == DM_COPY) {
+      // copy-engine transfer after the producer finished (the paper's
+      // "launch after the transfer completes" design): a strided
+      // 2-D copy (C channels per pixel, pixel pitches of both buffers)
+      const Loc& src = ex.loc[u][l];
+      const Loc& dst = ex.loc[u][d];
+      ck(cudaMemcpy2DAsync(ex.ptr(d, dst.off), (size_t)dst.ldc * ex.esz, ex.ptr(l, src.off), (size_t)src.ldc * ex.esz,
+                           (size_t)o.C * ex.esz, (size_t)o.H * o.W, cudaMemcpyDefault, st),
+         "cudaMemcpy2DAsync (copy transport)");
+    } else if (r.mode == DM_PUSH) {
       const Loc& src = ex.loc[u][l];
       const Loc& dst = ex.loc[u][d];
       if (ex.g.dtype == HIOS_BF16) {
@@ -879,19 +976,61 @@ void Executor::enqueue_stage_program(int l, bool timed) {
   int64_t nk = 0;
   launch_epoch(L.sync, s0);
   ++nk;
-  // back-pressure: do not overwrite a consumer GPU's buffers before it finished the previous run
+  // back-pressure: do not overwrite a consumer GPU's buffers before it finished
+  // the previous run (flag transports; NCCL receives land in the consumer's
+  // own stream order)
   std::set<int> consumers, producers;
   for (int v = 0; v < g.n; ++v) {
-    if (s.gpu_of[v] == l)
-      for (auto& r : ox[v].remote) consumers.insert(r.first);
-    else
-      for (int m = 0; m < M; ++m)
-        if (m == l && flag_index[v][l] >= 0) producers.insert(s.gpu_of[v]);
+    if (s.gpu_of[v] == l) {
+      for (auto& r : ox[v].remote)
+        if (r.mode != DM_NCCL) consumers.insert(r.gpu);
+    } else if (flag_index[v][l] >= 0) {
+      producers.insert(s.gpu_of[v]);
+    }
   }
   for (int c : consumers) {
     launch_wait(L.sync, L.sync + 1 + c, 1, s0);
     ++nk;
   }
+  // NCCL: this GPU's sends / receives in the global transfer order on its
+  // communication stream (forked from and joined back into s0)
+  std::vector<int> acts;
+  for (int k = 0; k < (int)xfers.size(); ++k)
+    if (xfers[k].src == l || xfers[k].dst == l) acts.push_back(k);
+  size_t next = 0;
+  std::vector<char> ready(xfers.size(), 0);
+  if (!acts.empty()) {
+    ck(cudaEventRecord(L.ev_fork, s0), "fork comm");
+    ck(cudaStreamWaitEvent(L.comm, L.ev_fork, 0), "fork comm wait");
+  }
+  auto post = [&](size_t upto) {
+    for (; next < upto; ++next) {
+      NcclXfer& x = xfers[acts[next]];
+      const Op& o = g.ops[x.u];
+      if (x.src == l) {
+        if (!ready[acts[next]])
+          fail(HIOS_E_STATE, "NCCL transfer order inconsistent with the stage order (op " + std::to_string(x.u) + ")");
+        ck(cudaStreamWaitEvent(L.comm, x.ev_ready, 0), "wait send-ready");
+        const void* p = x.send_off >= 0 ? ptr(l, x.send_off) : ptr(l, loc[x.u][l].off);
+        nccl_send(p, x.bytes, s.owner[x.dst], comm, L.comm);
+      } else {
+        void* p = x.recv_off >= 0 ? ptr(l, x.recv_off) : ptr(l, loc[x.u][l].off);
+        nccl_recv(p, x.bytes, s.owner[x.src], comm, L.comm);
+        if (x.recv_off >= 0) {  // unpack into the consumer's location (slice / pitch)
+          const Loc& d = loc[x.u][l];
+          if (g.dtype == HIOS_BF16) {
+            CopyArgs<bf16> c{(const bf16*)p, o.C, o.H * o.W, o.C, (bf16*)ptr(l, d.off), d.ldc};
+            launch_copy<bf16>(c, L.comm);
+          } else {
+            CopyArgs<float> c{(const float*)p, o.C, o.H * o.W, o.C, (float*)ptr(l, d.off), d.ldc};
+            launch_copy<float>(c, L.comm);
+          }
+          ++nk;
+        }
+        ck(cudaEventRecord(x.ev_recv, L.comm), "record recv");
+      }
+    }
+  };
   for (auto& S : s.Q[l]) {
     std::set<int> waits;
     for (int v : S)
@@ -900,6 +1039,16 @@ void Executor::enqueue_stage_program(int l, bool timed) {
         if (s.gpu_of[u] != l) waits.insert(u);
       }
     for (int u : waits) {
+      if (flag_index[u][l] < 0) {  // NCCL: post up to this receive, then wait for it
+        for (size_t i = 0; i < acts.size(); ++i) {
+          const NcclXfer& x = xfers[acts[i]];
+          if (x.u == u && x.dst == l) {
+            post(std::max(next, i + 1));
+            ck(cudaStreamWaitEvent(s0, x.ev_recv, 0), "wait recv");
+          }
+        }
+        continue;
+      }
       launch_wait(L.sync, L.sync + 1 + M + flag_index[u][l], 0, s0);
       ++nk;
     }
@@ -910,6 +1059,8 @@ void Executor::enqueue_stage_program(int l, bool timed) {
       if (timed) ck(cudaEventRecordWithFlags(op_ev1[v], st, cudaEventRecordExternal), "event record");
       nk += solo ? ox[v].n_kernels_solo : ox[v].n_kernels;
       nk += enqueue_deliver(*this, v, st);
+      for (int k : acts)
+        if (xfers[k].u == v && xfers[k].src == l) ready[k] = 1;
     };
     if (S.size() == 1) {
       run_one(S[0], s0);
@@ -922,6 +1073,11 @@ void Executor::enqueue_stage_program(int l, bool timed) {
         ck(cudaStreamWaitEvent(s0, L.ev_join[k], 0), "join wait");
       }
     }
+  }
+  if (!acts.empty()) {
+    post(acts.size());
+    ck(cudaEventRecord(L.ev_join[0], L.comm), "join comm");
+    ck(cudaStreamWaitEvent(s0, L.ev_join[0], 0), "join comm wait");
   }
   for (int p : producers) {
     launch_signal(L.sync, lg[p].sync + 1 + l, s0);

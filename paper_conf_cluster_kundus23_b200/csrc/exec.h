@@ -8,6 +8,24 @@
 
 namespace hios {
 
+// NCCL transport (nccl.cpp; libnccl.so.2 loaded at run time)
+struct NcclUniqueId { char internal[128]; };
+typedef struct ncclComm* NcclComm;
+void nccl_unique_id(NcclUniqueId* id);
+NcclComm nccl_comm_init(int dev, const NcclUniqueId& id, int nranks, int rank);
+void nccl_comm_destroy(NcclComm c);
+void nccl_send(const void* buf, size_t bytes, int peer, NcclComm c, cudaStream_t st);
+void nccl_recv(void* buf, size_t bytes, int peer, NcclComm c, cudaStream_t st);
+// global order of the (producer op, consumer logical GPU) transfers
+std::vector<std::pair<int, int>> transfer_order(const Schedule& s);
+
+// how one (producer, consumer GPU) edge is carried
+enum DeliverMode { DM_FUSED = 0, DM_PUSH = 1, DM_COPY = 2, DM_NCCL = 3 };
+struct Remote {
+  int gpu;   // consumer logical GPU
+  int mode;  // DeliverMode
+};
+
 struct Loc {
   int64_t off = -1;  // byte offset in the owning logical GPU's arena
   int ldc = 0;       // pixel stride in elements
@@ -31,8 +49,8 @@ struct OpExec {
   // s2d stem with its S' taps packed into one 64-element K row (overlapping
   // 4-pixel windows of the s2d tensor; weights W''[k][r'][s'*16 + ch])
   void* w_pack = nullptr;
-  // remote deliveries of this op's output: (consumer lgpu, fused-into-epilogue?)
-  std::vector<std::pair<int, bool>> remote;
+  // remote deliveries of this op's output
+  std::vector<Remote> remote;
   std::function<void(cudaStream_t)> run;  // enqueue the op's kernels (incl. fused out2)
   int n_kernels = 0;
   // the same op configured to run alone (a singleton stage / t(v) profiling):
@@ -55,6 +73,16 @@ struct LGpu {
   size_t sync_words = 0;
   std::vector<void*> allocs;   // weights etc. (owned)
   bool ipc_mapped = false;
+  cudaStream_t comm = nullptr;  // NCCL transport: send/recv stream
+};
+
+// one NCCL transfer of the global order, as this process sees it
+struct NcclXfer {
+  int u = -1, src = -1, dst = -1;  // producer op, producer / consumer logical GPU
+  int64_t send_off = -1, recv_off = -1;  // staging (packed H*W*C) or -1: direct
+  size_t bytes = 0;
+  cudaEvent_t ev_ready = nullptr;  // producer: op u finished (on its GPU)
+  cudaEvent_t ev_recv = nullptr;   // consumer: data landed
 };
 
 struct Executor {
@@ -68,6 +96,9 @@ struct Executor {
   std::vector<OpExec> ox;
   std::vector<std::vector<int>> flag_index;  // [op][lgpu] flag slot on that lgpu (-1 none)
   int n_streams = 1;
+  int transport = HIOS_TRANSPORT_PEER;  // cross-GPU edge transport (hios_schedule_transport)
+  NcclComm comm = nullptr;              // NCCL transport: this rank's communicator
+  std::vector<NcclXfer> xfers;          // NCCL transfers in the global order
   int cur_lgpu = 0;  // logical GPU whose closures are being built
   bool lowered = false, captured = false;
   int64_t kernels_per_run = 0;

@@ -82,6 +82,7 @@ struct Schedule {
   std::vector<int> devices;  // per logical GPU
   std::vector<int> owner;    // per logical GPU: process rank (empty = all local)
   int rank = 0;
+  int transport = HIOS_TRANSPORT_PEER;
   std::unique_ptr<Executor> exec;
   ~Schedule();
 };

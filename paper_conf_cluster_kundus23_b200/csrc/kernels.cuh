@@ -45,6 +45,18 @@ inline cudaError_t launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t
   return cudaLaunchKernelEx(&cfg, k, std::forward<Args>(args)...);
 }
 
+// Remote replicas of an op's output (cross-GPU edges fused into the
+// producer's epilogue): one per consumer GPU other than the
+// producer's; each store of the output is repeated into every replica (peer
+// memory over NVLink, or an aliased logical GPU's buffer).
+constexpr int kMaxDst = 7;
+template <typename T>
+struct Dst {
+  T* p[kMaxDst];
+  int ld[kMaxDst];  // pixel stride (elements)
+  int n;
+};
+
 // ------------------------------------------------------------------ conv
 // Implicit-GEMM convolution on tcgen05 tensor cores (bf16 in, fp32 TMEM
 // accumulate, bf16 out).  GEMM view: M = output pixels (tile = th x tw = 128
@@ -71,7 +83,7 @@ struct ConvTcArgs {
   const float* scale;  // [K]
   const float* shift;  // [K]
   bf16* out;  int ldo; // primary output (channel offset applied)
-  bf16* out2; int ldo2;// optional second destination (peer replica), or null
+  Dst<bf16> out2;      // remote replicas (fused cross-GPU stores)
   int bres;            // halo mode, one N tile: all weights resident in smem (loaded once per CTA)
   int tma_out;         // epilogue leaves smem by TMA bulk-tensor stores (else st.global)
   int out_sw;          // TMA-store slab width in channels (64 / 32 / 16 = 128B/64B/32B swizzle)
@@ -97,7 +109,7 @@ struct ConvSimtArgs {
   int P, Q, K, R, S, sh, sw, ph, pw, dh, dw, relu;
   const float* scale; const float* shift;
   float* out; int ldo;
-  float* out2; int ldo2;
+  Dst<float> out2;
 };
 
 // Depthwise stage of a separable conv: a = sum_i agg_i x_i ; relu? ; depthwise.
@@ -115,7 +127,7 @@ struct PoolArgs {
   const T* x; int H, W, C, ldx;
   int P, Q, kh, kw, sh, sw, ph, pw, is_max, cip;
   T* out; int ldo;
-  T* out2; int ldo2;
+  Dst<T> out2;
 };
 
 template <typename T>
@@ -123,7 +135,7 @@ struct AddArgs {
   const T* x[HIOS_MAX_IN]; int ldx[HIOS_MAX_IN]; float agg[HIOS_MAX_IN]; int n_in;
   int HW, C, relu;
   T* out; int ldo;
-  T* out2; int ldo2;
+  Dst<T> out2;
 };
 
 // direct conv for C <= 8 input channels (stems): fp32 weights [K][R][S][C]
@@ -132,7 +144,7 @@ struct ConvSmallArgs {
   const T* x; int H, W, C, ldx;
   const float* w; const float* scale; const float* shift;
   int P, Q, K, R, S, sh, sw, ph, pw, relu;
-  T* out; int ldo; T* out2; int ldo2;
+  T* out; int ldo; Dst<T> out2;
 };
 
 // space-to-depth of a stride-2 small-C stem input (exec.cu: s2d_conv)
@@ -171,7 +183,7 @@ struct ConvStem3Args {
   const T* x; int H, W, ldx;
   int P, Q, K, ph, pw, relu;
   int kst;  // channels stored per pixel: K, or rup(K, 8) when the pad channels are this op's own
-  T* out; int ldo; T* out2; int ldo2;
+  T* out; int ldo; Dst<T> out2;
 };
 template <typename T> void launch_conv_stem3(const ConvStem3Args<T>& a, const Stem3W& w, cudaStream_t st);
 

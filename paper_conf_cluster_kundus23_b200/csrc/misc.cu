@@ -134,7 +134,7 @@ __global__ void pool_kernel(const PoolArgs<T> a) {
       const size_t pix = (size_t)p * a.Q + q;
       const uint4 o = *reinterpret_cast<const uint4*>(m);
       *reinterpret_cast<uint4*>(a.out + pix * a.ldo + c) = o;
-      if (a.out2) *reinterpret_cast<uint4*>(a.out2 + pix * a.ldo2 + c) = o;
+      for (int d_ = 0; d_ < a.out2.n; ++d_) *reinterpret_cast<uint4*>(a.out2.p[d_] + pix * a.out2.ld[d_] + c) = o;
       return;
     }
     if (!a.is_max && c + 8 <= a.C) {
@@ -166,7 +166,7 @@ __global__ void pool_kernel(const PoolArgs<T> a) {
       for (int j = 0; j < 8; ++j) acc[j] *= inv;
       const size_t pix = (size_t)p * a.Q + q;
       store8(a.out + pix * a.ldo + c, c, a.C, acc);
-      if (a.out2) store8(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+      for (int d_ = 0; d_ < a.out2.n; ++d_) store8(a.out2.p[d_] + pix * a.out2.ld[d_] + c, c, a.C, acc);
       return;
     }
   }
@@ -201,7 +201,7 @@ __global__ void pool_kernel(const PoolArgs<T> a) {
   }
   const size_t pix = (size_t)p * a.Q + q;
   store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
-  if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+  for (int d_ = 0; d_ < a.out2.n; ++d_) store_vec(a.out2.p[d_] + pix * a.out2.ld[d_] + c, c, a.C, acc);
 }
 
 // Tiled pooling (same tiling as the depthwise kernel below): a CTA stages
@@ -283,12 +283,12 @@ __global__ void __launch_bounds__(256) pool_tiled_kernel(const PoolArgs<T> a) {
         const uint4 o = *reinterpret_cast<const uint4*>(m);
         if (c + 8 <= a.C) {
           *reinterpret_cast<uint4*>(a.out + pix * a.ldo + c) = o;
-          if (a.out2) *reinterpret_cast<uint4*>(a.out2 + pix * a.ldo2 + c) = o;
+          for (int d_ = 0; d_ < a.out2.n; ++d_) *reinterpret_cast<uint4*>(a.out2.p[d_] + pix * a.out2.ld[d_] + c) = o;
         } else {
           const bf16* e = reinterpret_cast<const bf16*>(&o);
           for (int j = 0; j < 8 && c + j < a.C; ++j) {
             a.out[pix * a.ldo + c + j] = e[j];
-            if (a.out2) a.out2[pix * a.ldo2 + c + j] = e[j];
+            for (int d_ = 0; d_ < a.out2.n; ++d_) a.out2.p[d_][pix * a.out2.ld[d_] + c + j] = e[j];
           }
         }
       }
@@ -326,7 +326,7 @@ __global__ void __launch_bounds__(256) pool_tiled_kernel(const PoolArgs<T> a) {
         for (int j = 0; j < 8; ++j) acc[j] *= inv;
         const size_t pix = (size_t)p * a.Q + q;
         store8(a.out + pix * a.ldo + c, c, a.C, acc);
-        if (a.out2) store8(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+        for (int d_ = 0; d_ < a.out2.n; ++d_) store8(a.out2.p[d_] + pix * a.out2.ld[d_] + c, c, a.C, acc);
       }
       return;
     }
@@ -366,7 +366,7 @@ __global__ void __launch_bounds__(256) pool_tiled_kernel(const PoolArgs<T> a) {
     }
     const size_t pix = (size_t)p * a.Q + q;
     store8(a.out + pix * a.ldo + c, c, a.C, acc);
-    if (a.out2) store8(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+    for (int d_ = 0; d_ < a.out2.n; ++d_) store8(a.out2.p[d_] + pix * a.out2.ld[d_] + c, c, a.C, acc);
   }
 }
 
@@ -430,7 +430,7 @@ __global__ void __launch_bounds__(256) pool_avg64_kernel(const PoolArgs<bf16> a)
     for (int k = 0; k < 8; ++k) acc[k] *= inv;
     const size_t pix = (size_t)p * a.Q + q;
     store8(a.out + pix * a.ldo + c, c, a.C, acc);
-    if (a.out2) store8(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+    for (int d_ = 0; d_ < a.out2.n; ++d_) store8(a.out2.p[d_] + pix * a.out2.ld[d_] + c, c, a.C, acc);
   }
 }
 
@@ -514,7 +514,7 @@ __global__ void __launch_bounds__(256) pool_rows_kernel(const PoolArgs<T> a, int
     }
     const size_t pix = (size_t)p * a.Q + q;
     store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
-    if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+    for (int d_ = 0; d_ < a.out2.n; ++d_) store_vec(a.out2.p[d_] + pix * a.out2.ld[d_] + c, c, a.C, acc);
     h += SS;
   }
 }
@@ -946,7 +946,7 @@ __global__ void add_kernel(const AddArgs<T> a) {
         for (int j = 0; j < N; ++j) acc[j] = fmaxf(acc[j], 0.f);
       }
       store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
-      if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+      for (int d_ = 0; d_ < a.out2.n; ++d_) store_vec(a.out2.p[d_] + pix * a.out2.ld[d_] + c, c, a.C, acc);
       return;
     }
   }
@@ -960,7 +960,7 @@ __global__ void add_kernel(const AddArgs<T> a) {
     for (int j = 0; j < N; ++j) acc[j] = fmaxf(acc[j], 0.f);
   }
   store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
-  if (a.out2) store_vec(a.out2 + pix * a.ldo2 + c, c, a.C, acc);
+  for (int d_ = 0; d_ < a.out2.n; ++d_) store_vec(a.out2.p[d_] + pix * a.out2.ld[d_] + c, c, a.C, acc);
 }
 
 template <typename T>
@@ -1303,7 +1303,7 @@ __global__ void __launch_bounds__(128) conv_small_c_kernel(const ConvSmallArgs<T
         const int k = k0 + kb + half;
         if (k >= a.K) break;
         store_vec(a.out + pix * a.ldo + k, k, a.K, acc[u] + half);
-        if (a.out2) store_vec(a.out2 + pix * a.ldo2 + k, k, a.K, acc[u] + half);
+        for (int d_ = 0; d_ < a.out2.n; ++d_) store_vec(a.out2.p[d_] + pix * a.out2.ld[d_] + k, k, a.K, acc[u] + half);
       }
     }
   }
@@ -1409,7 +1409,7 @@ __global__ void __launch_bounds__(128) conv_stem3_kernel(const ConvStem3Args<T> 
       if (kb + c0 >= a.K) break;
       // (pad channels past K, when stored, are exact zeros: zero weights, scale and shift)
       store_vec(a.out + pix * a.ldo + kb + c0, kb + c0, a.kst, acc[u] + c0);
-      if (a.out2) store_vec(a.out2 + pix * a.ldo2 + kb + c0, kb + c0, a.kst, acc[u] + c0);
+      for (int d_ = 0; d_ < a.out2.n; ++d_) store_vec(a.out2.p[d_] + pix * a.out2.ld[d_] + kb + c0, kb + c0, a.kst, acc[u] + c0);
     }
   }
 }

@@ -81,6 +81,10 @@ def load() -> C.CDLL:
         "hios_read_op_output": [VP, I32, P(C.c_float), I64],
         "hios_kernel_count": [VP, P(I64)],
         "hios_time_ops": [VP, I32, I64, P(I64)],
+        "hios_schedule_transport": [VP, I32],
+        "hios_nccl_unique_id": [VP],
+        "hios_schedule_nccl_init": [VP, VP, I32, I32],
+        "hios_schedule_transfers": [VP, P(I32), P(I32), I32, P(I32)],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -169,11 +173,35 @@ def pack_ops(ops: Sequence, weights: Optional[Dict[int, Dict]] = None):
                 sh = np.ascontiguousarray(w["shift"], dtype=np.float32)
         if "agg" in w:
             ag = np.ascontiguousarray(w["agg"], dtype=np.float32)
+        _check_sizes(a, wt, sc, sh, ag, getattr(o, "n_in", None))
         for x in (wt, sc, sh, ag):
             if x is not None:
                 keep.append(x)
         a.weight, a.scale, a.shift, a.agg = _fptr(wt), _fptr(sc), _fptr(sh), _fptr(ag)
     return arr, keep
+
+
+def _check_sizes(a, wt, sc, sh, ag, n_in):
+    """The library copies fixed counts from these arrays (include/hios.h hios_op
+    weight layouts): a wrongly sized array would be an out-of-bounds read."""
+    k = a.kind
+    exp = {}
+    if k == KIND["conv"]:
+        exp = {"weight": a.out_c * a.in_c * a.kh * a.kw, "scale": a.out_c, "shift": a.out_c}
+    elif k == KIND["sepconv"]:
+        reps = max(a.reps, 1)
+        tot, c = 0, a.in_c
+        for _ in range(reps):
+            tot += c * a.kh * a.kw + a.out_c * c
+            c = a.out_c
+        exp = {"weight": tot, "scale": reps * a.out_c, "shift": reps * a.out_c}
+    elif k == KIND["linear"]:
+        exp = {"weight": a.out_c * a.in_c, "shift": a.out_c}
+    for name, arr in (("weight", wt), ("scale", sc), ("shift", sh)):
+        if arr is not None and name in exp and arr.size != exp[name]:
+            raise HiosError(1, f"op kind {k}: {name} has {arr.size} elements, expected {exp[name]}")
+    if ag is not None and n_in is not None and ag.size != int(n_in):
+        raise HiosError(1, f"op kind {k}: agg has {ag.size} elements, expected {n_in} (one per input)")
 
 
 def pack_edges(edges: Sequence, costs: Optional[Sequence[int]] = None):
@@ -194,7 +222,9 @@ def hios_graph_create(ops, edges, in_c: int, in_h: int, in_w: int, dtype="bf16",
     _ck(lib.hios_graph_create(oa, len(ops), ea, len(edges), in_c, in_h, in_w,
                               DTYPE[dtype] if isinstance(dtype, str) else int(dtype), C.byref(h)))
     del keep
-    return Graph(h, len(ops), len(edges))
+    gr = Graph(h, len(ops), len(edges))
+    gr.in_numel = int(in_c) * int(in_h) * int(in_w)
+    return gr
 
 
 def hios_graph_shape(g: Graph, op: int):
@@ -302,6 +332,37 @@ def hios_schedule_bind_rank(s: Schedule, owner: Sequence[int], rank: int):
     _ck(load().hios_schedule_bind_rank(s.h, d.ctypes.data_as(C.POINTER(C.c_int32)), len(d), rank))
 
 
+TRANSPORT = {"peer": 0, "copy": 1, "nccl": 2}
+
+
+def hios_schedule_transport(s: Schedule, transport):
+    t = TRANSPORT[transport] if isinstance(transport, str) else int(transport)
+    _ck(load().hios_schedule_transport(s.h, t))
+
+
+def hios_nccl_unique_id() -> bytes:
+    buf = C.create_string_buffer(128)
+    _ck(load().hios_nccl_unique_id(buf))
+    return buf.raw
+
+
+def hios_schedule_nccl_init(s: Schedule, uid: bytes, nranks: int, rank: int):
+    assert len(uid) == 128
+    buf = C.create_string_buffer(uid, 128)
+    _ck(load().hios_schedule_nccl_init(s.h, buf, nranks, rank))
+
+
+def hios_schedule_transfers(s: Schedule):
+    """[(producer op, consumer logical GPU)] in the NCCL transport's global order."""
+    n = C.c_int32()
+    _ck(load().hios_schedule_transfers(s.h, None, None, 0, C.byref(n)))
+    a = np.zeros(max(n.value, 1), dtype=np.int32)
+    b = np.zeros(max(n.value, 1), dtype=np.int32)
+    _ck(load().hios_schedule_transfers(s.h, a.ctypes.data_as(C.POINTER(C.c_int32)),
+                                       b.ctypes.data_as(C.POINTER(C.c_int32)), len(a), C.byref(n)))
+    return [(int(a[i]), int(b[i])) for i in range(n.value)]
+
+
 def hios_ipc_export(s: Schedule) -> bytes:
     n = C.c_size_t(0)
     _ck(load().hios_ipc_export(s.h, None, C.byref(n)))
@@ -325,6 +386,9 @@ def hios_output_numel(s: Schedule) -> int:
 def hios_run(s: Schedule, x: Optional[np.ndarray]) -> np.ndarray:
     out = np.zeros(hios_output_numel(s), dtype=np.float32)
     xin = None if x is None else np.ascontiguousarray(x, dtype=np.float32)
+    want = getattr(s.graph, "in_numel", None)
+    if xin is not None and want is not None and xin.size != want:
+        raise HiosError(1, f"input has {xin.size} elements, expected in_c*in_h*in_w = {want}")
     _ck(load().hios_run(s.h, _fptr(xin), _fptr(out)))
     return out
 

@@ -12,11 +12,23 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
+def _n_gpus():
+    import torch
+    return torch.cuda.device_count()
+
+
+@pytest.mark.parametrize("transport", ["peer", "copy", "nccl"])
 @pytest.mark.parametrize("model,size", [("tiny", "56"), ("inception_v3", "299")])
-def test_two_process_ipc_run(model, size):
+def test_two_process_ipc_run(model, size, transport):
+    """peer: fused epilogue stores into the IPC-mapped consumer buffer; copy:
+    copy-engine transfer after the producer (P:286's launch-after-transfer);
+    nccl: ncclSend/ncclRecv in the global transfer order (needs 2 devices:
+    NCCL rejects two ranks on one GPU)."""
+    if transport == "nccl" and _n_gpus() < 2:
+        pytest.skip("NCCL transport needs one device per rank (this box has one GPU)")
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", "--master-port=29533", os.path.join(ROOT, "tools", "mp_check.py"),
-           model, size]
+           model, size, transport]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     assert "bit-identical to 1-process run: True" in r.stdout
