@@ -314,10 +314,11 @@ __device__ __forceinline__ void tile_pixel(const ConvTcArgs& a, int m_blk, int p
 
 __host__ __device__ inline uint32_t stage_pitch(int n_tile) { return (uint32_t)n_tile * 2u + 16u; }
 
-__global__ void __launch_bounds__(kThreads, 1)
-    conv_tc_kernel(const __grid_constant__ CUtensorMap mx, const __grid_constant__ CUtensorMap mw,
-                   const __grid_constant__ CUtensorMap mo, const __grid_constant__ CUtensorMap mo2,
-                   const ConvTcArgs a) {
+// One conv's persistent tile loop on CTAs cta = 0..ncta-1 of its SM range
+// (conv_tc_kernel: the whole grid; conv_tc_group_kernel: the op's partition).
+__device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUtensorMap* pmw,
+                                             const CUtensorMap* pmo, const CUtensorMap* pmo2, const ConvTcArgs& a,
+                                             const int cta, const int ncta) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int ST = a.stages;
@@ -371,11 +372,11 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(tempty0 + 8 * i, 32 * kEpi);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mx)) : "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mw)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(pmx)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(pmw)) : "memory");
     if (a.tma_out) {
-      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mo)) : "memory");
-      if (a.out2.n) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mo2)) : "memory");
+      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(pmo)) : "memory");
+      if (a.out2.n) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(pmo2)) : "memory");
     }
   }
   if (warp == kProducers) {
@@ -418,13 +419,13 @@ __global__ void __launch_bounds__(kThreads, 1)
           mbar_expect_tx(bres_bar, (uint32_t)nb * B_BYTES);
           for (int i = 0; i < nb; ++i) {
             const int c2 = i / RS;
-            tma_load_3d(sB0 + (uint32_t)i * B_BYTES, &mw, bres_bar, c2 * 64, i - c2 * RS, 0);
+            tma_load_3d(sB0 + (uint32_t)i * B_BYTES, pmw, bres_bar, c2 * 64, i - c2 * RS, 0);
           }
         }
         __syncwarp();
       }
       if (a.bres) mine = 1 << 30;  // no B ring
-      for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+      for (int tile = cta; tile < tiles; tile += ncta) {
         const int split = tile / tiles_mn, tmn = tile - split * tiles_mn;
         const int m_blk = tmn / a.tiles_n, n_blk = tmn - m_blk * a.tiles_n;
         const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
@@ -446,7 +447,7 @@ __global__ void __launch_bounds__(kThreads, 1)
                 mbar_arrive(afull0 + 8 * ab);
               } else {
                 mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.hrows * a.halo_w * 128u);
-                tma_load_3d(sA0 + ab * H_BYTES, &mx, afull0 + 8 * ab, cc * 64, x0, y0);
+                tma_load_3d(sA0 + ab * H_BYTES, pmx, afull0 + 8 * ab, cc * 64, x0, y0);
               }
             }
             __syncwarp();
@@ -472,9 +473,9 @@ __global__ void __launch_bounds__(kThreads, 1)
                 c2 = cc; rs2 = rs; r2 = r; s2 = s;
                 for (int j = 0; j < cnt; ++j) {
                   if (!a.halo)
-                    tma_load_3d(sA0 + st * A_STAGE + j * A_BYTES, &mx, full0 + 8 * st, c2 * 64, x0 + s2 * a.dw,
+                    tma_load_3d(sA0 + st * A_STAGE + j * A_BYTES, pmx, full0 + 8 * st, c2 * 64, x0 + s2 * a.dw,
                                 y0 + r2 * a.dh);
-                  tma_load_3d(sB0 + st * B_STAGE + j * B_BYTES, &mw, full0 + 8 * st, c2 * 64, rs2, n0);
+                  tma_load_3d(sB0 + st * B_STAGE + j * B_BYTES, pmw, full0 + 8 * st, c2 * 64, rs2, n0);
                   if (++s2 == a.S) { s2 = 0; ++r2; }
                   if (++rs2 == RS) { rs2 = 0; r2 = 0; s2 = 0; ++c2; }
                 }
@@ -531,7 +532,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const bool fixed_rs = !(a.dbg & 32) && ((a.R == 3 && a.S == 3) || (a.R == 1 && a.S == 1) ||
                                                 (a.R == 2 && a.S == 1) || (a.R == 4 && a.S == 1) ||
                                                 (a.R == 5 && a.S == 5));
-        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
+        for (int tile = cta; tile < tiles; tile += ncta, ++tcount) {
           mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
           tc_fence_after();
           const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
@@ -626,7 +627,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t ST_ = (uint32_t)ST;
         const uint64_t aD0 = umma_desc_sw128(sA0), bD0 = umma_desc_sw128(sB0);
         const uint64_t ast16 = A_STAGE >> 4, bst16 = B_STAGE >> 4, a16 = A_BYTES >> 4, b16 = B_BYTES >> 4;
-        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
+        for (int tile = cta; tile < tiles; tile += ncta, ++tcount) {
           mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
           tc_fence_after();
           const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
@@ -689,7 +690,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
     }
-    for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++tcount) {
+    for (int tile = cta; tile < tiles; tile += ncta, ++tcount) {
       const int split = tile / tiles_mn, tmn = tile - split * tiles_mn;
       const int m_blk = tmn / a.tiles_n, n_blk = tmn - m_blk * a.tiles_n;
       const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
@@ -915,8 +916,8 @@ __global__ void __launch_bounds__(kThreads, 1)
             const int c0 = n0 + (int)(sl << sw_log);
             if (c0 >= a.K) break;
             const uint32_t src = sOut_t + sl * 128u * SWB + (uint32_t)mr * SWB;
-            tma_store_3d(&mo, src, c0, q0 + ww0, p0 + hh0);
-            if (a.out2.n) tma_store_3d(&mo2, src, c0, q0 + ww0, p0 + hh0);
+            tma_store_3d(pmo, src, c0, q0 + ww0, p0 + hh0);
+            if (a.out2.n) tma_store_3d(pmo2, src, c0, q0 + ww0, p0 + hh0);
           }
           bulk_commit();
         }
@@ -988,6 +989,25 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
 }
 
+__global__ void __launch_bounds__(kThreads, 1)
+    conv_tc_kernel(const __grid_constant__ CUtensorMap mx, const __grid_constant__ CUtensorMap mw,
+                   const __grid_constant__ CUtensorMap mo, const __grid_constant__ CUtensorMap mo2,
+                   const ConvTcArgs a) {
+  conv_tc_body(&mx, &mw, &mo, &mo2, a, blockIdx.x, gridDim.x);
+}
+
+// A stage's convolutions in ONE launch (the stage's
+// concurrent group as one kernel partitioning the SMs across its operators,
+// P:84-86): CTAs [cta0[i], cta0[i+1]) run op i's persistent tile loop.  The
+// partition is explicit (sized by each op's work, exec.cu plan_group), so no op
+// of the stage can occupy SMs its peers need, and the stage costs one launch.
+__global__ void __launch_bounds__(kThreads, 1) conv_tc_group_kernel(const __grid_constant__ ConvTcGroup G) {
+  int i = 0;
+  while (i + 1 < G.n && (int)blockIdx.x >= G.cta0[i + 1]) ++i;
+  const ConvTcOp& o = G.op[i];
+  conv_tc_body(&o.mx, &o.mw, &o.mo, &o.mo2, o.a, (int)blockIdx.x - G.cta0[i], G.cta0[i + 1] - G.cta0[i]);
+}
+
 // sum the split-K partials, folded BN + ReLU, bf16, 16-byte stores
 __global__ void conv_splitk_finalize(const float* __restrict__ ws, int ksplit, size_t ws_split, int ws_ld, int PQ,
                                      int K, const float* __restrict__ scale, const float* __restrict__ shift,
@@ -1037,6 +1057,27 @@ size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
   return 1024 + A + B + (size_t)a.out_bufs * 128 * (size_t)stage_pitch(a.n_tile) +
          (2 * a.stages + 2 * kMaxABufs + 6) * 8 +
          2 * kScaleRes * 4;
+}
+
+void launch_conv_tc_group(const ConvTcGroup& G, size_t smem, cudaStream_t st) {
+  static bool attr_set[64] = {false};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 64 && !attr_set[dev]) {
+    cudaFuncSetAttribute(conv_tc_group_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    attr_set[dev] = true;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(G.cta0[G.n]);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaLaunchKernelEx(&cfg, conv_tc_group_kernel, G);
 }
 
 void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const CUtensorMap& mo, const CUtensorMap& mo2,

@@ -50,6 +50,12 @@ static bool s2d_conv(const Op& o) {
 // plan_conv_tc context: the op runs alone (singleton stage / t(v) profiling)
 // or next to other ops of its stage
 static thread_local bool g_conv_solo = false;
+// SM count of the device whose closures are being built (plan_conv_tc)
+static thread_local int g_num_sms = 148;
+// build_op of a plain tcgen05 conv records its launch descriptor here (the
+// group-context build only), so a stage's convs can share one launch
+static thread_local std::vector<ConvTcOp>* g_tc_out = nullptr;
+static thread_local size_t* g_tc_smem = nullptr;
 
 void ck(cudaError_t e, const char* what) {
   if (e != cudaSuccess) fail(HIOS_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
@@ -60,6 +66,7 @@ static inline int64_t rup64(int64_t x, int64_t m) { return (x + m - 1) / m * m; 
 
 Executor::Executor(Schedule& sch) : s(sch), g(*sch.g), M(sch.M) {
   esz = g.dtype == HIOS_BF16 ? 2 : 4;
+  group_convs = getenv("HIOS_NOGROUP") == nullptr;  // A/B switch: per-op streams for every stage
   transport = sch.transport;
   int ndev = 0;
   ck(cudaGetDeviceCount(&ndev), "cudaGetDeviceCount");
@@ -100,6 +107,7 @@ Executor::~Executor() {
     if (x.ev_ready) cudaEventDestroy(x.ev_ready);
     if (x.ev_recv) cudaEventDestroy(x.ev_recv);
   }
+  for (auto& kv : edge_ev) cudaEventDestroy(kv.second);
   for (auto& L : lg)
     if (L.comm) cudaStreamDestroy(L.comm);
   nccl_comm_destroy(comm);
@@ -374,13 +382,30 @@ void Executor::allocate() {
     for (auto& e : L.ev_join) ck(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
     ck(cudaEventCreate(&L.ev_start), "event");
     ck(cudaEventCreate(&L.ev_done), "event");
+    ck(cudaDeviceGetAttribute(&L.num_sms, cudaDevAttrMultiProcessorCount, L.dev), "SM count");
   }
+  // one CUDA graph per device (its local logical GPUs), owner = the first
+  graphs_by_dev.clear();
+  graph_of.assign(M, -1);
+  for (int l = 0; l < M; ++l)
+    if (lg[l].local) graphs_by_dev[lg[l].dev].push_back(l);
+  for (auto& kv : graphs_by_dev)
+    for (int l : kv.second) graph_of[l] = kv.second[0];
+  for (int u = 0; u < g.n; ++u)
+    for (auto& r : ox[u].remote)
+      if (same_graph(s.gpu_of[u], r.gpu)) {
+        ck(cudaSetDevice(lg[r.gpu].dev), "cudaSetDevice");
+        cudaEvent_t e;
+        ck(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
+        edge_ev[(int64_t)u * M + r.gpu] = e;
+      }
   for (auto& x : xfers) {
     for (int side = 0; side < 2; ++side) {
       const int l = side ? x.dst : x.src;
       if (!lg[l].local) continue;
       ck(cudaSetDevice(lg[l].dev), "cudaSetDevice");
-      if (!lg[l].comm) ck(cudaStreamCreateWithFlags(&lg[l].comm, cudaStreamNonBlocking), "comm stream");
+      LGpu& Lo = lg[graph_of[l]];
+      if (!Lo.comm) ck(cudaStreamCreateWithFlags(&Lo.comm, cudaStreamNonBlocking), "comm stream");
       cudaEvent_t& e = side ? x.ev_recv : x.ev_ready;
       ck(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
     }
@@ -456,7 +481,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     const double tma = std::max((c.halo ? 1.0 : 2.0) * 500.0 / 4.0, (a_bytes + nt * 128.0) / 64.0);
     const double epi = nt / 16.0 * 80.0 + 128.0 * nt * 2.0 / 64.0;
     const double tile = std::max(KI * std::max(mma, tma), epi) + 300.0;
-    const double waves = std::ceil((double)c.tiles_m * tn / 148.0);
+    const double waves = std::ceil((double)c.tiles_m * tn / (double)g_num_sms);
     const double cost = waves * tile + 1500.0;
     if (cost < best_cost * 0.98) { best_cost = cost; c.n_tile = nt; }
   }
@@ -476,7 +501,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     // alone on the GPU (singleton stage) a 64-wide tile doubles the CTAs
     // (measured: sequential Inception-1024 1.077 -> 0.981 ms with 64 for all)
     // (only when 128-wide tiles leave SMs idle)
-    int cap = (g_conv_solo && (int64_t)c.tiles_m * ((K + 127) / 128) < 148) ? 64 : 128;
+    int cap = (g_conv_solo && (int64_t)c.tiles_m * ((K + 127) / 128) < g_num_sms) ? 64 : 128;
     if (getenv("HIOS_TAPCAP")) cap = std::max(16, atoi(getenv("HIOS_TAPCAP")));
     const int nb = (K + cap - 1) / cap;
     c.n_tile = rup((K + nb - 1) / nb, 16);
@@ -515,7 +540,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   // Conv2d_2a re-read 36 KB of weights per 25 KB input tile)
   const size_t b_all = (size_t)c.c_chunks * R * S * B;
   c.bres = 0;
-  if (c.halo && c.tiles_n == 1 && c.tiles_m > 148 * c.occ && b_all <= 96 * 1024 && !getenv("HIOS_NOBRES") &&
+  if (c.halo && c.tiles_n == 1 && c.tiles_m > g_num_sms * c.occ && b_all <= 96 * 1024 && !getenv("HIOS_NOBRES") &&
       halo_bytes_of(c.hrows, hw) + b_all <= budget) {
     c.bres = 1;
     c.kps = std::min(4, R * S);
@@ -558,7 +583,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   if (!c.halo && getenv("HIOS_SPLITK") && tiles < 48 && KI >= 16) {
     // at most one wave of CTAs, >= ~6 K-steps each; splits may start at any
     // (chunk, tap) K-step
-    static const int cta_cap = getenv("HIOS_SPLIT_CTAS") ? atoi(getenv("HIOS_SPLIT_CTAS")) : 148;
+    const int cta_cap = g_num_sms;
     static const int min_k = getenv("HIOS_SPLIT_MINK") ? std::max(1, atoi(getenv("HIOS_SPLIT_MINK"))) : 6;
     int want = std::max(1, (cta_cap * c.occ) / tiles);
     want = std::min(want, KI / min_k);
@@ -654,7 +679,7 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
     if (!a.tma_out) a.epi = 0;
   }
   const size_t smem = conv_tc_smem_bytes(a);
-  const int grid = std::min(a.tiles_m * a.tiles_n * a.ksplit, 148 * a.occ);
+  const int grid = std::min(a.tiles_m * a.tiles_n * a.ksplit, g_num_sms * a.occ);
   if (a.ksplit > 1) {
     a.ws_ld = a.tiles_n * a.n_tile;
     a.ws_split = (size_t)P * Q * a.ws_ld;
@@ -669,6 +694,12 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
     };
   }
   nk += 1;
+  if (g_tc_out) {
+    ConvTcOp op;
+    op.mx = mx; op.mw = mw; op.mo = mo; op.mo2 = mo2; op.a = a;
+    g_tc_out->push_back(op);
+    *g_tc_smem = std::max(*g_tc_smem, smem);
+  }
   return [mx, mw, mo, mo2, a, smem, grid](cudaStream_t st) { launch_conv_tc(mx, mw, mo, mo2, a, grid, smem, st); };
 }
 
@@ -771,8 +802,16 @@ static void build_op(Executor& ex, int v) {
         ++nk;
         break;
       }
+      if (!g_conv_solo && ex.g.dtype == HIOS_BF16) {
+        x.tc.clear();
+        x.tc_smem = 0;
+        g_tc_out = &x.tc;
+        g_tc_smem = &x.tc_smem;
+      }
       fns.push_back(conv_closure<T>(ex, view_of(u, l), xi.H, xi.W, xi.C, x.w, x.scale[0], x.shift[0], o.out_c, o.kh,
                                     o.kw, o.sh, o.sw, o.ph, o.pw, o.dh, o.dw, o.H, o.W, o.relu, out, out2, nk));
+      g_tc_out = nullptr;
+      g_tc_smem = nullptr;
       break;
     }
     case HIOS_OP_SEPCONV: {
@@ -896,6 +935,7 @@ void Executor::build_closures() {
     if (!lg[l].local) continue;
     ck(cudaSetDevice(lg[l].dev), "cudaSetDevice");
     cur_lgpu = l;
+    g_num_sms = lg[l].num_sms;
     if (g.dtype == HIOS_BF16) build_op<bf16>(*this, v);
     else build_op<float>(*this, v);
     OpExec& x = ox[v];
@@ -964,74 +1004,220 @@ static int enqueue_deliver(Executor& ex, int u, cudaStream_t st) {
       }
       ++nk;
     }
-    launch_signal(ex.lg[l].sync, ex.lg[d].sync + 1 + ex.M + ex.flag_index[u][d], st);
-    ++nk;
+    if (ex.same_graph(l, d)) {
+      // consumer in the same CUDA graph (a logical GPU aliased on this
+      // device): a graph dependency, no device-side flag
+      ck(cudaEventRecord(ex.edge_event(u, d), st), "record edge");
+    } else {
+      launch_signal(ex.lg[l].sync, ex.lg[d].sync + 1 + ex.M + ex.flag_index[u][d], st);
+      ++nk;
+    }
   }
   return nk;
 }
 
-void Executor::enqueue_stage_program(int l, bool timed) {
+// SM partition of a stage's grouped convs: op i gets n_i CTAs (one per SM),
+// n_i = its tile count when all fit in `budget`, else proportional to its
+// measured solo time t(v) (equal finish times if the op scales with SMs),
+// capped by its tiles; leftovers go to the op with the largest t(v) / n_i.
+static std::vector<int> partition_ctas(const std::vector<int>& tiles, const std::vector<double>& work, int budget) {
+  const int n = (int)tiles.size();
+  std::vector<int> c(n, 1);
+  int64_t tot = 0;
+  for (int t : tiles) tot += t;
+  if (tot <= budget) return tiles;
+  double wsum = 0;
+  for (double w : work) wsum += w;
+  int used = 0;
+  for (int i = 0; i < n; ++i) {
+    c[i] = std::max(1, std::min(tiles[i], (int)std::floor(budget * work[i] / std::max(wsum, 1e-30))));
+    used += c[i];
+  }
+  while (used > budget) {  // rounding up to 1 CTA can overshoot
+    int j = -1;
+    for (int i = 0; i < n; ++i)
+      if (c[i] > 1 && (j < 0 || work[i] / c[i] < work[j] / c[j])) j = i;
+    if (j < 0) break;
+    --c[j];
+    --used;
+  }
+  while (used < budget) {
+    int j = -1;
+    for (int i = 0; i < n; ++i)
+      if (c[i] < tiles[i] && (j < 0 || work[i] / c[i] > work[j] / c[j])) j = i;
+    if (j < 0) break;
+    ++c[j];
+    ++used;
+  }
+  return c;
+}
+
+void Executor::enqueue_stage(int l, const std::vector<int>& S, bool timed, int64_t& nk,
+                             const std::function<void(int, cudaStream_t)>& post) {
   LGpu& L = lg[l];
   cudaStream_t s0 = L.streams[0];
+  auto run_one = [&](int v, cudaStream_t st) {
+    if (timed) ck(cudaEventRecordWithFlags(op_ev0[v], st, cudaEventRecordExternal), "event record");
+    const bool solo = S.size() == 1 && ox[v].run_solo;
+    (solo ? ox[v].run_solo : ox[v].run)(st);
+    if (timed) ck(cudaEventRecordWithFlags(op_ev1[v], st, cudaEventRecordExternal), "event record");
+    nk += solo ? ox[v].n_kernels_solo : ox[v].n_kernels;
+    post(v, st);
+  };
+  if (S.size() == 1) {
+    run_one(S[0], s0);
+    return;
+  }
+  std::vector<int> grp, rest;
+  for (int v : S) (group_convs && ox[v].tc.size() == 1 ? grp : rest).push_back(v);
+  if (grp.size() < 2 || (int)grp.size() > kMaxGroup) {
+    grp.clear();
+    rest = S;
+  }
+  const int n_streams_used = (int)rest.size() + (grp.empty() ? 0 : 1);
+  if (n_streams_used > 1) {
+    ck(cudaEventRecord(L.ev_fork, s0), "fork");
+    for (int k = 1; k < n_streams_used; ++k) ck(cudaStreamWaitEvent(L.streams[k], L.ev_fork, 0), "fork wait");
+  }
+  int k0 = 0;
+  if (!grp.empty()) {
+    // one launch for the stage's convs; the non-conv ops of the stage keep
+    // a share of the SMs proportional to their measured time
+    double wc = 0, wr = 0;
+    std::vector<int> tiles;
+    std::vector<double> work;
+    for (int v : grp) {
+      const ConvTcArgs& a = ox[v].tc[0].a;
+      tiles.push_back(a.tiles_m * a.tiles_n);
+      const double w = g.ops[v].cost > 0 ? (double)g.ops[v].cost : 1.0;
+      work.push_back(w);
+      wc += w;
+    }
+    for (int v : rest) wr += g.ops[v].cost > 0 ? (double)g.ops[v].cost : 1.0;
+    int budget = L.num_sms;
+    if (!rest.empty())
+      budget = std::max((int)grp.size(), std::min(L.num_sms - 16, (int)std::lround(L.num_sms * wc / (wc + wr))));
+    const std::vector<int> c = partition_ctas(tiles, work, budget);
+    ConvTcGroup G;
+    std::memset(&G, 0, sizeof(G));
+    G.n = (int)grp.size();
+    size_t smem = 0;
+    for (int i = 0; i < G.n; ++i) {
+      G.op[i] = ox[grp[i]].tc[0];
+      G.cta0[i + 1] = G.cta0[i] + c[i];
+      smem = std::max(smem, ox[grp[i]].tc_smem);
+    }
+    if (timed)
+      for (int v : grp) ck(cudaEventRecordWithFlags(op_ev0[v], s0, cudaEventRecordExternal), "event record");
+    launch_conv_tc_group(G, smem, s0);
+    ++nk;
+    if (timed)
+      for (int v : grp) ck(cudaEventRecordWithFlags(op_ev1[v], s0, cudaEventRecordExternal), "event record");
+    for (int v : grp) post(v, s0);
+    k0 = 1;
+  }
+  for (size_t i = 0; i < rest.size(); ++i) run_one(rest[i], L.streams[k0 + i]);
+  for (int k = 1; k < n_streams_used; ++k) {
+    ck(cudaEventRecord(L.ev_join[k], L.streams[k]), "join");
+    ck(cudaStreamWaitEvent(s0, L.ev_join[k], 0), "join wait");
+  }
+}
+
+// The stage programs of the local logical GPUs that share one device, captured
+// into ONE CUDA graph.  Several logical GPUs alias one device when a schedule
+// has more GPUs than the box; edges between them become graph dependencies
+// (event record -> stream wait inside the capture), not device-side flag
+// spins (a spinning wait kernel could block the hardware queue its signaller
+// sits behind).  Edges to other devices / processes keep the epoch flags
+// (peer / copy transports) or the NCCL send / receive pairs.  The stages of
+// all logical GPUs of the graph are captured in one topological order of the
+// stage DAG (the same order the NCCL transport posts its transfers in).
+void Executor::capture_device(const std::vector<int>& ls, bool timed) {
+  const std::set<int> lset(ls.begin(), ls.end());
+  const int l0 = ls[0];
+  LGpu& L0 = lg[l0];
+  cudaStream_t origin = L0.streams[0];
   int64_t nk = 0;
-  launch_epoch(L.sync, s0);
-  ++nk;
-  // back-pressure: do not overwrite a consumer GPU's buffers before it finished
-  // the previous run (flag transports; NCCL receives land in the consumer's
-  // own stream order)
-  std::set<int> consumers, producers;
-  for (int v = 0; v < g.n; ++v) {
-    if (s.gpu_of[v] == l) {
-      for (auto& r : ox[v].remote)
-        if (r.mode != DM_NCCL) consumers.insert(r.gpu);
-    } else if (flag_index[v][l] >= 0) {
-      producers.insert(s.gpu_of[v]);
+  ck(cudaStreamBeginCapture(origin, cudaStreamCaptureModeRelaxed), "begin capture");
+  if (ls.size() > 1) {
+    ck(cudaEventRecord(L0.ev_fork, origin), "fork lgpus");
+    for (size_t i = 1; i < ls.size(); ++i) ck(cudaStreamWaitEvent(lg[ls[i]].streams[0], L0.ev_fork, 0), "fork");
+  }
+  std::set<std::pair<int, int>> acks_out;  // (this lgpu, producer lgpu in another graph)
+  for (int l : ls) {
+    LGpu& L = lg[l];
+    cudaStream_t s0 = L.streams[0];
+    launch_epoch(L.sync, s0);
+    ++nk;
+    // back-pressure: do not overwrite a consumer GPU's buffers (in another
+    // graph) before it finished the previous run
+    std::set<int> consumers;
+    for (int v = 0; v < g.n; ++v) {
+      if (s.gpu_of[v] == l) {
+        for (auto& r : ox[v].remote)
+          if (r.mode != DM_NCCL && !lset.count(r.gpu)) consumers.insert(r.gpu);
+      } else if (flag_index[v][l] >= 0 && !lset.count(s.gpu_of[v])) {
+        acks_out.insert({l, s.gpu_of[v]});
+      }
+    }
+    for (int c : consumers) {
+      launch_wait(L.sync, L.sync + 1 + c, 1, s0);
+      ++nk;
     }
   }
-  for (int c : consumers) {
-    launch_wait(L.sync, L.sync + 1 + c, 1, s0);
-    ++nk;
-  }
-  // NCCL: this GPU's sends / receives in the global transfer order on its
-  // communication stream (forked from and joined back into s0)
+  // NCCL: this device's sends / receives in the global transfer order on one
+  // communication stream (forked from and joined back into the origin)
   std::vector<int> acts;
   for (int k = 0; k < (int)xfers.size(); ++k)
-    if (xfers[k].src == l || xfers[k].dst == l) acts.push_back(k);
+    if (lset.count(xfers[k].src) || lset.count(xfers[k].dst)) acts.push_back(k);
   size_t next = 0;
   std::vector<char> ready(xfers.size(), 0);
+  cudaStream_t cs = L0.comm;
   if (!acts.empty()) {
-    ck(cudaEventRecord(L.ev_fork, s0), "fork comm");
-    ck(cudaStreamWaitEvent(L.comm, L.ev_fork, 0), "fork comm wait");
+    ck(cudaEventRecord(L0.ev_fork, origin), "fork comm");
+    ck(cudaStreamWaitEvent(cs, L0.ev_fork, 0), "fork comm wait");
   }
   auto post = [&](size_t upto) {
     for (; next < upto; ++next) {
       NcclXfer& x = xfers[acts[next]];
       const Op& o = g.ops[x.u];
-      if (x.src == l) {
+      if (lset.count(x.src)) {
         if (!ready[acts[next]])
           fail(HIOS_E_STATE, "NCCL transfer order inconsistent with the stage order (op " + std::to_string(x.u) + ")");
-        ck(cudaStreamWaitEvent(L.comm, x.ev_ready, 0), "wait send-ready");
-        const void* p = x.send_off >= 0 ? ptr(l, x.send_off) : ptr(l, loc[x.u][l].off);
-        nccl_send(p, x.bytes, s.owner[x.dst], comm, L.comm);
+        ck(cudaStreamWaitEvent(cs, x.ev_ready, 0), "wait send-ready");
+        const void* p = x.send_off >= 0 ? ptr(x.src, x.send_off) : ptr(x.src, loc[x.u][x.src].off);
+        nccl_send(p, x.bytes, s.owner[x.dst], comm, cs);
       } else {
+        const int l = x.dst;
         void* p = x.recv_off >= 0 ? ptr(l, x.recv_off) : ptr(l, loc[x.u][l].off);
-        nccl_recv(p, x.bytes, s.owner[x.src], comm, L.comm);
+        nccl_recv(p, x.bytes, s.owner[x.src], comm, cs);
         if (x.recv_off >= 0) {  // unpack into the consumer's location (slice / pitch)
-          const Loc& d = loc[x.u][l];
+          const Loc& dl = loc[x.u][l];
           if (g.dtype == HIOS_BF16) {
-            CopyArgs<bf16> c{(const bf16*)p, o.C, o.H * o.W, o.C, (bf16*)ptr(l, d.off), d.ldc};
-            launch_copy<bf16>(c, L.comm);
+            CopyArgs<bf16> c{(const bf16*)p, o.C, o.H * o.W, o.C, (bf16*)ptr(l, dl.off), dl.ldc};
+            launch_copy<bf16>(c, cs);
           } else {
-            CopyArgs<float> c{(const float*)p, o.C, o.H * o.W, o.C, (float*)ptr(l, d.off), d.ldc};
-            launch_copy<float>(c, L.comm);
+            CopyArgs<float> c{(const float*)p, o.C, o.H * o.W, o.C, (float*)ptr(l, dl.off), dl.ldc};
+            launch_copy<float>(c, cs);
           }
           ++nk;
         }
-        ck(cudaEventRecord(x.ev_recv, L.comm), "record recv");
+        ck(cudaEventRecord(x.ev_recv, cs), "record recv");
       }
     }
   };
-  for (auto& S : s.Q[l]) {
+  // every stage of the graph's logical GPUs in one topological order
+  const std::vector<std::vector<int>> rank = stage_ranks(s);
+  std::vector<std::tuple<int, int, int>> order;
+  for (int l : ls)
+    for (int j = 0; j < (int)s.Q[l].size(); ++j) order.emplace_back(rank[l][j], l, j);
+  std::sort(order.begin(), order.end());
+  cur_graph = lset;
+  for (auto& it : order) {
+    const int l = std::get<1>(it), j = std::get<2>(it);
+    LGpu& L = lg[l];
+    cudaStream_t s0 = L.streams[0];
+    const auto& S = s.Q[l][j];
     std::set<int> waits;
     for (int v : S)
       for (int e : g.ops[v].in_edges) {
@@ -1039,7 +1225,10 @@ void Executor::enqueue_stage_program(int l, bool timed) {
         if (s.gpu_of[u] != l) waits.insert(u);
       }
     for (int u : waits) {
-      if (flag_index[u][l] < 0) {  // NCCL: post up to this receive, then wait for it
+      const int p = s.gpu_of[u];
+      if (lset.count(p)) {
+        ck(cudaStreamWaitEvent(s0, edge_event(u, l), 0), "wait edge");
+      } else if (flag_index[u][l] < 0) {  // NCCL: post up to this receive, then wait for it
         for (size_t i = 0; i < acts.size(); ++i) {
           const NcclXfer& x = xfers[acts[i]];
           if (x.u == u && x.dst == l) {
@@ -1047,43 +1236,45 @@ void Executor::enqueue_stage_program(int l, bool timed) {
             ck(cudaStreamWaitEvent(s0, x.ev_recv, 0), "wait recv");
           }
         }
-        continue;
+      } else {
+        launch_wait(L.sync, L.sync + 1 + M + flag_index[u][l], 0, s0);
+        ++nk;
       }
-      launch_wait(L.sync, L.sync + 1 + M + flag_index[u][l], 0, s0);
-      ++nk;
     }
-    auto run_one = [&](int v, cudaStream_t st) {
-      if (timed) ck(cudaEventRecordWithFlags(op_ev0[v], st, cudaEventRecordExternal), "event record");
-      const bool solo = S.size() == 1 && ox[v].run_solo;
-      (solo ? ox[v].run_solo : ox[v].run)(st);
-      if (timed) ck(cudaEventRecordWithFlags(op_ev1[v], st, cudaEventRecordExternal), "event record");
-      nk += solo ? ox[v].n_kernels_solo : ox[v].n_kernels;
+    enqueue_stage(l, S, timed, nk, [&](int v, cudaStream_t st) {
       nk += enqueue_deliver(*this, v, st);
       for (int k : acts)
-        if (xfers[k].u == v && xfers[k].src == l) ready[k] = 1;
-    };
-    if (S.size() == 1) {
-      run_one(S[0], s0);
-    } else {
-      ck(cudaEventRecord(L.ev_fork, s0), "fork");
-      for (size_t k = 1; k < S.size(); ++k) ck(cudaStreamWaitEvent(L.streams[k], L.ev_fork, 0), "fork wait");
-      for (size_t k = 0; k < S.size(); ++k) run_one(S[k], L.streams[k]);
-      for (size_t k = 1; k < S.size(); ++k) {
-        ck(cudaEventRecord(L.ev_join[k], L.streams[k]), "join");
-        ck(cudaStreamWaitEvent(s0, L.ev_join[k], 0), "join wait");
-      }
-    }
+        if (xfers[k].u == v && lset.count(xfers[k].src)) ready[k] = 1;
+    });
   }
+  cur_graph.clear();
   if (!acts.empty()) {
     post(acts.size());
-    ck(cudaEventRecord(L.ev_join[0], L.comm), "join comm");
-    ck(cudaStreamWaitEvent(s0, L.ev_join[0], 0), "join comm wait");
+    ck(cudaEventRecord(L0.ev_join[0], cs), "join comm");
+    ck(cudaStreamWaitEvent(origin, L0.ev_join[0], 0), "join comm wait");
   }
-  for (int p : producers) {
-    launch_signal(L.sync, lg[p].sync + 1 + l, s0);
+  for (auto& pr : acks_out) {
+    launch_signal(lg[pr.first].sync, lg[pr.second].sync + 1 + pr.first, lg[pr.first].streams[0]);
     ++nk;
   }
+  for (size_t i = 1; i < ls.size(); ++i) {
+    LGpu& L = lg[ls[i]];
+    ck(cudaEventRecord(L.ev_join[0], L.streams[0]), "join lgpu");
+    ck(cudaStreamWaitEvent(origin, L.ev_join[0], 0), "join lgpu wait");
+  }
+  cudaGraph_t graph;
+  ck(cudaStreamEndCapture(origin, &graph), "end capture");
+  cudaGraphExec_t ge;
+  ck(cudaGraphInstantiate(&ge, graph, 0), "graph instantiate");
+  cudaGraphDestroy(graph);
+  (timed ? L0.gexec_timed : L0.gexec) = ge;
   if (!timed) kernels_per_run += nk;
+}
+
+cudaEvent_t Executor::edge_event(int u, int d) {
+  auto it = edge_ev.find((int64_t)u * M + d);
+  if (it == edge_ev.end()) fail(HIOS_E_STATE, "no edge event");
+  return it->second;
 }
 
 void Executor::capture() {
@@ -1101,16 +1292,10 @@ void Executor::capture() {
         ck(cudaEventCreate(&op_ev0[v]), "event");
         ck(cudaEventCreate(&op_ev1[v]), "event");
       }
-    for (int timed = 0; timed < 2; ++timed) {
-      cudaGraph_t graph;
-      ck(cudaStreamBeginCapture(L.streams[0], cudaStreamCaptureModeRelaxed), "begin capture");
-      enqueue_stage_program(l, timed != 0);
-      ck(cudaStreamEndCapture(L.streams[0], &graph), "end capture");
-      cudaGraphExec_t ge;
-      ck(cudaGraphInstantiate(&ge, graph, 0), "graph instantiate");
-      cudaGraphDestroy(graph);
-      (timed ? L.gexec_timed : L.gexec) = ge;
-    }
+  }
+  for (auto& kv : graphs_by_dev) {
+    ck(cudaSetDevice(kv.first), "cudaSetDevice");
+    for (int timed = 0; timed < 2; ++timed) capture_device(kv.second, timed != 0);
   }
   captured = true;
 }
@@ -1131,46 +1316,44 @@ void Executor::run_device(const void* d_in, void* d_out, cudaStream_t user, bool
     ck(cudaEventCreateWithFlags(&ev_user, cudaEventDisableTiming), "event");
     ck(cudaEventRecord(ev_user, user), "record user");
   }
-  const int li = s.gpu_of[g.input_op], ls = s.gpu_of[g.sink_op];
-  for (int l = 0; l < M; ++l) {
-    LGpu& L = lg[l];
-    if (!L.local) continue;
+  const int li = s.gpu_of[g.input_op], lsk = s.gpu_of[g.sink_op];
+  for (auto& kv : graphs_by_dev) {
+    const int o = kv.second[0];
+    LGpu& L = lg[o];
     ck(cudaSetDevice(L.dev), "cudaSetDevice");
     if (ev_user) ck(cudaStreamWaitEvent(L.streams[0], ev_user, 0), "wait user");
     ck(cudaEventRecord(L.ev_start, L.streams[0]), "record start");
-    if (l == li && d_in) {
-      const Loc& lc = loc[g.input_op][l];
+    if (graph_of[li] == o && d_in) {
+      const Loc& lc = loc[g.input_op][li];
       if (g.dtype == HIOS_BF16)
-        launch_input<bf16>((const float*)d_in, g.in_c, g.in_h, g.in_w, (bf16*)ptr(l, lc.off), lc.ldc, L.streams[0]);
+        launch_input<bf16>((const float*)d_in, g.in_c, g.in_h, g.in_w, (bf16*)ptr(li, lc.off), lc.ldc, L.streams[0]);
       else
-        launch_input<float>((const float*)d_in, g.in_c, g.in_h, g.in_w, (float*)ptr(l, lc.off), lc.ldc,
+        launch_input<float>((const float*)d_in, g.in_c, g.in_h, g.in_w, (float*)ptr(li, lc.off), lc.ldc,
                             L.streams[0]);
     }
   }
-  for (int l = 0; l < M; ++l) {
-    LGpu& L = lg[l];
-    if (!L.local) continue;
+  for (auto& kv : graphs_by_dev) {
+    LGpu& L = lg[kv.second[0]];
     ck(cudaSetDevice(L.dev), "cudaSetDevice");
     ck(cudaGraphLaunch(timed ? L.gexec_timed : L.gexec, L.streams[0]), "graph launch");
   }
-  for (int l = 0; l < M; ++l) {
-    LGpu& L = lg[l];
-    if (!L.local) continue;
+  for (auto& kv : graphs_by_dev) {
+    const int o = kv.second[0];
+    LGpu& L = lg[o];
     ck(cudaSetDevice(L.dev), "cudaSetDevice");
-    if (l == ls && d_out) {
-      const Op& o = g.ops[g.sink_op];
-      const Loc& lc = loc[g.sink_op][l];
+    if (graph_of[lsk] == o && d_out) {
+      const Op& op = g.ops[g.sink_op];
+      const Loc& lc = loc[g.sink_op][lsk];
       if (g.dtype == HIOS_BF16)
-        launch_output<bf16>((const bf16*)ptr(l, lc.off), o.C, o.H, o.W, lc.ldc, (float*)d_out, L.streams[0]);
+        launch_output<bf16>((const bf16*)ptr(lsk, lc.off), op.C, op.H, op.W, lc.ldc, (float*)d_out, L.streams[0]);
       else
-        launch_output<float>((const float*)ptr(l, lc.off), o.C, o.H, o.W, lc.ldc, (float*)d_out, L.streams[0]);
+        launch_output<float>((const float*)ptr(lsk, lc.off), op.C, op.H, op.W, lc.ldc, (float*)d_out, L.streams[0]);
     }
     ck(cudaEventRecord(L.ev_done, L.streams[0]), "record done");
   }
   ck(cudaSetDevice(cur), "cudaSetDevice");
-  for (int l = 0; l < M; ++l) {
-    LGpu& L = lg[l];
-    if (!L.local) continue;
+  for (auto& kv : graphs_by_dev) {
+    LGpu& L = lg[kv.second[0]];
     if (user) ck(cudaStreamWaitEvent(user, L.ev_done, 0), "user wait");
     else ck(cudaEventSynchronize(L.ev_done), "synchronize");
   }

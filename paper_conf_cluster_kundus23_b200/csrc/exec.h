@@ -1,6 +1,8 @@
 // exec.h -- per-GPU stage executor.
 #pragma once
 #include <functional>
+#include <map>
+#include <set>
 #include <vector>
 
 #include "internal.h"
@@ -18,6 +20,8 @@ void nccl_send(const void* buf, size_t bytes, int peer, NcclComm c, cudaStream_t
 void nccl_recv(void* buf, size_t bytes, int peer, NcclComm c, cudaStream_t st);
 // global order of the (producer op, consumer logical GPU) transfers
 std::vector<std::pair<int, int>> transfer_order(const Schedule& s);
+// position of every stage (gpu, j) in one topological order of the stage DAG
+std::vector<std::vector<int>> stage_ranks(const Schedule& s);
 
 // how one (producer, consumer GPU) edge is carried
 enum DeliverMode { DM_FUSED = 0, DM_PUSH = 1, DM_COPY = 2, DM_NCCL = 3 };
@@ -57,6 +61,10 @@ struct OpExec {
   // tap-mode convs take narrower N tiles there (more CTAs); empty = run
   std::function<void(cudaStream_t)> run_solo;
   int n_kernels_solo = 0;
+  // a plain tcgen05 conv (one launch, group-context plan): its descriptor for
+  // the stage's grouped launch (conv_tc_group_kernel); empty otherwise
+  std::vector<ConvTcOp> tc;
+  size_t tc_smem = 0;
 };
 
 struct LGpu {
@@ -74,6 +82,7 @@ struct LGpu {
   std::vector<void*> allocs;   // weights etc. (owned)
   bool ipc_mapped = false;
   cudaStream_t comm = nullptr;  // NCCL transport: send/recv stream
+  int num_sms = 148;             // cudaDevAttrMultiProcessorCount
 };
 
 // one NCCL transfer of the global order, as this process sees it
@@ -118,9 +127,26 @@ struct Executor {
   char* ptr(int lgpu, int64_t off) const { return lg[lgpu].arena + off; }
   bool is_local(int l) const { return lg[l].local; }
   void read_output(int op, float* host, int64_t n);
-  void enqueue_stage_program(int l, bool timed);
+  // CUDA graph per device: its local logical GPUs' stage programs
+  void capture_device(const std::vector<int>& ls, bool timed);
+  std::map<int, std::vector<int>> graphs_by_dev;  // device -> local lgpus (first = owner)
+  std::vector<int> graph_of;                      // lgpu -> owner lgpu of its graph (-1 remote)
+  std::map<int64_t, cudaEvent_t> edge_ev;         // (u * M + consumer lgpu) -> same-graph edge event
+  std::set<int> cur_graph;
+  bool same_graph(int a, int b) const {
+    return a >= 0 && b >= 0 && a < (int)graph_of.size() && b < (int)graph_of.size() && graph_of[a] >= 0 &&
+           graph_of[a] == graph_of[b];
+  }
+  cudaEvent_t edge_event(int u, int d);
   // each local op's kernels alone, L2 flushed, as configured in Q (hios_time_ops)
   void time_ops(int reps, int64_t flush_bytes, int64_t* op_ns);
+  // one stage S of logical GPU l: its plain tcgen05 convs as ONE grouped
+  // launch on s0 with an explicit SM partition, the other ops forked onto
+  // streams 1.. (or every op on its own stream: group == false); post(v, st)
+  // runs after op v on the stream v ran on
+  void enqueue_stage(int l, const std::vector<int>& S, bool timed, int64_t& nk,
+                     const std::function<void(int, cudaStream_t)>& post);
+  bool group_convs = true;
 };
 
 void ck(cudaError_t e, const char* what);

@@ -163,6 +163,18 @@ struct CopyArgs {
 void launch_conv_tc(const CUtensorMap& mx, const CUtensorMap& mw, const CUtensorMap& mo, const CUtensorMap& mo2,
                     const ConvTcArgs& a, int grid, size_t smem, cudaStream_t st);
 size_t conv_tc_smem_bytes(const ConvTcArgs& a);
+// the convs of one stage in one launch (SM ranges per op)
+struct ConvTcOp {
+  CUtensorMap mx, mw, mo, mo2;
+  ConvTcArgs a;
+};
+constexpr int kMaxGroup = 8;
+struct ConvTcGroup {
+  ConvTcOp op[kMaxGroup];
+  int n;
+  int cta0[kMaxGroup + 1];  // op i owns CTAs [cta0[i], cta0[i+1])
+};
+void launch_conv_tc_group(const ConvTcGroup& G, size_t smem, cudaStream_t st);
 void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st);
 __host__ __device__ inline uint32_t halo_bytes_of(int R, int halo_w) {
   return ((uint32_t)R * halo_w * 128u + 1023u) & ~1023u;

@@ -96,7 +96,7 @@ void nccl_recv(void* buf, size_t bytes, int peer, NcclComm c, cudaStream_t st) {
   nck(nccl().Recv(buf, bytes, kNcclUint8, peer, c, st), "ncclRecv");
 }
 
-std::vector<std::pair<int, int>> transfer_order(const Schedule& s) {
+std::vector<std::vector<int>> stage_ranks(const Schedule& s) {
   const Graph& g = *s.g;
   // stages as nodes: id = offset[gpu] + stage
   std::vector<int> off(s.M + 1, 0);
@@ -126,6 +126,16 @@ std::vector<std::pair<int, int>> transfer_order(const Schedule& s) {
       if (--indeg[b] == 0) q.push(b);
   }
   if (r != ns) fail(HIOS_E_CYCLE, "stage graph has a cycle");
+  std::vector<std::vector<int>> out(s.M);
+  for (int i = 0; i < s.M; ++i)
+    for (int j = 0; j < (int)s.Q[i].size(); ++j) out[i].push_back(rank[off[i] + j]);
+  return out;
+}
+
+std::vector<std::pair<int, int>> transfer_order(const Schedule& s) {
+  const Graph& g = *s.g;
+  const std::vector<std::vector<int>> rk = stage_ranks(s);
+  auto node_rank = [&](int v) { return rk[s.gpu_of[v]][s.stage_of[v]]; };
   std::vector<std::tuple<int, int, int>> t;
   for (int u = 0; u < g.n; ++u) {
     std::set<int> dst;
@@ -133,7 +143,7 @@ std::vector<std::pair<int, int>> transfer_order(const Schedule& s) {
       const int l = s.gpu_of[g.edges[e].dst];
       if (l != s.gpu_of[u]) dst.insert(l);
     }
-    for (int l : dst) t.emplace_back(rank[node(u)], u, l);
+    for (int l : dst) t.emplace_back(node_rank(u), u, l);
   }
   std::sort(t.begin(), t.end());
   std::vector<std::pair<int, int>> out;

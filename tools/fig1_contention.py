@@ -10,6 +10,13 @@ Both numbers come from the framework's own profiler through the C-ABI:
 ratio = parallel / sequential; < 1 means running the two ops concurrently on
 one GPU pays (the paper's crossover on an A40 is between 64^2 and 128^2).
 
+Fig. 2 analog: ratio of the transfer time of the conv's input to its
+compute time.  With one GPU visible the transfer cannot cross NVLink, so two
+columns are given: the profiler's t(u, v) of the input edge measured on this
+device (a device-local peer-store push + flag release/acquire), and the
+NVLink model bytes / 770 GB/s (the measured B200 peer-copy bandwidth of
+B200_PROFILING.md, not measured here).
+
 usage: python tools/fig1_contention.py [--dtypes bf16,f32] [--out path.json]
 """
 import argparse
@@ -44,17 +51,23 @@ def main():
             g, a, b = pair_graph(hw)
             G = h.hios_graph_create(g.ops, g.edges, 48, hw, hw, dt, gen.make_weights(g))
             h.hios_profile(G, [0], args.reps)
-            t, _ = h.hios_get_costs(G)
+            t, te = h.hios_get_costs(G)
             seq = int(t[a] + t[b])
+            in_bytes = 48 * hw * hw * (2 if dt == "bf16" else 4)
+            e_in = [i for i, (u, v, _) in enumerate(g.edges) if v == a][0]
             par = h.hios_group_cost(G, [a, b])
             fl = 2.0 * 48 * 48 * 25 * hw * hw
             r = {"dtype": dt, "hw": hw, "t_a_us": t[a] / 1e3, "t_b_us": t[b] / 1e3,
                  "seq_us": seq / 1e3, "par_us": par / 1e3, "ratio_par_over_seq": par / seq,
-                 "tflops_alone": fl / t[a] / 1e3}
+                 "tflops_alone": fl / t[a] / 1e3,
+                 "fig2_input_bytes": in_bytes, "fig2_t_edge_local_us": te[e_in] / 1e3,
+                 "fig2_t_nvlink_model_us": in_bytes / 770e9 * 1e6,
+                 "fig2_ratio_local": te[e_in] / t[a], "fig2_ratio_nvlink_model": in_bytes / 770e9 * 1e9 / t[a]}
             rows.append(r)
             print(f"{dt:5s} {hw:5d}^2  t(A) {r['t_a_us']:9.2f} us  t(B) {r['t_b_us']:9.2f} us  "
                   f"t(A||B) {r['par_us']:9.2f} us  ratio {r['ratio_par_over_seq']:.3f}  "
-                  f"({r['tflops_alone']:.1f} TFLOP/s alone)", flush=True)
+                  f"({r['tflops_alone']:.1f} TFLOP/s alone)  fig2 xfer/compute local {r['fig2_ratio_local']:.2f} "
+                  f"nvlink-model {r['fig2_ratio_nvlink_model']:.3f}", flush=True)
     if args.out:
         with open(args.out, "w") as f:
             json.dump({"what": "Fig. 1 analog (P:62): two 5x5 48->48 convs, parallel/sequential",
