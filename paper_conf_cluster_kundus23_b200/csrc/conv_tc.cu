@@ -47,16 +47,27 @@ __device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
 __device__ __forceinline__ void mbar_arrive(uint32_t bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
+// try_wait suspends in hardware for a bounded time per probe; a barrier that
+// never completes (a producer / consumer mismatch) traps after ~2^26 probes
+// (seconds) instead of hanging the GPU
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred p;\n"
-      "HIOS_WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      "@!p bra HIOS_WAIT_%=;\n"
-      "}\n" ::"r"(bar),
-      "r"(parity)
-      : "memory");
+  uint32_t ok = 0;
+  for (uint32_t n = 0;; ++n) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+        "selp.u32 %0, 1, 0, p;\n"
+        "}\n"
+        : "=r"(ok)
+        : "r"(bar), "r"(parity)
+        : "memory");
+    if (ok) return;
+    if (n == (1u << 26)) {
+      printf("hios conv_tc: mbarrier wait timed out (block %d thread %d)\n", (int)blockIdx.x, (int)threadIdx.x);
+      __trap();
+    }
+  }
 }
 __device__ __forceinline__ void sts128(uint32_t addr, uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3) {
   asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a0), "r"(a1), "r"(a2), "r"(a3)
@@ -558,7 +569,8 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
               else if (a.R == 1 && S_ == 1) halo_taps_bres<1, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
               else if (a.R == 2 && S_ == 1) halo_taps_bres<2, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
               else if (a.R == 4 && S_ == 1) halo_taps_bres<4, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
-              else halo_taps_bres<5, 5>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
+              else if (a.R == 5 && S_ == 5) halo_taps_bres<5, 5>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
+              else __trap();  // unreachable: fixed_rs lists exactly these shapes
               accum = 1;
               mma_commit_on(aempty0 + 8 * ab, on);
               if (++ab == (uint32_t)abufs) { ab = 0; aph ^= 1u; }
@@ -568,15 +580,18 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
               // B ring, common shapes: the chunk's taps unrolled with
               // compile-time window offsets; stage waits / releases at
               // compile-time tap boundaries (kps taps per stage)
-              if (a.R == 3 && kps == 3) halo_taps_ring<3, 3, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 3 && kps == 2) halo_taps_ring<3, 3, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 3 && kps == 4) halo_taps_ring<3, 3, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 5 && kps == 4) halo_taps_ring<5, 5, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 1 && S_ == 7) halo_taps_ring<1, 7, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 7) halo_taps_ring<7, 1, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 1 && S_ == 3) halo_taps_ring<1, 3, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 3 && S_ == 1) halo_taps_ring<3, 1, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else halo_taps_ring<1, 1, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              // (dispatch on R, S and kps together: each template's stage
+              // boundaries must match the producer's)
+              if (a.R == 3 && S_ == 3 && kps == 3) halo_taps_ring<3, 3, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 3 && S_ == 3 && kps == 2) halo_taps_ring<3, 3, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 3 && S_ == 3 && kps == 4) halo_taps_ring<3, 3, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 5 && S_ == 5 && kps == 4) halo_taps_ring<5, 5, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 1 && S_ == 7 && kps == 4) halo_taps_ring<1, 7, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 7 && S_ == 1 && kps == 4) halo_taps_ring<7, 1, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 1 && S_ == 3 && kps == 3) halo_taps_ring<1, 3, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 3 && S_ == 1 && kps == 3) halo_taps_ring<3, 1, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else if (a.R == 1 && S_ == 1 && kps == 1) halo_taps_ring<1, 1, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              else __trap();  // unreachable: fixed_ring lists exactly these shapes
               accum = 1;
               mma_commit_on(aempty0 + 8 * ab, on);
               if (++ab == (uint32_t)abufs) { ab = 0; aph ^= 1u; }

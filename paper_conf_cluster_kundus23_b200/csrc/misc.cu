@@ -4,6 +4,7 @@
 // for cross-GPU edges (a10/a11).  NHWC with a pixel stride; each thread owns
 // one pixel x VEC channels (16-byte vectors: 8 bf16 or 4 fp32) so a warp reads
 // contiguous 512-byte runs.
+#include <cstdio>
 #include <algorithm>
 #include <type_traits>
 
@@ -1123,13 +1124,27 @@ __global__ void signal_kernel(const unsigned* epoch, unsigned* flag) {
   asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(flag), "r"(e) : "memory");
 }
 
+// a wait that has not seen its flag after kWaitTimeoutNs is a broken schedule
+// or a dead peer: report it and trap (the run fails with HIOS_E_CUDA instead
+// of hanging the GPU)
+constexpr unsigned long long kWaitTimeoutNs = 20ull * 1000 * 1000 * 1000;
 __global__ void wait_kernel(const unsigned* epoch, const unsigned* flag, unsigned lag) {
   const unsigned target = *epoch - lag;
   unsigned v;
-  while (true) {
+  unsigned long long t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  for (unsigned it = 0;; ++it) {
     asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
     if ((int)(v - target) >= 0) break;
     __nanosleep(64);
+    if ((it & 1023) == 1023) {
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      if (t - t0 > kWaitTimeoutNs) {
+        printf("hios: flag wait timed out: flag %p = %u, target %u (epoch %u, lag %u)\n", (const void*)flag, v,
+               target, *epoch, lag);
+        __trap();
+      }
+    }
   }
 }
 

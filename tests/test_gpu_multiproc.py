@@ -3,6 +3,7 @@ peer buffers and cross-process epoch flags.  On a 1-GPU box both ranks share
 the device (IPC across processes on one device), which exercises exactly the
 multi-GPU code path; the output must be bit-identical to a 1-process run."""
 import os
+import signal
 import subprocess
 import sys
 
@@ -10,6 +11,20 @@ import pytest
 
 pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _run_group(cmd, timeout):
+    """torchrun in its own session; on timeout the whole process group is
+    killed (no orphaned rank left spinning on the GPU)."""
+    p = subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.PIPE, text=True, cwd=ROOT,
+                         start_new_session=True)
+    try:
+        out, err = p.communicate(timeout=timeout)
+    except subprocess.TimeoutExpired:
+        os.killpg(p.pid, signal.SIGKILL)
+        out, err = p.communicate()
+        raise AssertionError(f"timed out after {timeout} s:\n{out[-3000:]}\n{err[-3000:]}")
+    return subprocess.CompletedProcess(cmd, p.returncode, out, err)
 
 
 def _n_gpus():
@@ -29,7 +44,7 @@ def test_two_process_ipc_run(model, size, transport):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", "--master-port=29533", os.path.join(ROOT, "tools", "mp_check.py"),
            model, size, transport]
-    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
+    r = _run_group(cmd, 300)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     assert "bit-identical to 1-process run: True" in r.stdout
 
@@ -39,7 +54,7 @@ def test_bench_two_ranks_smoke():
            "--master-addr=127.0.0.1", "--master-port=29534", os.path.join(ROOT, "bench.py"),
            "--gpus", "2", "--steps", "3", "--warmup", "3", "--model", "inception_v3", "--size", "299",
            "--no-cpu-baseline"]
-    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
+    r = _run_group(cmd, 300)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     import json
     line = [l for l in r.stdout.splitlines() if l.startswith("{")][-1]

@@ -98,6 +98,7 @@ CONV_CASES = [
     (160, 192, 62, 62, 7, 1, 1, 3, 0),    # 7x1: 10-row box (Wh = 62)
     (448, 384, 30, 30, 3, 3, 1, 1, 1),    # Mixed_7 3x3, K > 128 (staged epilogue), C tail
     (384, 384, 30, 30, 1, 3, 1, 0, 1),
+    (384, 384, 30, 30, 3, 1, 1, 1, 0),    # 3x1 (kps 3: its own unrolled tap loop)
     (40, 24, 13, 90, 3, 3, 1, 1, 1),      # Wh = 92, ragged last tile, small K
     (72, 200, 11, 7, 5, 5, 1, 2, 2),      # tiny image: one tile spans the whole output
     (64, 64, 20, 31, 3, 3, 1, 0, 0),      # no padding: Wh = Q + 2

@@ -45,9 +45,12 @@ def main():
     op_gpu, _, _ = h.hios_schedule_stages(S)
     used = sorted(set(op_gpu.tolist()))
     ys = []
-    for _ in range(3):
+    import time
+    for i in range(3):
         dist.barrier()
+        t0 = time.time()
         ys.append(h.hios_run(S, x))
+        print(f"rank {rank}: run {i} {time.time() - t0:.3f} s", flush=True)
     sink_rank = own[int(op_gpu[g.n_ops - 1])]
     ok = True
     if rank == sink_rank:
