@@ -430,13 +430,16 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   ConvTcArgs c{};
   int hw = 128 + (S - 1) * dw;
   c.halo = (sw == 1 && Q >= 96 && hw <= 256 && R * dh <= 256 && halo_bytes_of(R, hw) <= 100 * 1024) ? 1 : 0;
-  // virtual-grid halo (narrow stride-1 convs with R*S > 1, see ConvTcArgs):
-  // tap mode would stream the input R*S times through L2->SM; the box of
-  // whole padded rows streams it ~(128 + (R-1) dh Wh + (S-1) dw) / 128 times
+  // virtual-grid halo (narrow stride-1 square convs, see ConvTcArgs): tap
+  // mode would stream the input R*S times through L2->SM; the box of whole
+  // padded rows streams it ~(128 + (R-1) dh Wh + (S-1) dw) / 128 times.
+  // Measured (tools/op_times.py, Inception-1024): 3x3 at 30^2 15.6 -> 13.5 us,
+  // but 7x1 at 62^2 8.8 -> 9.9 us (a 10-row box per 128 outputs) and 1x3 /
+  // 3x1 at 30^2 +1 us: square kernels only
   const int Wh = Q + (S - 1) * dw;
   const int vrows = (Wh - 1 + 127 + (S - 1) * dw) / Wh + 1 + (R - 1) * dh;
   static const bool novgrid = getenv("HIOS_NOVGRID") != nullptr;  // A/B switch
-  if (!c.halo && !novgrid && sh == 1 && sw == 1 && dh == 1 && dw == 1 && R * S > 1 && Wh <= 256 && vrows <= 256 &&
+  if (!c.halo && !novgrid && sh == 1 && sw == 1 && dh == 1 && dw == 1 && R == S && R >= 3 && Wh <= 256 && vrows <= 256 &&
       halo_bytes_of(vrows, Wh) <= 96 * 1024) {
     c.halo = 1;
     c.vgrid = Wh;
@@ -1016,38 +1019,30 @@ static int enqueue_deliver(Executor& ex, int u, cudaStream_t st) {
   return nk;
 }
 
-// SM partition of a stage's grouped convs: op i gets n_i CTAs (one per SM),
-// n_i = its tile count when all fit in `budget`, else proportional to its
-// measured solo time t(v) (equal finish times if the op scales with SMs),
-// capped by its tiles; leftovers go to the op with the largest t(v) / n_i.
-static std::vector<int> partition_ctas(const std::vector<int>& tiles, const std::vector<double>& work, int budget) {
+// SM partition of a stage's grouped convs: op i gets n_i persistent CTAs (one
+// per SM) and runs ceil(T_i / n_i) rounds of tiles, each ~tau_i (its measured
+// solo time per round of tiles).  Greedy makespan minimisation: start at one
+// CTA each, repeatedly give the op with the latest finish the smallest number
+// of extra CTAs that removes one of its rounds, while the budget lasts.  SMs
+// the convs cannot use stay free for the stage's other ops.
+static std::vector<int> partition_ctas(const std::vector<int>& tiles, const std::vector<double>& tau, int budget) {
   const int n = (int)tiles.size();
   std::vector<int> c(n, 1);
-  int64_t tot = 0;
-  for (int t : tiles) tot += t;
-  if (tot <= budget) return tiles;
-  double wsum = 0;
-  for (double w : work) wsum += w;
-  int used = 0;
-  for (int i = 0; i < n; ++i) {
-    c[i] = std::max(1, std::min(tiles[i], (int)std::floor(budget * work[i] / std::max(wsum, 1e-30))));
-    used += c[i];
-  }
-  while (used > budget) {  // rounding up to 1 CTA can overshoot
+  int used = n;
+  auto rounds = [&](int i, int k) { return (tiles[i] + k - 1) / k; };
+  while (true) {
     int j = -1;
-    for (int i = 0; i < n; ++i)
-      if (c[i] > 1 && (j < 0 || work[i] / c[i] < work[j] / c[j])) j = i;
-    if (j < 0) break;
-    --c[j];
-    --used;
-  }
-  while (used < budget) {
-    int j = -1;
-    for (int i = 0; i < n; ++i)
-      if (c[i] < tiles[i] && (j < 0 || work[i] / c[i] > work[j] / c[j])) j = i;
-    if (j < 0) break;
-    ++c[j];
-    ++used;
+    double worst = -1;
+    for (int i = 0; i < n; ++i) {
+      const double f = rounds(i, c[i]) * tau[i];
+      if (f > worst) { worst = f; j = i; }
+    }
+    const int r = rounds(j, c[j]);
+    if (r <= 1) break;  // the latest op already runs in one round
+    const int need = (tiles[j] + r - 2) / (r - 1);  // fewest CTAs giving r - 1 rounds
+    if (used + need - c[j] > budget) break;
+    used += need - c[j];
+    c[j] = need;
   }
   return c;
 }
@@ -1085,19 +1080,20 @@ void Executor::enqueue_stage(int l, const std::vector<int>& S, bool timed, int64
     // a share of the SMs proportional to their measured time
     double wc = 0, wr = 0;
     std::vector<int> tiles;
-    std::vector<double> work;
+    std::vector<double> tau;
     for (int v : grp) {
       const ConvTcArgs& a = ox[v].tc[0].a;
-      tiles.push_back(a.tiles_m * a.tiles_n);
+      const int T = a.tiles_m * a.tiles_n;
+      tiles.push_back(T);
       const double w = g.ops[v].cost > 0 ? (double)g.ops[v].cost : 1.0;
-      work.push_back(w);
+      tau.push_back(w / ((T + L.num_sms - 1) / L.num_sms));  // per round of tiles
       wc += w;
     }
     for (int v : rest) wr += g.ops[v].cost > 0 ? (double)g.ops[v].cost : 1.0;
     int budget = L.num_sms;
     if (!rest.empty())
       budget = std::max((int)grp.size(), std::min(L.num_sms - 16, (int)std::lround(L.num_sms * wc / (wc + wr))));
-    const std::vector<int> c = partition_ctas(tiles, work, budget);
+    const std::vector<int> c = partition_ctas(tiles, tau, budget);
     ConvTcGroup G;
     std::memset(&G, 0, sizeof(G));
     G.n = (int)grp.size();

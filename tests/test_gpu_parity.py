@@ -108,7 +108,7 @@ CONV_CASES = [
 ]
 
 SPLITK_CASES = [
-    (448, 384, 10, 10, 3, 3, 1, 1, 1),    # split boundaries inside a chunk's taps
+    (448, 384, 19, 19, 3, 3, 2, 1, 1),    # split boundaries inside a chunk's taps (stride 2: tap mode)
     (2048, 384, 8, 8, 1, 1, 1, 0, 0),
     (288, 384, 35, 35, 3, 3, 2, 0, 0),
 ]
