@@ -19,8 +19,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
          "--expt-relaxed-constexpr", "-I", os.path.join(HERE, "..", "include")]
-SOURCES = ["graph.cpp", "sched.cpp", "conv_tc.cu", "conv_simt.cu", "misc.cu", "exec.cu",
-           "profile.cu", "nccl.cpp", "api.cu"]
+# every translation unit of the source tree (an A/B variant may have other files)
+SOURCES = sorted(f for f in os.listdir(CSRC) if f.endswith((".cu", ".cpp")))
 
 
 def _compile(src: str) -> str:

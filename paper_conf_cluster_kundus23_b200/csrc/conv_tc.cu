@@ -48,26 +48,26 @@ __device__ __forceinline__ void mbar_arrive(uint32_t bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
 // try_wait suspends in hardware for a bounded time per probe; a barrier that
-// never completes (a producer / consumer mismatch) traps after ~2^26 probes
-// (seconds) instead of hanging the GPU
+// never completes (a producer / consumer mismatch) traps after 2^26 failed
+// probes (seconds) instead of hanging the GPU (the run then fails with a CUDA
+// error).  Kept as one tight asm loop: the wait sits in the MMA issue path.
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
-  uint32_t ok = 0;
-  for (uint32_t n = 0;; ++n) {
-    asm volatile(
-        "{\n"
-        ".reg .pred p;\n"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
-        "selp.u32 %0, 1, 0, p;\n"
-        "}\n"
-        : "=r"(ok)
-        : "r"(bar), "r"(parity)
-        : "memory");
-    if (ok) return;
-    if (n == (1u << 26)) {
-      printf("hios conv_tc: mbarrier wait timed out (block %d thread %d)\n", (int)blockIdx.x, (int)threadIdx.x);
-      __trap();
-    }
-  }
+  asm volatile(
+      "{\n"
+      ".reg .pred p, q;\n"
+      ".reg .u32 n;\n"
+      "mov.u32 n, 0;\n"
+      "HIOS_WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@p bra HIOS_DONE_%=;\n"
+      "add.u32 n, n, 1;\n"
+      "setp.lt.u32 q, n, 67108864;\n"
+      "@q bra HIOS_WAIT_%=;\n"
+      "trap;\n"
+      "HIOS_DONE_%=:\n"
+      "}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
 }
 __device__ __forceinline__ void sts128(uint32_t addr, uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3) {
   asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a0), "r"(a1), "r"(a2), "r"(a3)
