@@ -47,7 +47,22 @@ def peaks():
     except Exception:
         pass
     p["nvlink_gbs"] = 770.0  # measured peer copy per direction (B200_PROFILING.md)
+    # FP32 CUDA-core peak (the fp32 path's roofline): measured by tools/fp32_peak.cu
+    # on this pool's B200 (profiles/fp32_peak.json), else 148 SMs x 128 lanes x 2 x 1.965 GHz
+    p["fp32_tflops"], p["fp32_src"] = 74.45, "nominal (148 x 128 FFMA lanes x 2 x 1.965 GHz)"
+    try:
+        with open(os.path.join(ROOT, "profiles", "fp32_peak.json")) as f:
+            p["fp32_tflops"] = float(json.load(f)["fp32_tflops"])
+            p["fp32_src"] = "measured (tools/fp32_peak.cu, profiles/fp32_peak.json)"
+    except Exception:
+        pass
     return p
+
+
+def compute_peak(pk, dtype):
+    """Dense-contraction peak for the path's arithmetic (TFLOP/s): tcgen05 bf16
+    burst for bf16, the FP32 CUDA-core peak for fp32."""
+    return pk["bf16_tflops"] if dtype == "bf16" else pk["fp32_tflops"]
 
 
 # the paper's own relative results (PAPER.md §VI-D/E), quoted with its hardware;
@@ -106,12 +121,12 @@ def op_work(g, shapes, esz):
     return F, B
 
 
-def critical_path_bound(g, F, B, op_gpu, op_stage, n_gpus, pk, esz, shapes):
+def critical_path_bound(g, F, B, op_gpu, op_stage, n_gpus, pk, esz, shapes, dtype="bf16"):
     """Schedule critical-path lower bound: stage roof =
     max(max_v roof(v), sum F / Pi, sum B / beta); stages on a GPU serialise;
     cross-GPU edges cost bytes / NVLink (overlap form: an edge may start when
     its producer starts, so it adds max(0, t_edge - roof(u))).  Returns s."""
-    Pi = pk["bf16_tflops"] * 1e12
+    Pi = compute_peak(pk, dtype) * 1e12
     beta = pk["hbm_gbs"] * 1e9
     nvl = pk["nvlink_gbs"] * 1e9
     roof = np.maximum(F / Pi, B / beta)
@@ -346,7 +361,7 @@ def max_over_ranks(dist, x, world):
 
 
 # ------------------------------------------------------------ workload sweep
-def measure_workload(h, torch, model, sz, M, args, dev, stream, flush, pk, esz):
+def measure_workload(h, torch, model, sz, M, args, dev, stream, flush, pk, dtype):
     """One more BASELINE.json workload (another size or another benchmark DAG)
     in the same run: profile, then HIOS-LP (M, w), sequential (1, 1) and the
     IOS-style stand-in (1, w), each timed like the main line (device events,
@@ -355,18 +370,28 @@ def measure_workload(h, torch, model, sz, M, args, dev, stream, flush, pk, esz):
     gs = graphs.build(model, sz)
     Ws = gen.make_weights(gs)
     xs = gen.make_input(gs)
-    Gs = h.hios_graph_create(gs.ops, gs.edges, gs.in_c, gs.in_h, gs.in_w, args.dtype, Ws)
+    esz = 2 if dtype == "bf16" else 4
+    Gs = h.hios_graph_create(gs.ops, gs.edges, gs.in_c, gs.in_h, gs.in_w, dtype, Ws)
     shp = {o.id: h.hios_graph_shape(Gs, o.id) for o in gs.ops}
     t0 = time.perf_counter()
     h.hios_profile(Gs, [dev], 5)
-    row = {"input": f"1x{gs.in_c}x{sz}x{sz}", "ops": gs.n_ops, "deps": gs.n_edges,
+    row = {"input": f"1x{gs.in_c}x{sz}x{sz}", "dtype": dtype, "ops": gs.n_ops, "deps": gs.n_edges,
            "profile_s": time.perf_counter() - t0}
     din = torch.from_numpy(xs).to(f"cuda:{dev}")
     dout = None
     for name, (m_, w_) in {"hios_lp": (M, args.window), "sequential": (1, 1),
-                           "ios_style": (1, args.window)}.items():
+                           "ios_style": (1, args.window), "ios": (1, args.window)}.items():
         t0 = time.perf_counter()
-        Sx = h.hios_schedule_lp(Gs, m_, w_)
+        if name == "ios":
+            # exact single-GPU DP, state budget bounded so the lazily
+            # profiled t(S) stay within the bench's time (NASNet: see DESIGN)
+            try:
+                Sx = h.hios_schedule_ios(Gs, w_, 1 << 14)
+            except h.HiosError as ex:
+                row["ios_unavailable"] = str(ex)
+                continue
+        else:
+            Sx = h.hios_schedule_lp(Gs, m_, w_)
         t_s = time.perf_counter() - t0
         if m_ > 1:
             ndev = torch.cuda.device_count()
@@ -389,9 +414,10 @@ def measure_workload(h, torch, model, sz, M, args, dev, stream, flush, pk, esz):
         if name == "hios_lp":
             og, ost, _ = h.hios_schedule_stages(Sx)
             Fs, Bs = op_work(gs, shp, esz)
-            row["cp_bound_ms"] = critical_path_bound(gs, Fs, Bs, og, ost, M, pk, esz, shp) * 1e3
-            row["seq_roofline_ms"] = float(np.maximum(Fs / (pk["bf16_tflops"] * 1e12),
+            row["cp_bound_ms"] = critical_path_bound(gs, Fs, Bs, og, ost, M, pk, esz, shp, dtype) * 1e3
+            row["seq_roofline_ms"] = float(np.maximum(Fs / (compute_peak(pk, dtype) * 1e12),
                                                       Bs / (pk["hbm_gbs"] * 1e9)).sum() * 1e3)
+            row["compute_peak_tflops"] = compute_peak(pk, dtype)
             row["gflop"] = float(Fs.sum() / 1e9)
             row["gpus_used"] = int(len(set(og.tolist())))
             row["schedule_s"] = t_s
@@ -399,6 +425,8 @@ def measure_workload(h, torch, model, sz, M, args, dev, stream, flush, pk, esz):
     row["cp_frac"] = row["cp_bound_ms"] / row["hios_lp_ms"]
     row["speedup_vs_sequential"] = row["sequential_ms"] / row["hios_lp_ms"]
     row["speedup_vs_ios_style"] = row["ios_style_ms"] / row["hios_lp_ms"]
+    if "ios_ms" in row:
+        row["speedup_vs_ios"] = row["ios_ms"] / row["hios_lp_ms"]
     del Gs
     return row
 
@@ -419,7 +447,7 @@ def main():
     ap.add_argument("--ref-budget", type=float, default=200.0,
                     help="seconds of oracle CPU work for the whole --impl reference run")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--sweep", default="2048,4096,randwire_ws@2048,nasnet_a_large@2048,squeezenet@2048",
+    ap.add_argument("--sweep", default="2048,4096,randwire_ws@2048,nasnet_a_large@2048,squeezenet@2048,4096:f32",
                     help="extra input sizes timed on 1 GPU (HIOS-LP / sequential / IOS-style), '' to skip")
     ap.add_argument("--logical", type=int, default=0,
                     help="single process: schedule over this many logical GPUs (aliased on visible devices)")
@@ -614,24 +642,24 @@ def main():
                              "frac": mb / ms_ / 1e9 / pk["hbm_gbs"], "launches_per_step": len(mem_ids),
                              "algorithmic_bytes_per_launch": mb / len(mem_ids)}
 
-    cp_s = critical_path_bound(g, F, B, op_gpu, op_stage, M, pk, esz, shapes)
+    cp_s = critical_path_bound(g, F, B, op_gpu, op_stage, M, pk, esz, shapes, args.dtype)
     # single-GPU references measured in the same run (rank 0, N == 1 only)
     extra = {}
     if world == 1:
+        # M = 1 also times HIOS-LP / HIOS-MR / LP-inter-only over 2 LOGICAL GPUs
+        # aliased on this device (one CUDA graph; a schedule-structure
+        # comparison executed on the hardware, not a 2-GPU measurement)
+        M2 = M if M > 1 else 2
         for name, (m_, w_) in {"sequential": (1, 1), "ios_style": (1, args.window), "ios": (1, args.window),
-                               "lp_inter_only": (M, 1), "hios_mr": (M, args.window)}.items():
-            if name in ("lp_inter_only", "hios_mr") and M == 1:
-                continue
-            if name == "ios" and g.n_ops > 150:
-                # the exact DP measures t(S) of every candidate group it visits:
-                # 11 min for NASNet-A (364 ops) -- reported as skipped, not run
-                extra[name] = {"unavailable": f"exact DP skipped for {g.n_ops} ops (bench time bound)"}
+                               "lp_inter_only": (M2, 1), "hios_mr": (M2, args.window),
+                               "hios_lp_2lgpu": (2, args.window)}.items():
+            if name == "hios_lp_2lgpu" and M > 1:
                 continue
             t_s0 = time.perf_counter()
             try:
                 if name == "hios_mr":
                     Sx = h.hios_schedule_mr(G, m_, w_)
-                elif name == "ios":  # exact single-GPU DP, t(S) profiled lazily
+                elif name == "ios":  # exact single-GPU DP, t(S) profiled lazily, bounded
                     Sx = h.hios_schedule_ios(G, w_)
                 else:
                     Sx = h.hios_schedule_lp(G, m_, w_)
@@ -649,17 +677,20 @@ def main():
                            "predicted_ms": h.hios_schedule_latency_ns(Sx) / 1e6,
                            "gpus_used": int(len(set(h.hios_schedule_stages(Sx)[0].tolist()))),
                            "schedule_s": t_sched_x}
+            if m_ > 1 and M == 1:
+                extra[name]["logical_gpus_aliased_on_one_device"] = m_
             del Sx
 
     sweep = {}
     if world == 1 and args.sweep and not os.environ.get("HIOS_NCU"):
         for item in [v for v in args.sweep.split(",") if v]:
-            model, sz = (item.split("@") if "@" in item else (args.model, item))
+            spec, dt = (item.split(":") if ":" in item else (item, args.dtype))
+            model, sz = (spec.split("@") if "@" in spec else (args.model, spec))
+            key = f"{model}@{sz}" + ("" if dt == args.dtype else f":{dt}")
             try:
-                sweep[f"{model}@{sz}"] = measure_workload(h, torch, model, int(sz), M, args, dev, stream,
-                                                          flush, pk, esz)
+                sweep[key] = measure_workload(h, torch, model, int(sz), M, args, dev, stream, flush, pk, dt)
             except Exception as ex:  # noqa: BLE001 -- reported, never silently dropped
-                sweep[f"{model}@{sz}"] = {"error": f"{type(ex).__name__}: {ex}"}
+                sweep[key] = {"error": f"{type(ex).__name__}: {ex}"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

@@ -1,84 +1,118 @@
-// conv_simt.cu -- fp32 implicit-GEMM convolution on CUDA cores (FFMA).
-// The fp32 path exists for the 1e-4 parity bar (north star); TF32 tensor
-// cores would not meet it (SURVEY §7 "fp32 parity at 1e-4 rules out TF32").
-// 64 pixels x 64 out-channels per CTA, K = R*S*C in steps of 16, 256 threads,
-// 4 x 4 outputs per thread, double-buffered smem tiles.
+// conv_simt.cu -- fp32 implicit-GEMM convolution on CUDA cores (FFMA), the
+// fp32 path (the north star's 1e-4 parity bar; TF32 tensor cores would not
+// meet it).
+//
+// GEMM view M = output pixels, N = output channels, K = R*S*C walked as
+// (tap (r, s), 16-channel chunk): for a fixed tap, the 16 channels of one input
+// pixel are contiguous in NHWC, so an A-tile row is 4 float4 loads and no
+// per-element index arithmetic (no div/mod in the K loop).  Weights are laid
+// out [K][R*S][Cp] with Cp = C rounded up to 16 and zero-padded, so a B-tile
+// row is 4 aligned float4 loads too.  CTA tile 128 x 128 x 16, 256 threads,
+// 8 x 8 outputs per thread: per k, two LDS.128 of A and two of B feed 64 FFMA
+// (FFMA-bound, not shared-memory bound); double-buffered shared tiles with the
+// next chunk's global loads in flight under the current chunk's FFMAs.
+// Roofline: 2*K*C*R*S*P*Q FLOP at the measured FP32 CUDA-core peak
+// (tools/fp32_peak.cu: 72.5 TFLOP/s on B200).
 #include "kernels.cuh"
 
 namespace hios {
 
-constexpr int SBM = 64, SBN = 64, SBK = 16;
+constexpr int SBM = 128, SBN = 128, SBK = 16, SPAD = 4;
 
 __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
   pdl_enter();
-  __shared__ float As[2][SBK][SBM + 4];
-  __shared__ float Bs[2][SBK][SBN + 4];
+  __shared__ __align__(16) float As[2][SBK][SBM + SPAD];
+  __shared__ __align__(16) float Bs[2][SBK][SBN + SPAD];
   const int t = threadIdx.x, tx = t & 15, ty = t >> 4;
   const int m0 = blockIdx.x * SBM, n0 = blockIdx.y * SBN;
-  const int M = a.P * a.Q, RSC = a.R * a.S * a.C;
-  // each thread loads 4 A elements and 4 B elements per K step: k = e % 16, row = e / 16
-  int am[4], aih[4], aiw[4];
-  bool avalid[4];
+  const int M = a.P * a.Q, RS = a.R * a.S, Cp = (a.C + 15) & ~15, nch = Cp >> 4;
+  // loads: 128 rows x 16 k = 512 float4 per operand, two per thread:
+  // row = t >> 1 (+ 0 / 128? no: rows t>>2 and 64 + (t>>2)), quad = t & 3
+  const int lrow = t >> 2, lq = (t & 3) * 4;
+  int ih[2], iw[2];
+  bool mval[2];
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const int e = t + i * 256, row = e >> 4;
-    const int m = m0 + row;
-    avalid[i] = m < M;
-    const int p = avalid[i] ? m / a.Q : 0, q = avalid[i] ? m % a.Q : 0;
-    am[i] = m;
-    aih[i] = p * a.sh - a.ph;
-    aiw[i] = q * a.sw - a.pw;
+  for (int i = 0; i < 2; ++i) {
+    const int m = m0 + lrow + 64 * i;
+    mval[i] = m < M;
+    const int p = mval[i] ? m / a.Q : 0, q = mval[i] ? m - (m / a.Q) * a.Q : 0;
+    ih[i] = p * a.sh - a.ph;
+    iw[i] = q * a.sw - a.pw;
   }
-  float acc[4][4];
+  bool nval[2];
+  const float* wrow[2];
 #pragma unroll
-  for (int i = 0; i < 4; ++i)
+  for (int i = 0; i < 2; ++i) {
+    const int n = n0 + lrow + 64 * i;
+    nval[i] = n < a.K;
+    wrow[i] = a.w + (size_t)(nval[i] ? n : 0) * RS * Cp;
+  }
+  float acc[8][8];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) acc[i][j] = 0.f;
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
 
-  float ra[4], rb[4];
-  auto gload = [&](int k0) {
+  float4 ra[2], rb[2];
+  auto gload = [&](int rs, int c0) {
+    const int r = rs / a.S, s = rs - r * a.S;  // once per 16-channel chunk
+    const int c = c0 + lq;
 #pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int e = t + i * 256, k = e & 15, row = e >> 4;
-      const int kg = k0 + k;
-      float v = 0.f;
-      if (avalid[i] && kg < RSC) {
-        const int rs = kg / a.C, c = kg - rs * a.C;
-        const int r = rs / a.S, s = rs - r * a.S;
-        const int h = aih[i] + r * a.dh, w = aiw[i] + s * a.dw;
-        if (h >= 0 && h < a.H && w >= 0 && w < a.W) v = __ldg(a.x + ((size_t)h * a.W + w) * a.ldx + c);
+    for (int i = 0; i < 2; ++i) {
+      float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+      const int h = ih[i] + r * a.dh, w = iw[i] + s * a.dw;
+      if (mval[i] && h >= 0 && h < a.H && w >= 0 && w < a.W) {
+        const float* px = a.x + ((size_t)h * a.W + w) * a.ldx;
+        if (c + 4 <= a.C) {
+          v = __ldg(reinterpret_cast<const float4*>(px + c));
+        } else {
+          if (c < a.C) v.x = __ldg(px + c);
+          if (c + 1 < a.C) v.y = __ldg(px + c + 1);
+          if (c + 2 < a.C) v.z = __ldg(px + c + 2);
+        }
       }
       ra[i] = v;
-      const int n = n0 + row;
-      rb[i] = (n < a.K && kg < RSC) ? __ldg(a.w + (size_t)n * RSC + kg) : 0.f;
+      rb[i] = nval[i] ? __ldg(reinterpret_cast<const float4*>(wrow[i] + (size_t)rs * Cp + c))
+                      : make_float4(0.f, 0.f, 0.f, 0.f);
     }
   };
   auto sstore = [&](int buf) {
 #pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int e = t + i * 256, k = e & 15, row = e >> 4;
-      As[buf][k][row] = ra[i];
-      Bs[buf][k][row] = rb[i];
+    for (int i = 0; i < 2; ++i) {
+      const int row = lrow + 64 * i;
+      As[buf][lq + 0][row] = ra[i].x;
+      As[buf][lq + 1][row] = ra[i].y;
+      As[buf][lq + 2][row] = ra[i].z;
+      As[buf][lq + 3][row] = ra[i].w;
+      Bs[buf][lq + 0][row] = rb[i].x;
+      Bs[buf][lq + 1][row] = rb[i].y;
+      Bs[buf][lq + 2][row] = rb[i].z;
+      Bs[buf][lq + 3][row] = rb[i].w;
     }
   };
-  gload(0);
+  const int nsteps = RS * nch;
+  gload(0, 0);
   sstore(0);
   __syncthreads();
-  int buf = 0;
-  for (int k0 = 0; k0 < RSC; k0 += SBK) {
-    const bool more = k0 + SBK < RSC;
-    if (more) gload(k0 + SBK);
+  int buf = 0, rs = 0, ch = 0;
+  for (int step = 0; step < nsteps; ++step) {
+    const bool more = step + 1 < nsteps;
+    if (more) {
+      if (++ch == nch) { ch = 0; ++rs; }
+      gload(rs, ch * 16);
+    }
 #pragma unroll
     for (int kk = 0; kk < SBK; ++kk) {
-      float av[4], bv[4];
+      const float4 a0 = *reinterpret_cast<const float4*>(&As[buf][kk][ty * 4]);
+      const float4 a1 = *reinterpret_cast<const float4*>(&As[buf][kk][64 + ty * 4]);
+      const float4 b0 = *reinterpret_cast<const float4*>(&Bs[buf][kk][tx * 4]);
+      const float4 b1 = *reinterpret_cast<const float4*>(&Bs[buf][kk][64 + tx * 4]);
+      const float av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+      const float bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
 #pragma unroll
-      for (int i = 0; i < 4; ++i) av[i] = As[buf][kk][ty * 4 + i];
+      for (int i = 0; i < 8; ++i)
 #pragma unroll
-      for (int j = 0; j < 4; ++j) bv[j] = Bs[buf][kk][tx * 4 + j];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
     }
     if (more) {
       sstore(buf ^ 1);
@@ -86,18 +120,31 @@ __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
       buf ^= 1;
     }
   }
+  // epilogue: rows ty*4 + {0..3} and 64 + ty*4 + {0..3}; columns likewise
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const int m = m0 + ty * 4 + i;
+  for (int i = 0; i < 8; ++i) {
+    const int m = m0 + (i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4);
     if (m >= M) continue;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int n = n0 + tx * 4 + j;
-      if (n >= a.K) continue;
-      float y = acc[i][j] * a.scale[n] + a.shift[n];
-      if (a.relu) y = fmaxf(y, 0.f);
-      a.out[(size_t)m * a.ldo + n] = y;
-      for (int d_ = 0; d_ < a.out2.n; ++d_) a.out2.p[d_][(size_t)m * a.out2.ld[d_] + n] = y;
+    for (int h2 = 0; h2 < 2; ++h2) {
+      const int nb = n0 + h2 * 64 + tx * 4;
+      float y[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int n = min(nb + j, a.K - 1);
+        y[j] = acc[i][h2 * 4 + j] * __ldg(a.scale + n) + __ldg(a.shift + n);
+        if (a.relu) y[j] = fmaxf(y[j], 0.f);
+      }
+      float* o = a.out + (size_t)m * a.ldo;
+      if (nb + 4 <= a.K && ((a.ldo | nb) & 3) == 0 && (reinterpret_cast<uintptr_t>(a.out) & 15) == 0) {
+        *reinterpret_cast<float4*>(o + nb) = make_float4(y[0], y[1], y[2], y[3]);
+      } else {
+        for (int j = 0; j < 4 && nb + j < a.K; ++j) o[nb + j] = y[j];
+      }
+      for (int d_ = 0; d_ < a.out2.n; ++d_) {
+        float* o2 = a.out2.p[d_] + (size_t)m * a.out2.ld[d_];
+        for (int j = 0; j < 4 && nb + j < a.K; ++j) o2[nb + j] = y[j];
+      }
     }
   }
 }

@@ -276,7 +276,8 @@ static void upload_weights_T(Executor& ex, int v) {
   const bool tc = ex.g.dtype == HIOS_BF16;
   switch (o.kind) {
     case HIOS_OP_CONV: {
-      const int Cp = tc ? rup(o.in_c, 64) : o.in_c;  // bf16: whole 64-channel chunks (zero-padded)
+      // bf16: whole 64-channel chunks, fp32 SIMT: whole 16-channel chunks (zero-padded)
+      const int Cp = tc ? rup(o.in_c, 64) : rup(o.in_c, 16);
       if (tc && s2d_conv(o)) {
         // W'[k][r'*S'+s'][(a*2+b)*C + c] (see s2d_conv)
         const int R2 = (o.kh + 1) / 2, S2 = (o.kw + 1) / 2, C = o.in_c, Cp2 = rup(4 * C, 64);
@@ -321,7 +322,7 @@ static void upload_weights_T(Executor& ex, int v) {
           for (int rs = 0; rs < RS; ++rs) dw[(size_t)rs * c + ch] = o.weight[off + (size_t)ch * RS + rs];
         off += (size_t)c * RS;
         x.dw.push_back((float*)upload(L, dw));
-        const int Cp = tc ? rup(c, 64) : c;
+        const int Cp = tc ? rup(c, 64) : rup(c, 16);
         x.pw.push_back(upload(L, conv_layout<T>(o.weight.data() + off, o.out_c, c, 1, 1, Cp)));
         off += (size_t)o.out_c * c;
         std::vector<float> sc(o.scale.begin() + (size_t)r * o.out_c, o.scale.begin() + (size_t)(r + 1) * o.out_c);
@@ -1059,13 +1060,14 @@ void Executor::enqueue_stage(int l, const std::vector<int>& S, bool timed, int64
     nk += solo ? ox[v].n_kernels_solo : ox[v].n_kernels;
     post(v, st);
   };
-  if (S.size() == 1) {
+  static const int gmode = getenv("HIOS_GROUP_MODE") ? atoi(getenv("HIOS_GROUP_MODE")) : 0;  // A/B (temporary)
+  if (S.size() == 1 && gmode != 2) {
     run_one(S[0], s0);
     return;
   }
   std::vector<int> grp, rest;
   for (int v : S) (group_convs && ox[v].tc.size() == 1 ? grp : rest).push_back(v);
-  if (grp.size() < 2 || (int)grp.size() > kMaxGroup) {
+  if (grp.size() < (gmode == 2 ? 1u : 2u) || (int)grp.size() > kMaxGroup) {
     grp.clear();
     rest = S;
   }
@@ -1091,9 +1093,9 @@ void Executor::enqueue_stage(int l, const std::vector<int>& S, bool timed, int64
     }
     for (int v : rest) wr += g.ops[v].cost > 0 ? (double)g.ops[v].cost : 1.0;
     int budget = L.num_sms;
-    if (!rest.empty())
+    if (!rest.empty() && gmode != 3)
       budget = std::max((int)grp.size(), std::min(L.num_sms - 16, (int)std::lround(L.num_sms * wc / (wc + wr))));
-    const std::vector<int> c = partition_ctas(tiles, tau, budget);
+    const std::vector<int> c = gmode == 1 ? tiles : partition_ctas(tiles, tau, budget);
     ConvTcGroup G;
     std::memset(&G, 0, sizeof(G));
     G.n = (int)grp.size();

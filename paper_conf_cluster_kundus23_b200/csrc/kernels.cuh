@@ -168,7 +168,7 @@ struct ConvTcOp {
   CUtensorMap mx, mw, mo, mo2;
   ConvTcArgs a;
 };
-constexpr int kMaxGroup = 8;
+constexpr int kMaxGroup = 6;
 struct ConvTcGroup {
   ConvTcOp op[kMaxGroup];
   int n;

@@ -87,6 +87,8 @@ def load() -> C.CDLL:
         "hios_schedule_transfers": [VP, P(I32), P(I32), I32, P(I32)],
     }
     for name, args in sig.items():
+        if not hasattr(lib, name):  # an older build (A/B timing via HIOS_LIB)
+            continue
         f = getattr(lib, name)
         f.argtypes = args
         f.restype = C.c_int
