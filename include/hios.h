@@ -229,6 +229,22 @@ hios_status hios_schedule_place(hios_schedule s, const int32_t* devices, int32_t
 typedef enum { HIOS_TRANSPORT_PEER = 0, HIOS_TRANSPORT_COPY = 1, HIOS_TRANSPORT_NCCL = 2 } hios_transport;
 hios_status hios_schedule_transport(hios_schedule s, int32_t transport);
 
+/* How a stage's concurrent group is launched; must
+ * precede the first run.
+ *   HIOS_STAGE_STREAMS (default): every op of the stage on its own stream of
+ *     the GPU (fork from / join into the stage's first stream), each kernel
+ *     free to take any SM the hardware gives it.
+ *   HIOS_STAGE_GROUPED: the stage's plain tcgen05 convolutions as ONE
+ *     persistent launch (conv_tc_group_kernel) that partitions the SMs across
+ *     them -- op i owns a CTA range sized to minimise the stage's makespan from
+ *     the measured t(v) -- and the stage's other ops on forked streams.
+ *     (hios_profile measures t(S) with streams.)  (Measured on one B200,
+ *     Inception-v3 HIOS-LP w = 5: 0.80 ms grouped vs 0.74 ms streams at 1024^2;
+ *     DESIGN.md §6.)
+ * Errors: HIOS_E_INVALID (unknown mode), HIOS_E_STATE (already run). */
+typedef enum { HIOS_STAGE_STREAMS = 0, HIOS_STAGE_GROUPED = 1 } hios_stage_mode;
+hios_status hios_schedule_stage_mode(hios_schedule s, int32_t mode);
+
 /* NCCL transport set-up.  hios_nccl_unique_id writes a 128-byte ncclUniqueId
  * (call on one rank, broadcast the bytes); hios_schedule_nccl_init creates
  * this rank's communicator (nranks processes, this one = rank, on the device

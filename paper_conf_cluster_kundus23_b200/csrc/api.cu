@@ -272,6 +272,15 @@ hios_status hios_schedule_transport(hios_schedule s, int32_t transport) {
   });
 }
 
+hios_status hios_schedule_stage_mode(hios_schedule s, int32_t mode) {
+  return guard([&] {
+    NEED(s, HIOS_E_INVALID, "NULL schedule");
+    NEED(mode == HIOS_STAGE_STREAMS || mode == HIOS_STAGE_GROUPED, HIOS_E_INVALID, "unknown stage mode");
+    NEED(!s->s->exec, HIOS_E_STATE, "set the stage mode before the first run");
+    s->s->stage_mode = mode;
+  });
+}
+
 hios_status hios_nccl_unique_id(void* id128) {
   return guard([&] {
     NEED(id128, HIOS_E_INVALID, "NULL id");

@@ -66,7 +66,7 @@ static inline int64_t rup64(int64_t x, int64_t m) { return (x + m - 1) / m * m; 
 
 Executor::Executor(Schedule& sch) : s(sch), g(*sch.g), M(sch.M) {
   esz = g.dtype == HIOS_BF16 ? 2 : 4;
-  group_convs = getenv("HIOS_NOGROUP") == nullptr;  // A/B switch: per-op streams for every stage
+  group_convs = sch.stage_mode == HIOS_STAGE_GROUPED;
   transport = sch.transport;
   int ndev = 0;
   ck(cudaGetDeviceCount(&ndev), "cudaGetDeviceCount");
@@ -1060,14 +1060,13 @@ void Executor::enqueue_stage(int l, const std::vector<int>& S, bool timed, int64
     nk += solo ? ox[v].n_kernels_solo : ox[v].n_kernels;
     post(v, st);
   };
-  static const int gmode = getenv("HIOS_GROUP_MODE") ? atoi(getenv("HIOS_GROUP_MODE")) : 0;  // A/B (temporary)
-  if (S.size() == 1 && gmode != 2) {
+  if (S.size() == 1) {
     run_one(S[0], s0);
     return;
   }
   std::vector<int> grp, rest;
   for (int v : S) (group_convs && ox[v].tc.size() == 1 ? grp : rest).push_back(v);
-  if (grp.size() < (gmode == 2 ? 1u : 2u) || (int)grp.size() > kMaxGroup) {
+  if (grp.size() < 2 || (int)grp.size() > kMaxGroup) {
     grp.clear();
     rest = S;
   }
@@ -1093,9 +1092,9 @@ void Executor::enqueue_stage(int l, const std::vector<int>& S, bool timed, int64
     }
     for (int v : rest) wr += g.ops[v].cost > 0 ? (double)g.ops[v].cost : 1.0;
     int budget = L.num_sms;
-    if (!rest.empty() && gmode != 3)
+    if (!rest.empty())
       budget = std::max((int)grp.size(), std::min(L.num_sms - 16, (int)std::lround(L.num_sms * wc / (wc + wr))));
-    const std::vector<int> c = gmode == 1 ? tiles : partition_ctas(tiles, tau, budget);
+    const std::vector<int> c = partition_ctas(tiles, tau, budget);
     ConvTcGroup G;
     std::memset(&G, 0, sizeof(G));
     G.n = (int)grp.size();

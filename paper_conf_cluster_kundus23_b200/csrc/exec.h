@@ -146,7 +146,7 @@ struct Executor {
   // runs after op v on the stream v ran on
   void enqueue_stage(int l, const std::vector<int>& S, bool timed, int64_t& nk,
                      const std::function<void(int, cudaStream_t)>& post);
-  bool group_convs = true;
+  bool group_convs = false;  // hios_schedule_stage_mode
 };
 
 void ck(cudaError_t e, const char* what);

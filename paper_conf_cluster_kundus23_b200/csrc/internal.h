@@ -83,6 +83,7 @@ struct Schedule {
   std::vector<int> owner;    // per logical GPU: process rank (empty = all local)
   int rank = 0;
   int transport = HIOS_TRANSPORT_PEER;
+  int stage_mode = HIOS_STAGE_STREAMS;
   std::unique_ptr<Executor> exec;
   ~Schedule();
 };

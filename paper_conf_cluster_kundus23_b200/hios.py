@@ -82,6 +82,7 @@ def load() -> C.CDLL:
         "hios_kernel_count": [VP, P(I64)],
         "hios_time_ops": [VP, I32, I64, P(I64)],
         "hios_schedule_transport": [VP, I32],
+        "hios_schedule_stage_mode": [VP, I32],
         "hios_nccl_unique_id": [VP],
         "hios_schedule_nccl_init": [VP, VP, I32, I32],
         "hios_schedule_transfers": [VP, P(I32), P(I32), I32, P(I32)],
@@ -340,6 +341,14 @@ TRANSPORT = {"peer": 0, "copy": 1, "nccl": 2}
 def hios_schedule_transport(s: Schedule, transport):
     t = TRANSPORT[transport] if isinstance(transport, str) else int(transport)
     _ck(load().hios_schedule_transport(s.h, t))
+
+
+STAGE_MODE = {"streams": 0, "grouped": 1}
+
+
+def hios_schedule_stage_mode(s: Schedule, mode):
+    m = STAGE_MODE[mode] if isinstance(mode, str) else int(mode)
+    _ck(load().hios_schedule_stage_mode(s.h, m))
 
 
 def hios_nccl_unique_id() -> bytes:

@@ -139,3 +139,24 @@ def test_transports_bit_identical(name, size, transport):
         assert len(set(og.tolist())) > 1
         y = h.hios_run(S, x)
         assert np.array_equal(y, y1), (M, w, transport)
+
+
+@pytest.mark.parametrize("name,size", [("inception_v3", 299), ("inception_v3", 1024), ("randwire_ws", 224)])
+def test_grouped_stage_kernel_bit_identical(name, size):
+    """HIOS_STAGE_GROUPED (f2: a stage's tcgen05 convs in one launch with an
+    explicit SM partition, conv_tc_group_kernel) computes exactly what the
+    per-op streams compute, on 1 GPU and on 2 logical GPUs; fewer kernels."""
+    h = hios()
+    g = graphs.build(name, size)
+    W = gen.make_weights(g)
+    x = gen.make_input(g)
+    G = h.hios_graph_create(g.ops, g.edges, g.in_c, g.in_h, g.in_w, "bf16", W)
+    h.hios_profile(G, [0], 3)
+    for M, w in [(1, 5), (2, 3)]:
+        S1 = h.hios_schedule_lp(G, M, w)
+        y1 = h.hios_run(S1, x)
+        S2 = h.hios_schedule_lp(G, M, w)
+        h.hios_schedule_stage_mode(S2, "grouped")
+        y2 = h.hios_run(S2, x)
+        assert np.array_equal(y1, y2), (M, w)
+        assert h.hios_kernel_count(S2) <= h.hios_kernel_count(S1)
