@@ -33,8 +33,9 @@ def main():
     out = {"workload": workload, "launches": len(launches), "bytes_per_launch": tot / max(len(launches), 1),
            "source": os.path.basename(path) + " (ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,"
                      "dram__bytes_write.sum --clock-control none, cold caches)"}
-    dst = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles",
-                       f"conv_traffic_{workload}.json")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    # on the GPU box only gpurun_out/ comes back: write there, copy to profiles/ here
+    dst = os.path.join(root, sys.argv[3] if len(sys.argv) > 3 else "profiles", f"conv_traffic_{workload}.json")
     json.dump(out, open(dst, "w"), indent=1)
     print(json.dumps(out))
 
