@@ -76,7 +76,7 @@ typedef enum {
 
 /* One vertex of G.  Weight layouts (fp32, copied at create):
  *   CONV     weight [out_c][in_c][kh][kw]; scale/shift [out_c] (folded BN;
- *            NULL = 1 / 0); y = relu?(scale * conv(x, W) + shift)
+ *            NULL = 1 / 0); y = relu?(scale * conv(pre_relu ? relu(x) : x, W) + shift)
  *   SEPCONV  weight = concat over r < reps of { dw [c_r][kh][kw], pw [out_c][c_r] }
  *            with c_0 = in_c, c_r = out_c for r > 0; scale/shift [reps][out_c];
  *            stride (sh, sw) on r = 0 only; pad (ph, pw); pre_relu before each

@@ -12,8 +12,9 @@ evaluated in topological order, in float64 by default (the paper does not fix
 the precision).
 
 Operator definitions (NCHW, batch 1, zero padding):
-  conv    y[k,p,q] = act(scale[k] * sum_{c,r,s} x[c, p*sh-ph+r*dh, q*sw-pw+s*dw]
+  conv    y[k,p,q] = act(scale[k] * sum_{c,r,s} x'[c, p*sh-ph+r*dh, q*sw-pw+s*dw]
                                                * W[k,c,r,s] + shift[k])
+          x' = relu(x) when the op has pre_relu (NASNet's ReLU -> conv -> BN), else x
           (conv + folded BN + ReLU = one operator)
   sepconv per repetition: a = sum_i agg_i x_i ; a = relu(a) if pre_relu ;
           d[c,p,q] = sum_{r,s} a[c, p*sh-ph+r, q*sw-pw+s] * Wd[c,r,s] ;
@@ -114,7 +115,8 @@ def relu(a):
 def run_op(op, ins: List[np.ndarray], w: Dict, dtype=np.float64) -> np.ndarray:
     k = op.kind
     if k == "conv":
-        y = conv2d(ins[0], w["weight"].astype(dtype), op.sh, op.sw, op.ph, op.pw, op.dh, op.dw)
+        x = relu(ins[0]) if getattr(op, "pre_relu", 0) else ins[0]
+        y = conv2d(x, w["weight"].astype(dtype), op.sh, op.sw, op.ph, op.pw, op.dh, op.dw)
         y = y * w["scale"].astype(dtype)[:, None, None] + w["shift"].astype(dtype)[:, None, None]
         return relu(y) if op.relu else y
     if k == "sepconv":

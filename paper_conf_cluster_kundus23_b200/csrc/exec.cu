@@ -182,6 +182,24 @@ void Executor::plan() {
       }
     }
   }
+  // pre-ReLU convs: one ReLU'd copy of the input per (producer, GPU) when the
+  // producer runs on that GPU (made right after it), else a per-consumer scratch
+  relu_loc.clear();
+  for (int v = 0; v < n; ++v) {
+    const Op& o = g.ops[v];
+    if (o.kind != HIOS_OP_CONV || !o.pre_relu) continue;
+    const int u = g.edges[o.in_edges[0]].src, l = s.gpu_of[v];
+    const Op& ou = g.ops[u];
+    const int ldc = rup(ou.C, 8);
+    const int64_t bytes = (int64_t)ou.H * ou.W * ldc * esz;
+    if (s.gpu_of[u] == l && ou.kind != HIOS_OP_INPUT) {
+      const int64_t key = (int64_t)u * M + l;
+      if (!relu_loc.count(key)) relu_loc[key] = Loc{alloc(l, bytes), ldc};
+    } else {
+      ox[v].relubuf = alloc(l, bytes);
+      ox[v].relu_ldc = ldc;
+    }
+  }
   // remote deliveries and flags
   flag_index.assign(n, std::vector<int>(M, -1));
   std::vector<int> nflags(M, 0);
@@ -744,8 +762,24 @@ static void build_op(Executor& ex, int v) {
     case HIOS_OP_CONV: {
       const int u = in_op(0);
       const Op& xi = g.ops[u];
+      // the conv's input: u's output, or (pre-ReLU conv) its ReLU'd copy --
+      // made once after u on u's GPU (shared by every pre-ReLU consumer there)
+      // or, for a remote / input producer, here into this op's scratch
+      View cin = view_of(u, l);
+      if (o.pre_relu) {
+        auto it = ex.relu_loc.find((int64_t)u * ex.M + l);
+        if (it != ex.relu_loc.end()) {
+          cin = View{ex.ptr(l, it->second.off), it->second.ldc};
+        } else {
+          const View rv{ex.ptr(l, x.relubuf), x.relu_ldc};
+          CopyArgs<T> c{(const T*)cin.p, cin.ldc, xi.H * xi.W, xi.C, (T*)rv.p, rv.ldc};
+          fns.push_back([c](cudaStream_t st) { launch_relu_copy<T>(c, st); });
+          ++nk;
+          cin = rv;
+        }
+      }
       if (stem3_conv(o)) {
-        View iv = view_of(u, l);
+        View iv = cin;
         if (iv.ldc < (int)(16 / sizeof(T))) fail(HIOS_E_UNSUPPORTED, "stem input pixel pitch below 16 bytes");
         ConvStem3Args<T> c{};
         c.x = (const T*)iv.p; c.H = xi.H; c.W = xi.W; c.ldx = iv.ldc;
@@ -773,7 +807,7 @@ static void build_op(Executor& ex, int v) {
         break;
       }
       if (x.s2dbuf >= 0) {
-        View iv = view_of(u, l);
+        View iv = cin;
         const int R2 = (o.kh + 1) / 2, S2 = (o.kw + 1) / 2;
         const int H2 = o.H + R2 - 1, W2 = o.W + S2 - 1;
         View sv{ex.ptr(l, x.s2dbuf), x.s2d_ldc};
@@ -794,7 +828,7 @@ static void build_op(Executor& ex, int v) {
         break;
       }
       if (small_c_conv(o)) {
-        View iv = view_of(u, l);
+        View iv = cin;
         ConvSmallArgs<T> c{};
         c.x = (const T*)iv.p; c.H = xi.H; c.W = xi.W; c.C = xi.C; c.ldx = iv.ldc;
         c.w = x.w_small; c.scale = x.scale[0]; c.shift = x.shift[0];
@@ -812,7 +846,7 @@ static void build_op(Executor& ex, int v) {
         g_tc_out = &x.tc;
         g_tc_smem = &x.tc_smem;
       }
-      fns.push_back(conv_closure<T>(ex, view_of(u, l), xi.H, xi.W, xi.C, x.w, x.scale[0], x.shift[0], o.out_c, o.kh,
+      fns.push_back(conv_closure<T>(ex, cin, xi.H, xi.W, xi.C, x.w, x.scale[0], x.shift[0], o.out_c, o.kh,
                                     o.kw, o.sh, o.sw, o.ph, o.pw, o.dh, o.dw, o.H, o.W, o.relu, out, out2, nk));
       g_tc_out = nullptr;
       g_tc_smem = nullptr;
@@ -924,6 +958,14 @@ static void build_op(Executor& ex, int v) {
       fns.push_back([c](cudaStream_t st) { launch_copy<T>(c, st); });
       ++nk;
       break;
+    }
+  }
+  {  // ReLU'd copy of this op's output for the pre-ReLU convs that read it here
+    auto it = ex.relu_loc.find((int64_t)v * ex.M + l);
+    if (it != ex.relu_loc.end()) {
+      CopyArgs<T> c{(const T*)out.p, out.ldc, o.H * o.W, o.C, (T*)ex.ptr(l, it->second.off), it->second.ldc};
+      fns.push_back([c](cudaStream_t st) { launch_relu_copy<T>(c, st); });
+      ++nk;
     }
   }
   x.run = [fns](cudaStream_t st) {

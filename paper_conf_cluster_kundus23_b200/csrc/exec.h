@@ -46,6 +46,9 @@ struct OpExec {
   int ldw = 0;
   // sepconv scratch (arena offsets)
   int64_t dwbuf = -1, midbuf = -1;
+  // pre-ReLU conv whose producer is remote / the input: its ReLU'd input copy
+  int64_t relubuf = -1;
+  int relu_ldc = 0;
   int dw_ldc = 0, mid_ldc = 0;
   // stride-2 small-C stem (bf16): space-to-depth copy of the input (arena offset)
   int64_t s2dbuf = -1;
@@ -101,6 +104,7 @@ struct Executor {
   int esz;  // element size
   std::vector<LGpu> lg;
   std::vector<std::vector<Loc>> loc;   // loc[op][lgpu]
+  std::map<int64_t, Loc> relu_loc;     // (producer * M + lgpu) -> ReLU'd copy for pre-ReLU convs
   std::vector<char> inplace;           // per edge: producer writes into the concat slice
   std::vector<OpExec> ox;
   std::vector<std::vector<int>> flag_index;  // [op][lgpu] flag slot on that lgpu (-1 none)

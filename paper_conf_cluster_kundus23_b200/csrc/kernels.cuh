@@ -203,6 +203,7 @@ template <typename T> void launch_dw(const DwArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_pool(const PoolArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_add(const AddArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_copy(const CopyArgs<T>& a, cudaStream_t st);
+template <typename T> void launch_relu_copy(const CopyArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_s2d(const S2dArgs<T>& a, cudaStream_t st);
 template <typename T> void launch_gap(const T* x, int HW, int C, int ldx, T* out, cudaStream_t st);
 template <typename T> void launch_linear(const T* x, int Cin, const T* w, int ldw, const float* b, int K,

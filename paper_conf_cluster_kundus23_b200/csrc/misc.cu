@@ -1010,6 +1010,48 @@ void launch_copy(const CopyArgs<T>& a, cudaStream_t st) {
   launch_pdl(copy_kernel<T>, dim3(grid_for(n, 256)), dim3(256), 0, st, a);
 }
 
+// ReLU copy (the input of a pre-ReLU conv, NASNet's ReLU -> conv -> BN): one
+// thread per (pixel, N-channel vector), 16-byte vectors when aligned.
+template <typename T>
+__global__ void relu_copy_kernel(const CopyArgs<T> a) {
+  pdl_enter();
+  constexpr int N = Vec<T>::N;
+  const int CG = (a.C + N - 1) / N;
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= a.HW * CG) return;
+  const int c = (idx % CG) * N;
+  const size_t pix = idx / CG;
+  const T* src = a.x + pix * a.ldx + c;
+  T* dst = a.out + pix * a.ldo + c;
+  const uintptr_t al = reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst);
+  if (c + N <= a.C && (al & 15) == 0) {
+    uint4 v = *reinterpret_cast<const uint4*>(src);
+    if constexpr (sizeof(T) == 2) {
+      __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&v);
+      const __nv_bfloat162 z = __floats2bfloat162_rn(0.f, 0.f);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) h[j] = __hmax2(h[j], z);
+    } else {
+      float* f = reinterpret_cast<float*>(&v);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) f[j] = fmaxf(f[j], 0.f);
+    }
+    *reinterpret_cast<uint4*>(dst) = v;
+  } else {
+    for (int j = 0; j < N && c + j < a.C; ++j) {
+      const float f = to_f(src[j]);
+      dst[j] = from_f<T>(f > 0.f ? f : 0.f);
+    }
+  }
+}
+
+template <typename T>
+void launch_relu_copy(const CopyArgs<T>& a, cudaStream_t st) {
+  constexpr int N = Vec<T>::N;
+  long long n = (long long)a.HW * ((a.C + N - 1) / N);
+  launch_pdl(relu_copy_kernel<T>, dim3(grid_for(n, 256)), dim3(256), 0, st, a);
+}
+
 // ------------------------------------------------------------------- GAP
 // one block per 8/4-channel group; threads stride over pixels; smem reduce
 template <typename T>
@@ -1205,6 +1247,7 @@ void launch_s2d(const S2dArgs<T>& a, cudaStream_t st) {
   template void launch_dw<T>(const DwArgs<T>&, cudaStream_t);                                          \
   template void launch_add<T>(const AddArgs<T>&, cudaStream_t);                                        \
   template void launch_copy<T>(const CopyArgs<T>&, cudaStream_t);                                      \
+  template void launch_relu_copy<T>(const CopyArgs<T>&, cudaStream_t);                                 \
   template void launch_s2d<T>(const S2dArgs<T>&, cudaStream_t);                                        \
   template void launch_gap<T>(const T*, int, int, int, T*, cudaStream_t);                              \
   template void launch_linear<T>(const T*, int, const T*, int, const float*, int, T*, cudaStream_t);        \

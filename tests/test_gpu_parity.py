@@ -317,3 +317,33 @@ def test_stem3_concat_slice(dtype):
     _, S, y = run_graph_gpu(g, W, x, dtype, profile=False)
     ref = infer.run_graph(g, W, x)[g.n_ops - 1]
     assert nerr(y.reshape(ref.shape), ref) <= TOL[dtype] / (4 if dtype == "bf16" else 1)
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+@pytest.mark.parametrize("M", [1, 2])
+def test_pre_relu_conv_and_factorized_reduction(dtype, M):
+    """NASNet pieces: pre-ReLU 1x1 convs sharing one ReLU'd copy of their input
+    (made after the producer), the factorized reduction (stride-2 1x1 conv +
+    single-tap 3x3/s2/p1 conv + concat) on an odd-sized input, and on M = 2
+    logical GPUs the consumer-side ReLU copy of a remote input."""
+    g = graphs.GraphSpec("nasfr", 24, 45, 37)
+    x0 = g.input()
+    a = g.conv(x0, 40, 3, p=1, relu=0)
+    f1 = g.conv(a, 32, 1, relu=0, pre_relu=1)
+    f2 = g.conv(a, 16, 1, relu=0, pre_relu=1)
+    fr = graphs._nas_factorized(g, a, 48, "fr")
+    g.concat([g.maxpool(f1, 3, 2, 1), g.maxpool(f2, 3, 2, 1), fr])
+    W = gen.make_weights(g)
+    x = gen.make_input(g) - 0.5
+    h = hios()
+    G = h.hios_graph_create(g.ops, g.edges, g.in_c, g.in_h, g.in_w, dtype, W)
+    for op in g.ops:
+        h.hios_set_op_cost(G, op.id, 0 if op.kind == "input" else 10000)
+    for e in range(g.n_edges):
+        h.hios_set_edge_cost(G, e, 50)
+    h.hios_set_group_model(G, 9, 10)
+    S = h.hios_schedule_lp(G, M, 2)
+    y = h.hios_run(S, x)
+    per_op_check(g, W, S, dtype)
+    ref = infer.run_graph(g, W, x)[g.n_ops - 1].reshape(-1)
+    assert nerr(y, ref) <= TOL[dtype]

@@ -252,3 +252,56 @@ def test_identity_is_a_copy():
     y = I.run_op(g.ops[i], [out[c]], {})
     y += 1.0                                       # a copy, not a view of the input
     assert np.array_equal(out[i], out[c])
+
+
+def test_conv_pre_relu_vs_torch():
+    """conv with pre_relu (NASNet's ReLU -> conv -> BN): torch fp64 relu then conv2d."""
+    g = graphs.GraphSpec("pr", 5, 9, 11)
+    x0 = g.input()
+    c = g.conv(x0, 7, 3, s=2, p=1, relu=0, pre_relu=1)
+    W = gen.make_weights(g)
+    x = gen.make_input(g) - 0.5            # negative inputs: the pre-ReLU matters
+    out = I.run_graph(g, W, x)
+    t = F.relu(torch.from_numpy(x.astype(np.float64)))
+    ref = F.conv2d(t, torch.from_numpy(W[c]["weight"].astype(np.float64)), stride=2, padding=1)[0]
+    ref = ref * torch.from_numpy(W[c]["scale"].astype(np.float64))[:, None, None] + \
+        torch.from_numpy(W[c]["shift"].astype(np.float64))[:, None, None]
+    np.testing.assert_allclose(out[c], ref.numpy(), rtol=1e-12, atol=1e-12)
+    assert not np.allclose(out[c], I.conv2d(x[0].astype(np.float64), W[c]["weight"].astype(np.float64), 2, 2, 1, 1)
+                           * W[c]["scale"][:, None, None] + W[c]["shift"][:, None, None])
+
+
+@pytest.mark.parametrize("H", [12, 13])
+def test_nasnet_factorized_reduction_vs_reference_formulation(H):
+    """The factorized reduction as the public NASNet-A code writes it (ReLU;
+    path 1 = AvgPool(1, stride 2) -> 1x1 conv; path 2 = pad (0,1,0,1), drop
+    the first row / column, AvgPool(1, stride 2) -> 1x1 conv; concat) against
+    this IR's reading: a stride-2 1x1 conv and a 3x3 / stride 2 / pad 1 conv
+    whose only non-zero tap is (2, 2) (workloads/graphs.py _nas_factorized),
+    even and odd input sizes."""
+    g = graphs.GraphSpec("fr", 6, H, H)
+    x0 = g.input()
+    cat = graphs._nas_factorized(g, x0, 8, "fr")
+    p1, p2 = g.preds(cat)
+    W = gen.make_weights(g)
+    x = gen.make_input(g) - 0.5
+    out = I.run_graph(g, W, x)
+    t = F.relu(torch.from_numpy(x.astype(np.float64)))
+    a = F.avg_pool2d(t, 1, stride=2, count_include_pad=False)
+    w1 = torch.from_numpy(W[p1]["weight"].astype(np.float64))
+    y1 = F.conv2d(a, w1)
+    b = F.pad(t, (0, 1, 0, 1))[:, :, 1:, 1:]
+    b = F.avg_pool2d(b, 1, stride=2, count_include_pad=False)
+    w2 = torch.from_numpy(W[p2]["weight"][:, :, 2, 2].astype(np.float64))[:, :, None, None]
+    y2 = F.conv2d(b, w2)
+
+    def bn(y, v):
+        return y * torch.from_numpy(W[v]["scale"].astype(np.float64))[None, :, None, None] + \
+            torch.from_numpy(W[v]["shift"].astype(np.float64))[None, :, None, None]
+    ref = torch.cat([bn(y1, p1), bn(y2, p2)], 1)[0].numpy()
+    assert out[cat].shape == ref.shape
+    np.testing.assert_allclose(out[cat], ref, rtol=1e-12, atol=1e-12)
+    # the single-tap conv's other taps are zero in the generated weights
+    wt = W[p2]["weight"].copy()
+    wt[:, :, 2, 2] = 0
+    assert not wt.any()

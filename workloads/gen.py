@@ -6,6 +6,7 @@ float32 arrays.
 
   input  x ~ U[0, 1), shape (1, C, H, W), seed 0
   conv   W ~ N(0, 2 / fan_in) (He-normal), shape (K, C, kh, kw), seed 1000 + op id
+         (a single-tap conv, op.tap = (r, s): fan_in = C and every other tap zero)
          folded BN: scale ~ U[0.5, 1.5], shift ~ N(0, 0.1^2)  (same generator)
   sepconv  per repetition r: depthwise Wd ~ N(0, 2/(kh*kw)) shape (C, kh, kw),
            pointwise Wp ~ N(0, 2/C) shape (K, C), scale, shift
@@ -34,9 +35,14 @@ def make_weights(g: GraphSpec, base_seed: int = 1000) -> Dict[int, Dict[str, np.
         rng = np.random.default_rng(base_seed + op.id)
         w: Dict[str, np.ndarray] = {}
         if op.kind == "conv":
-            fan_in = op.in_c * op.kh * op.kw
+            tap = getattr(op, "tap", None)
+            fan_in = op.in_c * (1 if tap else op.kh * op.kw)
             w["weight"] = rng.normal(0.0, np.sqrt(2.0 / fan_in),
                                      (op.out_c, op.in_c, op.kh, op.kw)).astype(np.float32)
+            if tap:  # single-tap conv: the other taps are structurally zero
+                mask = np.zeros((op.kh, op.kw), dtype=np.float32)
+                mask[tap[0], tap[1]] = 1.0
+                w["weight"] *= mask
             w["scale"] = rng.uniform(0.5, 1.5, op.out_c).astype(np.float32)
             w["shift"] = rng.normal(0.0, 0.1, op.out_c).astype(np.float32)
         elif op.kind == "sepconv":

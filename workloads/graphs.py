@@ -49,6 +49,7 @@ class OpSpec:
     agg: int = 0           # add / sepconv: weighted aggregation of the inputs
     reps: int = 1          # sepconv: (ReLU -> dw -> pw -> BN) repetitions
     n_in: int = 0
+    tap: Optional[Tuple[int, int]] = None  # conv: the only non-zero kernel tap (weights sized by in_c)
 
 
 @dataclass
@@ -77,12 +78,15 @@ class GraphSpec:
     def input(self) -> int:
         return self._add("input", [], name="input", out_c=self.in_c)
 
-    def conv(self, x: int, out_c: int, k, s=1, p=0, relu=1, name="") -> int:
+    def conv(self, x: int, out_c: int, k, s=1, p=0, relu=1, name="", pre_relu=0, tap=None) -> int:
+        """conv (+ folded BN) (+ ReLU); pre_relu: ReLU applied to the input
+        first (NASNet's ReLU -> conv -> BN); tap: a single-tap conv (a shifted,
+        strided 1x1 conv: the other taps' weights are zero, workloads/gen.py)."""
         kh, kw = (k, k) if isinstance(k, int) else k
         sh, sw = (s, s) if isinstance(s, int) else s
         ph, pw = (p, p) if isinstance(p, int) else p
         return self._add("conv", [x], name, in_c=self.chan(x), out_c=out_c,
-                         kh=kh, kw=kw, sh=sh, sw=sw, ph=ph, pw=pw, relu=relu)
+                         kh=kh, kw=kw, sh=sh, sw=sw, ph=ph, pw=pw, relu=relu, pre_relu=pre_relu, tap=tap)
 
     def sepconv(self, xs: List[int], out_c: int, k: int, s: int = 1,
                 pre_relu=1, relu=0, agg=None, reps=1, name="") -> int:
@@ -343,18 +347,40 @@ def randwire_ws(h: int = 224, w: Optional[int] = None, c: int = 78) -> GraphSpec
 # ============================================================================
 # NASNet-A large (north star: "NASNet-A large"; P:297 counts 374 ops / 576 deps)
 # ============================================================================
+# Zoph et al. [17] cells as in the public NASNet-A-large (N = 6, penultimate
+# filters 4032, F = 168): every cell input passes ReLU -> 1x1 conv -> BN
+# ("fit"); a previous-cell input at twice the resolution passes the factorized
+# reduction (ReLU -> two stride-2 1x1 convs, the second on the input shifted by
+# one pixel -> concat -> BN); separable branches are (ReLU -> sep kxk -> BN)
+# twice; the network ends ReLU -> GAP -> FC.
 def _nas_sep(g, x, c, k, s, pfx):
     """NASNet separable block: (ReLU -> sep kxk -> BN) twice, the first with
     stride s -- one operator (IOS-style sequential block)."""
     return g.sepconv([x], c, k, s=s, pre_relu=1, reps=2, name=pfx)
 
 
-def _nas_normal(g, h, h_prev, c, pfx):
-    """NASNet-A normal cell (Zoph et al. [17], Fig. 4 left): 5 blocks over
-    (h, h_prev) adjusted to c channels; output = concat of h_prev' and the 5
-    block outputs."""
-    x = g.conv(h, c, 1, relu=0, name=f"{pfx}.fit_h")          # ReLU-1x1-BN on h
-    p = g.conv(h_prev, c, 1, relu=0, name=f"{pfx}.fit_prev")  # and on h_prev
+def _nas_fit(g, x, c, pfx):
+    """ReLU -> 1x1 conv -> BN."""
+    return g.conv(x, c, 1, relu=0, pre_relu=1, name=pfx)
+
+
+def _nas_factorized(g, x, c, pfx):
+    """Factorized reduction of a 2x-resolution input to c channels: path 1 =
+    ReLU -> 1x1 conv stride 2 (pixels 2p, 2q); path 2 = the same on the input
+    shifted by one pixel (pixels 2p+1, 2q+1, zero past the edge) -- a 3x3 /
+    stride 2 / pad 1 conv whose only non-zero tap is (2, 2); concat; the BN is
+    folded into each path's conv (per output channel)."""
+    a = g.conv(x, c // 2, 1, s=2, relu=0, pre_relu=1, name=f"{pfx}.path1")
+    b = g.conv(x, c - c // 2, 3, s=2, p=1, relu=0, pre_relu=1, tap=(2, 2), name=f"{pfx}.path2")
+    return g.concat([a, b], name=f"{pfx}.cat")
+
+
+def _nas_normal(g, h, h_prev, c, pfx, first=False):
+    """NASNet-A normal cell (Fig. 4 left of [17]); FirstCell when h_prev has
+    twice h's resolution (factorized reduction of h_prev).  Output = concat of
+    the adjusted h_prev and the 5 block outputs."""
+    x = _nas_fit(g, h, c, f"{pfx}.fit_h")
+    p = _nas_factorized(g, h_prev, c, f"{pfx}.fact_prev") if first else _nas_fit(g, h_prev, c, f"{pfx}.fit_prev")
     b0 = g.add([_nas_sep(g, x, c, 5, 1, f"{pfx}.b0l"), _nas_sep(g, p, c, 3, 1, f"{pfx}.b0r")],
                name=f"{pfx}.b0")
     b1 = g.add([_nas_sep(g, p, c, 5, 1, f"{pfx}.b1l"), _nas_sep(g, p, c, 3, 1, f"{pfx}.b1r")],
@@ -366,10 +392,9 @@ def _nas_normal(g, h, h_prev, c, pfx):
     return g.concat([p, b0, b1, b2, b3, b4], name=f"{pfx}.concat")
 
 
-def _nas_reduction(g, h, h_prev, c, pfx):
-    """NASNet-A reduction cell (Zoph et al. [17], Fig. 4 right)."""
-    x = g.conv(h, c, 1, relu=0, name=f"{pfx}.fit_h")
-    p = g.conv(h_prev, c, 1, relu=0, name=f"{pfx}.fit_prev")
+def _nas_reduction(g, x, p, c, pfx):
+    """NASNet-A reduction cell (Fig. 4 right of [17]) on the adjusted inputs
+    x (from h) and p (from h_prev)."""
     b0 = g.add([_nas_sep(g, x, c, 5, 2, f"{pfx}.b0l"), _nas_sep(g, p, c, 7, 2, f"{pfx}.b0r")],
                name=f"{pfx}.b0")
     b1 = g.add([g.maxpool(x, 3, 2, 1, name=f"{pfx}.b1l"), _nas_sep(g, p, c, 7, 2, f"{pfx}.b1r")],
@@ -384,40 +409,38 @@ def _nas_reduction(g, h, h_prev, c, pfx):
 
 def nasnet_a_large(h: int = 331, w: Optional[int] = None, n: int = 6, f: int = 168,
                    stem_c: int = 96) -> GraphSpec:
-    """NASNet-A large (N=6 normal cells per stack, F=168): stem conv 3x3 s2,
-    two stem reduction cells, 3 stacks of N normal cells separated by two
-    reduction cells, ReLU -> GAP -> FC.  Spatial shapes follow the cell
-    strides; a strided cell input is brought to the new resolution by a
-    stride-2 1x1 conv (factorized reduction simplified)."""
+    """NASNet-A large (N = 6 normal cells per stack, F = 168): stem conv 3x3 s2
+    (+BN), cell_stem_0 (its second input is the raw stem output, whose
+    separable branches map 96 -> F/4 channels), cell_stem_1 (factorized
+    reduction of the stem output), 3 stacks of N normal cells (the first of
+    each a FirstCell) separated by two reduction cells, ReLU -> GAP -> FC."""
     w = h if w is None else w
     g = GraphSpec(f"nasnet_a_large_{h}", 3, h, w)
     x = g.input()
     stem = g.conv(x, stem_c, 3, s=2, relu=0, name="conv0")
-    # stem cells (reductions at F/4 and F/2 filters)
-    prev, cur = stem, stem
+    # cell_stem_0: x1 = fit(stem); the "left" separable branches read the raw stem
     c = f // 4
-    r = _nas_reduction(g, cur, prev, c, "cell_stem_0")
-    prev, cur = _down(g, cur, g.chan(cur), "cell_stem_0.down"), r
+    cur = _nas_reduction(g, _nas_fit(g, stem, c, "cell_stem_0.fit_h"), stem, c, "cell_stem_0")
+    # cell_stem_1: fit(cell_stem_0), factorized reduction of the stem output
     c = f // 2
-    r = _nas_reduction(g, cur, prev, c, "cell_stem_1")
-    prev, cur = _down(g, cur, g.chan(cur), "cell_stem_1.down"), r
+    nxt = _nas_reduction(g, _nas_fit(g, cur, c, "cell_stem_1.fit_h"), _nas_factorized(g, stem, c, "cell_stem_1.fact_prev"),
+                         c, "cell_stem_1")
+    prev, cur = cur, nxt
     c = f
     for stack in range(3):
         for i in range(n):
-            nxt = _nas_normal(g, cur, prev, c, f"cell_{stack}_{i}")
+            nxt = _nas_normal(g, cur, prev, c, f"cell_{stack}_{i}", first=(i == 0))
             prev, cur = cur, nxt
         if stack < 2:
             c *= 2
-            r = _nas_reduction(g, cur, prev, c, f"reduction_cell_{stack}")
-            prev, cur = _down(g, cur, g.chan(cur), f"reduction_cell_{stack}.down"), r
-    x = g.gap(cur, name="avgpool")
+            r = _nas_reduction(g, _nas_fit(g, cur, c, f"reduction_cell_{stack}.fit_h"),
+                               _nas_fit(g, prev, c, f"reduction_cell_{stack}.fit_prev"), c,
+                               f"reduction_cell_{stack}")
+            prev, cur = cur, r
+    x = g.add([cur], relu=1, name="relu")
+    x = g.gap(x, name="avgpool")
     g.linear(x, 1000, name="last_linear")
     return g
-
-
-def _down(g, x, c, name):
-    """Bring a cell input to half resolution (stride-2 1x1 conv + BN)."""
-    return g.conv(x, c, 1, s=2, relu=0, name=name)
 
 
 BUILDERS = {
