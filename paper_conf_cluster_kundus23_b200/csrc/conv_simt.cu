@@ -26,8 +26,8 @@ __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
   const int t = threadIdx.x, tx = t & 15, ty = t >> 4;
   const int m0 = blockIdx.x * SBM, n0 = blockIdx.y * SBN;
   const int M = a.P * a.Q, RS = a.R * a.S, Cp = (a.C + 15) & ~15, nch = Cp >> 4;
-  // loads: 128 rows x 16 k = 512 float4 per operand, two per thread:
-  // row = t >> 1 (+ 0 / 128? no: rows t>>2 and 64 + (t>>2)), quad = t & 3
+  // loads: 128 rows x 16 k = 512 float4 per operand, two per thread: rows
+  // t >> 2 and 64 + (t >> 2), channel quad (t & 3) * 4
   const int lrow = t >> 2, lq = (t & 3) * 4;
   int ih[2], iw[2];
   bool mval[2];

@@ -4,8 +4,15 @@ on cuda:0 (hios_profile, 5 reps), then HIOS-LP with M = 1, w = 5 through
 hios_run.  The fp64 oracle outputs are cached (tests/golden/oracle_cache/,
 written by tools/make_oracle_cache.py, which calls only oracle/): the logits in
 full, and for six intermediate operators 4096 sampled NCHW elements with the
-whole tensor's max|y|, so each check is the normwise-max metric of SURVEY C22
-restricted to the sample: max_i |y_i - yhat_i| / max_all |yhat| <= 2e-2 (bf16).
+whole tensor's max|y|.  Checks (normwise-max metric of SURVEY C22):
+
+* network output (the logits) vs the cached end-to-end oracle: <= 2e-2 (bf16);
+* each sampled intermediate operator in isolation: the oracle operator
+  (oracle/infer.py run_op) evaluated on the GPU's own inputs of that operator
+  (read back through hios_read_op_output) vs the GPU output: <= 2e-2;
+* the end-to-end drift of those intermediates vs the cached oracle values
+  (bf16 storage of every activation through up to ~370 operators) is reported
+  and bounded by 5e-2.
 """
 import os
 
@@ -43,13 +50,25 @@ def test_bench_config_vs_cached_oracle(model, size):
     h.hios_profile(G, [0], 5)
     S = h.hios_schedule_lp(G, 1, 5)
     y = h.hios_run(S, x)
-    errs = {}
+    from oracle import infer
+    sink = g.sinks()[0]
+    drift, iso = {}, {}
     for v in c["ops"]:
         v = int(v)
         shape = tuple(int(a) for a in c[f"shape_{v}"])
-        yv = y if v == g.sinks()[0] else h.hios_read_op_output(S, v, shape)
-        yv = np.asarray(yv, np.float64).reshape(-1)[c[f"idx_{v}"]]
-        errs[g.ops[v].name] = float(np.abs(yv - c[f"val_{v}"]).max() / float(c[f"absmax_{v}"]))
-    print(model, size, {k: f"{e:.2e}" for k, e in errs.items()})
-    bad = {k: e for k, e in errs.items() if not e <= TOL_BF16}
+        full = np.asarray(y if v == sink else h.hios_read_op_output(S, v, shape), np.float64)
+        yv = full.reshape(-1)[c[f"idx_{v}"]]
+        drift[g.ops[v].name] = float(np.abs(yv - c[f"val_{v}"]).max() / float(c[f"absmax_{v}"]))
+        if v != sink:
+            ins = []
+            for u in g.preds(v):
+                ins.append(np.asarray(h.hios_read_op_output(S, u, tuple(h.hios_graph_shape(G, u))), np.float64))
+            ref = infer.run_op(g.ops[v], ins, W[v]).reshape(-1)
+            iso[g.ops[v].name] = float(np.abs(full.reshape(-1) - ref).max() / float(np.abs(ref).max()))
+    print(model, size, "end-to-end drift", {k: f"{e:.2e}" for k, e in drift.items()},
+          "isolated", {k: f"{e:.2e}" for k, e in iso.items()})
+    assert drift[g.ops[sink].name] <= TOL_BF16, drift
+    bad = {k: e for k, e in iso.items() if not e <= TOL_BF16}
+    assert not bad, bad
+    bad = {k: e for k, e in drift.items() if not e <= 5e-2}
     assert not bad, bad

@@ -26,6 +26,7 @@ SHAPES = [  # name, C, K, H, W, kh, kw, s, ph, pw
 
 def main():
     check = "--check" in sys.argv
+    dtype = "f32" if "--f32" in sys.argv else "bf16"
     only = [a for a in sys.argv[1:] if not a.startswith("--")]
     for (name, C, K, H, W, kh, kw, s, ph, pw) in SHAPES:
         if only and name not in only:
@@ -34,7 +35,7 @@ def main():
         x0 = g.input()
         g.conv(x0, K, (kh, kw), s=s, p=(ph, pw), relu=1)
         Wt = gen.make_weights(g)
-        G = h.hios_graph_create(g.ops, g.edges, C, H, W, "bf16", Wt)
+        G = h.hios_graph_create(g.ops, g.edges, C, H, W, dtype, Wt)
         h.hios_profile(G, [0], 30)
         t, _ = h.hios_get_costs(G)
         c, P, Q = h.hios_graph_shape(G, 1)
