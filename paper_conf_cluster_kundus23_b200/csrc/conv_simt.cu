@@ -17,9 +17,13 @@
 
 namespace hios {
 
-constexpr int SBM = 128, SBN = 128, SBK = 16, SPAD = 4;
+constexpr int SBK = 16, SPAD = 4;
 
+// BT x BT CTA tile (BT = 128: 8 x 8 outputs per thread; BT = 64: 4 x 4, for
+// convs whose 128-tiles would leave most SMs idle -- small spatial extents)
+template <int BT>
 __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
+  constexpr int SBM = BT, SBN = BT, TT = BT / 16, HALF = BT / 2;  // TT outputs per thread per dim
   pdl_enter();
   __shared__ __align__(16) float As[2][SBK][SBM + SPAD];
   __shared__ __align__(16) float Bs[2][SBK][SBN + SPAD];
@@ -28,37 +32,38 @@ __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
   const int M = a.P * a.Q, RS = a.R * a.S, Cp = (a.C + 15) & ~15, nch = Cp >> 4;
   // loads: 128 rows x 16 k = 512 float4 per operand, two per thread: rows
   // t >> 2 and 64 + (t >> 2), channel quad (t & 3) * 4
+  constexpr int NL = BT / 64;  // float4 loads per operand per thread
   const int lrow = t >> 2, lq = (t & 3) * 4;
-  int ih[2], iw[2];
-  bool mval[2];
+  int ih[NL], iw[NL];
+  bool mval[NL];
 #pragma unroll
-  for (int i = 0; i < 2; ++i) {
+  for (int i = 0; i < NL; ++i) {
     const int m = m0 + lrow + 64 * i;
     mval[i] = m < M;
     const int p = mval[i] ? m / a.Q : 0, q = mval[i] ? m - (m / a.Q) * a.Q : 0;
     ih[i] = p * a.sh - a.ph;
     iw[i] = q * a.sw - a.pw;
   }
-  bool nval[2];
-  const float* wrow[2];
+  bool nval[NL];
+  const float* wrow[NL];
 #pragma unroll
-  for (int i = 0; i < 2; ++i) {
+  for (int i = 0; i < NL; ++i) {
     const int n = n0 + lrow + 64 * i;
     nval[i] = n < a.K;
     wrow[i] = a.w + (size_t)(nval[i] ? n : 0) * RS * Cp;
   }
-  float acc[8][8];
+  float acc[TT][TT];
 #pragma unroll
-  for (int i = 0; i < 8; ++i)
+  for (int i = 0; i < TT; ++i)
 #pragma unroll
-    for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+    for (int j = 0; j < TT; ++j) acc[i][j] = 0.f;
 
-  float4 ra[2], rb[2];
+  float4 ra[NL], rb[NL];
   auto gload = [&](int rs, int c0) {
     const int r = rs / a.S, s = rs - r * a.S;  // once per 16-channel chunk
     const int c = c0 + lq;
 #pragma unroll
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < NL; ++i) {
       float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
       const int h = ih[i] + r * a.dh, w = iw[i] + s * a.dw;
       if (mval[i] && h >= 0 && h < a.H && w >= 0 && w < a.W) {
@@ -78,7 +83,7 @@ __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
   };
   auto sstore = [&](int buf) {
 #pragma unroll
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < NL; ++i) {
       const int row = lrow + 64 * i;
       As[buf][lq + 0][row] = ra[i].x;
       As[buf][lq + 1][row] = ra[i].y;
@@ -103,16 +108,18 @@ __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
     }
 #pragma unroll
     for (int kk = 0; kk < SBK; ++kk) {
-      const float4 a0 = *reinterpret_cast<const float4*>(&As[buf][kk][ty * 4]);
-      const float4 a1 = *reinterpret_cast<const float4*>(&As[buf][kk][64 + ty * 4]);
-      const float4 b0 = *reinterpret_cast<const float4*>(&Bs[buf][kk][tx * 4]);
-      const float4 b1 = *reinterpret_cast<const float4*>(&Bs[buf][kk][64 + tx * 4]);
-      const float av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-      const float bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+      float av[TT], bv[TT];
 #pragma unroll
-      for (int i = 0; i < 8; ++i)
+      for (int h = 0; h < TT / 4; ++h) {  // float4 groups at rows h * HALF + ty * 4
+        const float4 a4 = *reinterpret_cast<const float4*>(&As[buf][kk][h * HALF + ty * 4]);
+        const float4 b4 = *reinterpret_cast<const float4*>(&Bs[buf][kk][h * HALF + tx * 4]);
+        av[4 * h] = a4.x; av[4 * h + 1] = a4.y; av[4 * h + 2] = a4.z; av[4 * h + 3] = a4.w;
+        bv[4 * h] = b4.x; bv[4 * h + 1] = b4.y; bv[4 * h + 2] = b4.z; bv[4 * h + 3] = b4.w;
+      }
 #pragma unroll
-        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+      for (int i = 0; i < TT; ++i)
+#pragma unroll
+        for (int j = 0; j < TT; ++j) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
     }
     if (more) {
       sstore(buf ^ 1);
@@ -120,14 +127,14 @@ __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
       buf ^= 1;
     }
   }
-  // epilogue: rows ty*4 + {0..3} and 64 + ty*4 + {0..3}; columns likewise
+  // epilogue: rows (i / 4) * HALF + ty * 4 + i % 4; columns likewise
 #pragma unroll
-  for (int i = 0; i < 8; ++i) {
-    const int m = m0 + (i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4);
+  for (int i = 0; i < TT; ++i) {
+    const int m = m0 + (i / 4) * HALF + ty * 4 + (i % 4);
     if (m >= M) continue;
 #pragma unroll
-    for (int h2 = 0; h2 < 2; ++h2) {
-      const int nb = n0 + h2 * 64 + tx * 4;
+    for (int h2 = 0; h2 < TT / 4; ++h2) {
+      const int nb = n0 + h2 * HALF + tx * 4;
       float y[4];
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
@@ -150,8 +157,15 @@ __global__ void __launch_bounds__(256) conv_simt_kernel(const ConvSimtArgs a) {
 }
 
 void launch_conv_simt(const ConvSimtArgs& a, cudaStream_t st) {
-  dim3 grid((a.P * a.Q + SBM - 1) / SBM, (a.K + SBN - 1) / SBN);
-  launch_pdl(conv_simt_kernel, grid, dim3(256), 0, st, a);
+  const int M = a.P * a.Q;
+  const long long big = (long long)((M + 127) / 128) * ((a.K + 127) / 128);
+  if (big >= 148) {
+    dim3 grid((M + 127) / 128, (a.K + 127) / 128);
+    launch_pdl(conv_simt_kernel<128>, grid, dim3(256), 0, st, a);
+  } else {  // small spatial extent: 64-tiles give 4x the CTAs
+    dim3 grid((M + 63) / 64, (a.K + 63) / 64);
+    launch_pdl(conv_simt_kernel<64>, grid, dim3(256), 0, st, a);
+  }
 }
 
 }  // namespace hios
