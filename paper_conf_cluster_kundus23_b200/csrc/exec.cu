@@ -37,13 +37,12 @@ namespace hios {
 // smem-weight CUDA-core kernel ~380 us (tools/stem_micro.py).  HIOS_NOSTEM3=1
 // restores the s2d path.
 static bool stem3_conv(const Op& o) {
-  static const bool off = getenv("HIOS_NOSTEM3") != nullptr;
-  return !off && o.kind == HIOS_OP_CONV && o.in_c == 3 && o.kh == 3 && o.kw == 3 && o.sh == 2 && o.sw == 2 &&
+  return o.kind == HIOS_OP_CONV && o.in_c == 3 && o.kh == 3 && o.kw == 3 && o.sh == 2 && o.sw == 2 &&
          o.dh == 1 && o.dw == 1 && o.out_c <= kStem3MaxK;
 }
 static bool s2d_conv(const Op& o) {
   return o.kind == HIOS_OP_CONV && !stem3_conv(o) && o.in_c <= 4 && o.sh == 2 && o.sw == 2 && o.dh == 1 && o.dw == 1 &&
-         o.kh * o.kw >= 4 && !getenv("HIOS_NOS2D");
+         o.kh * o.kw >= 4;
 }
 
 
@@ -524,23 +523,11 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     // (measured: sequential Inception-1024 1.077 -> 0.981 ms with 64 for all)
     // (only when 128-wide tiles leave SMs idle)
     int cap = (g_conv_solo && (int64_t)c.tiles_m * ((K + 127) / 128) < g_num_sms) ? 64 : 128;
-    if (getenv("HIOS_TAPCAP")) cap = std::max(16, atoi(getenv("HIOS_TAPCAP")));
     const int nb = (K + cap - 1) / cap;
     c.n_tile = rup((K + nb - 1) / nb, 16);
   }
   c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
   c.n_mma = 1;  // measured: splitting N over several MMA warps does not pay (tools/conv_micro.py)
-  // debug overrides for tuning experiments (tools/conv_micro.py)
-  if (getenv("HIOS_NTILE")) {
-    c.n_tile = std::min(256, rup(atoi(getenv("HIOS_NTILE")), 16));
-    c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
-    c.n_mma = n_mma_of(c.n_tile);
-  }
-  if (getenv("HIOS_NMMA")) {
-    const int want = atoi(getenv("HIOS_NMMA"));
-    c.n_mma = 1;
-    for (int m2 : {4, 2}) if (m2 <= want && c.n_tile % (16 * m2) == 0) { c.n_mma = m2; break; }
-  }
   const size_t B = (size_t)c.n_tile * 128;
   const size_t stage_out = 128 * ((size_t)c.n_tile * 2 + 16);
   // epilogue: two staging tiles for N tiles <= 128 (the stores of tile i
@@ -550,25 +537,25 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   c.occ = 1;
   // epilogue mode (HIOS_EPI overrides): direct register stores for N tiles
   // <= 128 (no staging tile), TMA bulk-tensor stores for wider tiles
-  c.epi = getenv("HIOS_EPI") ? atoi(getenv("HIOS_EPI")) : (c.n_tile <= 128 ? 2 : 1);
-  c.out_bufs = c.epi == 2 ? 0 : ((c.n_tile <= (c.occ == 2 ? 48 : 128) && !getenv("HIOS_OUT1")) ? 2 : 1);
-  c.sres = (c.tiles_n * c.n_tile <= kScaleRes && !getenv("HIOS_NOSRES")) ? 1 : 0;
+  c.epi = c.n_tile <= 128 ? 2 : 1;
+  c.out_bufs = c.epi == 2 ? 0 : (c.n_tile <= (c.occ == 2 ? 48 : 128) ? 2 : 1);
+  c.sres = c.tiles_n * c.n_tile <= kScaleRes ? 1 : 0;
   // occupancy: 1 CTA/SM (212 KB) or 2 CTAs/SM (104 KB each, TMEM <= 256 cols)
   const size_t budget = (c.occ == 2 ? 104 * 1024 : 212 * 1024) - c.out_bufs * stage_out;
   // K-steps per stage: amortise the ~0.3 us full/empty handshake (measured)
-  c.kps = getenv("HIOS_KPS") ? std::max(1, atoi(getenv("HIOS_KPS"))) : 0;
+  c.kps = 0;
   // resident weights (halo mode, one N tile, CTAs that walk several tiles):
   // the whole B is loaded once per CTA instead of once per tile (measured:
   // Conv2d_2a re-read 36 KB of weights per 25 KB input tile)
   const size_t b_all = (size_t)c.c_chunks * R * S * B;
   c.bres = 0;
-  if (c.halo && c.tiles_n == 1 && c.tiles_m > g_num_sms * c.occ && b_all <= 96 * 1024 && !getenv("HIOS_NOBRES") &&
+  if (c.halo && c.tiles_n == 1 && c.tiles_m > g_num_sms * c.occ && b_all <= 96 * 1024 &&
       halo_bytes_of(c.hrows, hw) + b_all <= budget) {
     c.bres = 1;
     c.kps = std::min(4, R * S);
     // as many input boxes in flight as fit (measured: the halo TMA latency,
     // ~2 us, bounds a 2-deep ring at small K; tools/conv_trace2.py)
-    const int cap = getenv("HIOS_ABUFS") ? std::max(1, std::min(kMaxABufs, atoi(getenv("HIOS_ABUFS")))) : kMaxABufs;
+    const int cap = kMaxABufs;
     c.a_bufs = 1;
     while (c.a_bufs < cap && (c.a_bufs + 1) * halo_bytes_of(c.hrows, hw) + b_all <= budget) ++c.a_bufs;
     c.stages = 2;
@@ -579,7 +566,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     while (c.kps > 1 && H + 2 * c.kps * B > budget) --c.kps;
     c.a_bufs = (2 * H + 2 * c.kps * B <= budget) ? 2 : 1;
     {  // deeper input ring while >= 4 B stages still fit
-      const int cap = getenv("HIOS_ABUFS") ? std::max(1, std::min(kMaxABufs, atoi(getenv("HIOS_ABUFS")))) : 4;
+      const int cap = 4;
       while (c.a_bufs < cap && (c.a_bufs + 1) * H + 4 * c.kps * B <= budget) ++c.a_bufs;
     }
     if (H + 2 * c.kps * B > budget) fail(HIOS_E_UNSUPPORTED, "conv halo plan does not fit shared memory");
@@ -606,7 +593,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     // at most one wave of CTAs, >= ~6 K-steps each; splits may start at any
     // (chunk, tap) K-step
     const int cta_cap = g_num_sms;
-    static const int min_k = getenv("HIOS_SPLIT_MINK") ? std::max(1, atoi(getenv("HIOS_SPLIT_MINK"))) : 6;
+    const int min_k = 6;
     int want = std::max(1, (cta_cap * c.occ) / tiles);
     want = std::min(want, KI / min_k);
     if (want >= 2) {
@@ -614,7 +601,6 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
       c.ksplit = (KI + c.kpsplit - 1) / c.kpsplit;
     }
   }
-  if (getenv("HIOS_STAGES")) c.stages = std::max(2, atoi(getenv("HIOS_STAGES")));
   return c;
 }
 
@@ -659,8 +645,7 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   // ~16 B/cycle/SM whatever the number of issuing warps, 2-7x slower than an
   // in-bounds box.  Those channels meet zero weights (pitch rup(C, 64)) or are
   // skipped (K=16 slices past C are not issued).
-  static const bool nopad = getenv("HIOS_NOCHANPAD") != nullptr;
-  const int Cm = (C % 64 && !nopad) ? rup(C, 64) : C;
+  const int Cm = C % 64 ? rup(C, 64) : C;
   if (a.vgrid)  // hrows whole padded input rows (x from -pw) per channel chunk
     ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w,
                       a.hrows, 1, 1);
@@ -676,10 +661,10 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
     fail(HIOS_E_CUDA, "tensor map (weights)");
   a.P = P; a.Q = Q; a.K = K; a.C = C; a.R = R; a.S = S; a.sh = sh; a.sw = sw; a.ph = ph; a.pw = pw;
   a.dh = dh; a.dw = dw; a.relu = relu; a.scale = scale; a.shift = shift;
-  a.bo_mode = getenv("HIOS_BO") ? atoi(getenv("HIOS_BO")) : 0;
-  a.trace = getenv("HIOS_TRACE") ? 1 : 0;
-  a.spin = getenv("HIOS_SPIN") ? atoi(getenv("HIOS_SPIN")) : 0;
-  a.dbg = getenv("HIOS_DBG") ? atoi(getenv("HIOS_DBG")) : 0;
+  a.bo_mode = 0;
+  a.trace = getenv("HIOS_TRACE") ? 1 : 0;  // per-CTA globaltimer timeline (tools/conv_trace.py)
+  a.spin = 0;
+  a.dbg = 0;
   a.out = (bf16*)out.p; a.ldo = out.ldc;
   a.out2 = dst_of<bf16>(out2);
   // epilogue by TMA bulk-tensor stores: output tensor map {K, Q, P} over the
@@ -687,7 +672,7 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   CUtensorMap mo = mx, mo2 = mx;
   a.out_sw = a.n_tile % 64 == 0 ? 64 : (a.n_tile % 32 == 0 ? 32 : 16);
   if (a.vgrid && a.epi == 1) a.epi = 0;  // tiles are not rectangular: no TMA-store boxes
-  a.tma_out = !getenv("HIOS_NOTMASTORE") && a.ksplit == 1 && a.epi == 1 ? 1 : 0;
+  a.tma_out = a.ksplit == 1 && a.epi == 1 ? 1 : 0;
   if (a.ksplit > 1 || (a.epi == 1 && !a.tma_out)) a.epi = 0;
   if (a.tma_out) {
     const int sb = a.out_sw * 2;
@@ -814,8 +799,7 @@ static void build_op(Executor& ex, int v) {
         S2dArgs<T> d{(const T*)iv.p, xi.H, xi.W, xi.C, iv.ldc, o.ph, o.pw, (T*)sv.p, H2, W2, sv.ldc};
         fns.push_back([d](cudaStream_t st) { launch_s2d<T>(d, st); });
         ++nk;
-        static const bool nopack = getenv("HIOS_NOPACK") != nullptr;
-        if (x.w_pack && !nopack) {
+        if (x.w_pack) {
           // packed taps: a virtual 64-channel input whose pixel j is the
           // 4-pixel window j..j+3 of the s2d tensor (pixel stride 32 B)
           View pv{sv.p, sv.ldc, W2};
@@ -975,7 +959,6 @@ static void build_op(Executor& ex, int v) {
 }
 
 void Executor::build_closures() {
-  static const bool nosolo = getenv("HIOS_NOSOLO") != nullptr;
   for (int v = 0; v < g.n; ++v) {
     const int l = s.gpu_of[v];
     if (!lg[l].local) continue;
@@ -986,7 +969,7 @@ void Executor::build_closures() {
     else build_op<float>(*this, v);
     OpExec& x = ox[v];
     const int k = g.ops[v].kind;
-    if (g.dtype == HIOS_BF16 && !nosolo && (k == HIOS_OP_CONV || k == HIOS_OP_SEPCONV)) {
+    if (g.dtype == HIOS_BF16 && (k == HIOS_OP_CONV || k == HIOS_OP_SEPCONV)) {
       auto run = x.run;
       const int nk = x.n_kernels;
       g_conv_solo = true;

@@ -15,15 +15,12 @@ namespace hios {
 
 typedef __nv_bfloat16 bf16;
 
-// Programmatic dependent launch (PDL) for the memory-bound kernels: launched
-// with programmatic stream serialisation, a kernel's launch and prologue
-// overlap the tail of its predecessor in the stream (CUDA graphs keep these as
-// programmatic edges).  pdl_enter() = wait until the predecessor grid has
-// completed and flushed (before reading any activation), then let our own
-// dependents start launching; it is a no-op for a normal launch.  Measured on
-// Inception-v3 1024 under HIOS w=4: PDL on these kernels LOSES ~2.5 % (their
-// early-resident CTAs compete with the concurrent stages), so it is off unless
-// HIOS_PDL_MISC=1; the tcgen05 conv keeps PDL (its prologue is long).
+// Memory-bound kernels are launched WITHOUT programmatic dependent launch:
+// measured on Inception-v3 1024 under HIOS w=4, PDL on these kernels LOSES
+// ~2.5 % (their early-resident CTAs compete with the concurrent stages); the
+// tcgen05 conv keeps PDL (its prologue is long).  pdl_enter() (wait for the
+// predecessor grid, then let dependents launch) is a no-op for a normal
+// launch, so the kernels stay correct under either launch mode.
 __device__ __forceinline__ void pdl_enter() {
   asm volatile("griddepcontrol.wait;" ::: "memory");
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
@@ -40,8 +37,7 @@ inline cudaError_t launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  static const bool on = getenv("HIOS_PDL_MISC") != nullptr;  // measurement switch
-  cfg.numAttrs = on ? 1 : 0;
+  cfg.numAttrs = 0;  // see above: measured faster without PDL
   return cudaLaunchKernelEx(&cfg, k, std::forward<Args>(args)...);
 }
 

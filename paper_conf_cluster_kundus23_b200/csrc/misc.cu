@@ -448,117 +448,33 @@ static void launch_pool_tiled(const PoolArgs<T>& a, size_t smem, cudaStream_t st
   launch_pdl(pool_tiled_kernel<T, KS>, grid, dim3(256), smem, st, a);
 }
 
-// Row-streaming 3x3 pooling (stride SS = 1 or 2): a thread owns one output
-// column x one 16-byte channel vector and walks a strip of TP output rows
-// down the image, keeping the horizontal 3-tap reductions of the last three
-// input rows in registers, so every input row is read from HBM once per
-// strip (the horizontal neighbours come from L1: adjacent columns are
-// adjacent threads of the same warp) and each output vector is written once,
-// coalesced -- (1 + 2/TP) x input + 1 x output bytes per launch.
-template <typename T, int SS>
-__global__ void __launch_bounds__(256) pool_rows_kernel(const PoolArgs<T> a, int TP) {
-  pdl_enter();
-  constexpr int N = Vec<T>::N;
-  const int CG = (a.C + N - 1) / N;
-  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= (long long)a.Q * CG) return;
-  const int q = (int)(idx / CG), cg = (int)(idx - (long long)q * CG), c = cg * N;
-  const int p0 = blockIdx.y * TP, p1 = min(a.P, p0 + TP);
-  const int w0 = q * SS - a.pw;
-  const bool is_max = a.is_max != 0;
-  const float pad = is_max ? -INFINITY : 0.f;
-  auto hrow = [&](int h, float* o) {
-#pragma unroll
-    for (int j = 0; j < N; ++j) o[j] = pad;
-    if (h < 0 || h >= a.H) return;
-    const T* rp = a.x + (size_t)h * a.W * a.ldx + c;
-#pragma unroll
-    for (int s = 0; s < 3; ++s) {
-      const int w = w0 + s;
-      if (w < 0 || w >= a.W) continue;
-      float v[N];
-      load_vec(rp + (size_t)w * a.ldx, c, a.C, v);
-#pragma unroll
-      for (int j = 0; j < N; ++j) o[j] = is_max ? fmaxf(o[j], v[j]) : o[j] + v[j];
-    }
-  };
-  float r0[N], r1[N], r2[N];
-  int h = p0 * SS - a.ph;
-  hrow(h, r0);
-  hrow(h + 1, r1);
-  hrow(h + 2, r2);
-  const int wlo = max(w0, 0), whi = min(w0 + 3, a.W);
-  for (int p = p0; p < p1; ++p) {
-    float acc[N];
-#pragma unroll
-    for (int j = 0; j < N; ++j)
-      acc[j] = is_max ? fmaxf(fmaxf(r0[j], r1[j]), r2[j]) : r0[j] + r1[j] + r2[j];
-    if (!is_max) {
-      int div;
-      if (a.cip) div = (min(h + 3, a.H + a.ph) - h) * (min(w0 + 3, a.W + a.pw) - w0);
-      else div = (min(h + 3, a.H) - max(h, 0)) * (whi - wlo);
-      const float inv = 1.f / (float)div;
-#pragma unroll
-      for (int j = 0; j < N; ++j) acc[j] *= inv;
-    }
-    if (p + 1 < p1) {  // next rows' loads issued ahead of this row's store
-      if (SS == 1) {
-#pragma unroll
-        for (int j = 0; j < N; ++j) { r0[j] = r1[j]; r1[j] = r2[j]; }
-        hrow(h + 3, r2);
-      } else {
-#pragma unroll
-        for (int j = 0; j < N; ++j) r0[j] = r2[j];
-        hrow(h + 3, r1);
-        hrow(h + 4, r2);
-      }
-    }
-    const size_t pix = (size_t)p * a.Q + q;
-    store_vec(a.out + pix * a.ldo + c, c, a.C, acc);
-    for (int d_ = 0; d_ < a.out2.n; ++d_) store_vec(a.out2.p[d_] + pix * a.out2.ld[d_] + c, c, a.C, acc);
-    h += SS;
-  }
-}
-
 template <typename T>
 void launch_pool(const PoolArgs<T>& a, cudaStream_t st) {
   constexpr int N = Vec<T>::N;
-  if (a.kh == 3 && a.kw == 3 && a.sh == a.sw && (a.sh == 1 || a.sh == 2) && getenv("HIOS_POOL_ROWS")) {
-    // strip height: >= ~2 waves of 2048-thread SMs, at most 16 rows
-    const long long cols = (long long)a.Q * ((a.C + N - 1) / N);
-    const int TP = (int)std::max(1LL, std::min(16LL, cols * a.P / (148LL * 2048 * 2)));
-    dim3 grid(grid_for(cols, 256), (a.P + TP - 1) / TP);
-    if (a.sh == 1) launch_pdl(pool_rows_kernel<T, 1>, grid, dim3(256), 0, st, a, TP);
-    else launch_pdl(pool_rows_kernel<T, 2>, grid, dim3(256), 0, st, a, TP);
-    return;
-  }
   const size_t smem = (size_t)2 * ((kPoolTP - 1) * a.sh + a.kh) * ((kPoolTQ - 1) * a.sw + a.kw) * 8 * sizeof(T);
   // measured (tools/op_micro.py, B200): tiled 3x3/s1 avgpool 139 us vs 187 us
   // direct; 3x3/s2 maxpool 297 us vs 205 us direct -- stride 1 only
   // bf16 3x3: the direct kernel with all tap loads in flight (measured faster
-  // than the smem-tiled kernel; HIOS_POOL_TILED3 keeps the tiled one)
-  // measured: direct wins for stride 2 and for small stride-1 pools (Mixed_6/7
-  // at 1024^2), the tiled kernel for large stride-1 average pools
-  static const bool tiled3 = getenv("HIOS_POOL_TILED3") != nullptr;
+  // than the smem-tiled kernel); direct wins for stride 2 and for small
+  // stride-1 pools (Mixed_6/7 at 1024^2), the tiled kernel for large stride-1
+  // average pools.  (A row-streaming kernel measured slower on every shape and
+  // was removed, round 2.)
   const bool big_s1 = a.sh == 1 && (long long)a.P * a.Q * a.C >= (4LL << 20);
-  static const bool no64 = getenv("HIOS_POOL_NO64") != nullptr;
   if constexpr (std::is_same<T, bf16>::value) {
     // large stride-1 3x3 average pools with whole 8-channel vectors: 64-channel CTAs
-    if (big_s1 && !a.is_max && a.kh == 3 && a.kw == 3 && a.sw == 1 && a.C % 8 == 0 && !no64 && !tiled3) {
+    if (big_s1 && !a.is_max && a.kh == 3 && a.kw == 3 && a.sw == 1 && a.C % 8 == 0) {
       dim3 grid((a.C + 63) / 64, (a.Q + kP64TQ - 1) / kP64TQ, (a.P + kP64TP - 1) / kP64TP);
       launch_pdl(pool_avg64_kernel, grid, dim3(256), 0, st, a);
       return;
     }
   }
-  if (std::is_same<T, bf16>::value && a.kh == 3 && a.kw == 3 && !tiled3 && !big_s1) {
+  if (std::is_same<T, bf16>::value && a.kh == 3 && a.kw == 3 && !big_s1) {
     const int per_row = a.Q * ((a.C + N - 1) / N);
     dim3 grid((per_row + 255) / 256, a.P);
     launch_pdl(pool_kernel<T, 3, 3>, grid, dim3(256), 0, st, a);
     return;
   }
-  static const bool s2_tiled = getenv("HIOS_POOL_S2TILED") != nullptr;
-  if (((a.sw == 1 && a.sh == 1) || (s2_tiled && a.sw == 2 && a.sh == 2)) && a.kh * a.kw > 1 && smem <= 200 * 1024 &&
-      !getenv("HIOS_POOL_OLD")) {
+  if (a.sw == 1 && a.sh == 1 && a.kh * a.kw > 1 && smem <= 200 * 1024) {
     if (a.kh == 3 && a.kw == 3) return launch_pool_tiled<T, 3>(a, smem, st);
     return launch_pool_tiled<T, 0>(a, smem, st);
   }
@@ -868,8 +784,7 @@ template <typename T>
 static bool try_dw_reg(const DwArgs<T>&, cudaStream_t) { return false; }
 template <>
 bool try_dw_reg<bf16>(const DwArgs<bf16>& a, cudaStream_t st) {
-  static const bool off = getenv("HIOS_DW_NOREG") != nullptr;
-  if (off || a.R != a.S || a.sh != a.sw || (a.sh != 1 && a.sh != 2)) return false;
+  if (a.R != a.S || a.sh != a.sw || (a.sh != 1 && a.sh != 2)) return false;
   if (a.sh == 1) {
     if (a.R == 3) { launch_dw_reg<3, 1, 4>(a, st); return true; }
     if (a.R == 5) { launch_dw_reg<5, 1, 4>(a, st); return true; }
@@ -901,7 +816,7 @@ void launch_dw(const DwArgs<T>& a, cudaStream_t st) {
   const size_t smem = (size_t)a.R * a.S * 16 * sizeof(float) +
                       (size_t)2 * dw_tile_rows(a.R, a.sh) * dw_tile_cols(a.S, a.sw) * 8 * sizeof(T);
   if (try_dw_reg(a, st)) return;
-  if ((a.sw == 1 || a.sw == 2) && smem <= 200 * 1024 && !getenv("HIOS_DW_OLD")) {
+  if ((a.sw == 1 || a.sw == 2) && smem <= 200 * 1024) {
     if (a.R == 3 && a.S == 3) return launch_dw_tiled<T, 3>(a, smem, st);
     if (a.R == 5 && a.S == 5) return launch_dw_tiled<T, 5>(a, smem, st);
     if (a.R == 7 && a.S == 7) return launch_dw_tiled<T, 7>(a, smem, st);

@@ -1,7 +1,7 @@
 """Time single conv ops through the C-ABI (hios_profile's median of reps =
 back-to-back launches of the op's kernel) for a list of Inception-1024 shapes;
-optional parity check vs the oracle.  Env overrides (HIOS_NTILE, HIOS_STAGES,
-HIOS_NOHALO, HIOS_BO) select kernel variants."""
+optional parity check vs the oracle (--check), fp32 path (--f32).  Kernel
+variants are compared as separate builds (tools/build_variant.sh, HIOS_LIB)."""
 import os
 import sys
 

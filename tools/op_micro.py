@@ -1,7 +1,7 @@
 """Time single ops through the C-ABI (hios_profile: median of back-to-back
 in-graph replays of the op's kernels) for the heaviest shapes of the benchmark
 DAGs (gpurun_out/ops_*.json); env switches (HIOS_POOL_OLD, HIOS_DW_OLD,
-HIOS_NOS2D, ...) select kernel variants for A/B runs.
+...; A/B variants are separate builds, HIOS_LIB=ab/libhios_<name>.so) select kernel variants.
 
 usage: python tools/op_micro.py [name ...]
 """
