@@ -1,8 +1,8 @@
 """Time the stride-2 small-C stem convs (Inception/RandWire 3x3 3->32,
 SqueezeNet 7x7 3->96) alone through the C-ABI (hios_profile's t(v), which
 includes the s2d staging kernel when the s2d path is taken); --check adds
-parity vs the oracle.  (A/B against another build: HIOS_LIB=ab/libhios_<name>.so,
-the tensor-core s2d path with the direct CUDA-core kernel."""
+parity vs the oracle.  Compare the tensor-core s2d path with the direct
+CUDA-core kernel as two builds (tools/build_variant.sh, HIOS_LIB=ab/libhios_<name>.so)."""
 import os
 import sys
 
