@@ -21,6 +21,13 @@ SHAPES = [  # name, C, K, H, W, kh, kw, s, ph, pw
     ("6e_1x7", 192, 192, 62, 62, 1, 7, 1, 0, 3),
     ("7c_1x1", 2048, 384, 30, 30, 1, 1, 1, 0, 0),
     ("7c_3x3", 448, 384, 30, 30, 3, 3, 1, 1, 1),
+    # Inception-v3 at 4096^2 (compute-heavy)
+    ("4a_4096", 80, 192, 1022, 1022, 3, 3, 1, 0, 0),
+    ("2a_4096", 32, 32, 2047, 2047, 3, 3, 1, 0, 0),
+    ("2b_4096", 32, 64, 2045, 2045, 3, 3, 1, 1, 1),
+    ("5b5x5_4096", 48, 64, 509, 509, 5, 5, 1, 2, 2),
+    ("7c1x1_4096", 2048, 448, 126, 126, 1, 1, 1, 0, 0),
+    ("7b3x3_4096", 448, 384, 126, 126, 3, 3, 1, 1, 1),
 ]
 
 
