@@ -386,7 +386,7 @@ def measure_workload(h, torch, model, sz, M, args, dev, stream, flush, pk, dtype
             # exact single-GPU DP, state budget bounded so the lazily
             # profiled t(S) stay within the bench's time (NASNet: see DESIGN)
             try:
-                Sx = h.hios_schedule_ios(Gs, w_, 1 << 14)
+                Sx = h.hios_schedule_ios(Gs, w_, args.ios_states)
             except h.HiosError as ex:
                 row["ios_unavailable"] = str(ex)
                 continue
@@ -449,6 +449,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--sweep", default="2048,4096,randwire_ws@2048,nasnet_a_large@2048,squeezenet@2048,4096:f32",
                     help="extra input sizes timed on 1 GPU (HIOS-LP / sequential / IOS-style), '' to skip")
+    ap.add_argument("--ios-states", type=int, default=1 << 14,
+                    help="state budget of the exact IOS DP in the size sweep (its t(S) are profiled lazily: "
+                         "NASNet-A 2048^2 needs 2^18, ~5 min)")
     ap.add_argument("--logical", type=int, default=0,
                     help="single process: schedule over this many logical GPUs (aliased on visible devices)")
     args = ap.parse_args()

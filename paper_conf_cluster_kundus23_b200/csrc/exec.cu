@@ -739,6 +739,7 @@ static void build_op(Executor& ex, int v) {
   std::vector<View> out2;
   for (auto& r : x.remote)
     if (r.mode == DM_FUSED) out2.push_back(view_of(v, r.gpu));
+  if (x.probe_out) out2.push_back(View{x.probe_out, x.probe_ldc});  // profiler: C15 edge probe
   std::vector<std::function<void(cudaStream_t)>> fns;
   int nk = 0;
   switch (o.kind) {
@@ -958,29 +959,35 @@ static void build_op(Executor& ex, int v) {
   x.n_kernels = nk;
 }
 
-void Executor::build_closures() {
-  for (int v = 0; v < g.n; ++v) {
-    const int l = s.gpu_of[v];
-    if (!lg[l].local) continue;
-    ck(cudaSetDevice(lg[l].dev), "cudaSetDevice");
-    cur_lgpu = l;
-    g_num_sms = lg[l].num_sms;
-    if (g.dtype == HIOS_BF16) build_op<bf16>(*this, v);
-    else build_op<float>(*this, v);
-    OpExec& x = ox[v];
-    const int k = g.ops[v].kind;
-    if (g.dtype == HIOS_BF16 && (k == HIOS_OP_CONV || k == HIOS_OP_SEPCONV)) {
-      auto run = x.run;
-      const int nk = x.n_kernels;
-      g_conv_solo = true;
-      build_op<bf16>(*this, v);
-      g_conv_solo = false;
-      x.run_solo = x.run;
-      x.n_kernels_solo = x.n_kernels;
-      x.run = run;
-      x.n_kernels = nk;
-    }
+void Executor::build_op_closures(int v) {
+  const int l = s.gpu_of[v];
+  ck(cudaSetDevice(lg[l].dev), "cudaSetDevice");
+  cur_lgpu = l;
+  g_num_sms = lg[l].num_sms;
+  if (g.dtype == HIOS_BF16) build_op<bf16>(*this, v);
+  else build_op<float>(*this, v);
+  OpExec& x = ox[v];
+  const int k = g.ops[v].kind;
+  if (g.dtype == HIOS_BF16 && (k == HIOS_OP_CONV || k == HIOS_OP_SEPCONV)) {
+    auto run = x.run;
+    const int nk = x.n_kernels;
+    auto tc = x.tc;
+    const size_t tcs = x.tc_smem;
+    g_conv_solo = true;
+    build_op<bf16>(*this, v);
+    g_conv_solo = false;
+    x.run_solo = x.run;
+    x.n_kernels_solo = x.n_kernels;
+    x.run = run;
+    x.n_kernels = nk;
+    x.tc = tc;
+    x.tc_smem = tcs;
   }
+}
+
+void Executor::build_closures() {
+  for (int v = 0; v < g.n; ++v)
+    if (lg[s.gpu_of[v]].local) build_op_closures(v);
 }
 
 // deliveries of op u's output to other logical GPUs: push (unless fused) + flag release

@@ -68,6 +68,9 @@ struct OpExec {
   // the stage's grouped launch (conv_tc_group_kernel); empty otherwise
   std::vector<ConvTcOp> tc;
   size_t tc_smem = 0;
+  // profiler only: one extra epilogue destination (the t(u, v) probe of C15)
+  char* probe_out = nullptr;
+  int probe_ldc = 0;
 };
 
 struct LGpu {
@@ -126,6 +129,7 @@ struct Executor {
   void plan();             // locations, flags (host only)
   void allocate();         // arenas, sync words, weights (local lgpus)
   void build_closures();   // per-op kernel launchers
+  void build_op_closures(int v);  // op v's launchers (group and solo configs)
   void capture();          // per-lgpu CUDA graphs
   void run_device(const void* d_in, void* d_out, cudaStream_t user, bool timed);
   char* ptr(int lgpu, int64_t off) const { return lg[lgpu].arena + off; }

@@ -4,9 +4,11 @@
 // each possible data transfer between GPUs ...").
 //
 //   t(v)    median of `reps` CUDA-event timings of op v's kernels alone
-//   t(u,v)  median time of pushing u's output tensor into another GPU's buffer
-//           with the peer-store copy kernel, plus one flag release/acquire pair
-//           (the executor's transfer path); same for every edge leaving u
+//   t(u,v)  SURVEY C15: for ops whose epilogue stores straight into the
+//           consumer GPU's buffer (conv / sepconv / pools / add), the
+//           incremental cost of that extra destination, t(u fused) - t(u);
+//           for the others the time of the peer-store push kernel; plus one
+//           flag release/acquire pair; the same for every edge leaving u
 //   t(S)    measured on demand (Profiler::measure_group): the ops of S forked
 //           onto |S| streams from one event and joined, median of reps
 #include <algorithm>
@@ -155,6 +157,22 @@ std::shared_ptr<Profiler> run_profile(std::shared_ptr<Graph> G, const int32_t* d
     if (g.ops[u].out_edges.empty()) continue;
     const Op& o = g.ops[u];
     const Loc& lc = E.loc[u][0];
+    // C15: ops whose epilogue can store straight into the consumer GPU's
+    // buffer (conv / sepconv / pools / add) pay only the INCREMENTAL cost of
+    // that extra destination: t(u with the remote store) - t(u), >= 0
+    const bool fusable = o.kind == HIOS_OP_CONV || o.kind == HIOS_OP_SEPCONV || o.kind == HIOS_OP_MAXPOOL ||
+                         o.kind == HIOS_OP_AVGPOOL || o.kind == HIOS_OP_ADD;
+    if (fusable && u != g.input_op) {
+      OpExec& x = E.ox[u];
+      x.probe_out = (char*)dst;
+      x.probe_ldc = (o.C + 7) / 8 * 8;
+      E.build_op_closures(u);
+      const int64_t t_fused = impl->time_ns(x.run_solo ? x.run_solo : x.run, st);
+      x.probe_out = nullptr;
+      E.build_op_closures(u);
+      push[u] = std::max<int64_t>(0, t_fused - g.ops[u].cost);
+      continue;
+    }
     std::function<void(cudaStream_t)> f;
     if (g.dtype == HIOS_BF16) {
       CopyArgs<bf16> c{(const bf16*)E.ptr(0, lc.off), lc.ldc, o.H * o.W, o.C, (bf16*)dst, (o.C + 7) / 8 * 8};
