@@ -264,7 +264,8 @@ hios_status hios_schedule_nccl_init(hios_schedule s, const void* id128, int32_t 
 hios_status hios_schedule_transfers(hios_schedule s, int32_t* src_op, int32_t* dst_gpu, int32_t cap, int32_t* n);
 
 /* Multi-process execution (one process per GPU): this process executes only
- * the logical GPUs i with owner[i] == rank.  Cross-process edges use CUDA IPC
+ * the logical GPUs i with owner[i] == rank (all of them placed on one device;
+ * hios_ipc_import rejects a rank spanning several devices, HIOS_E_UNSUPPORTED).  Cross-process edges use CUDA IPC
  * peer memory: after hios_ipc_export on every rank, each rank imports every
  * other rank's blob.  blob is caller-owned; *len in: capacity, out: size. */
 hios_status hios_schedule_bind_rank(hios_schedule s, const int32_t* owner, int32_t n, int32_t rank);

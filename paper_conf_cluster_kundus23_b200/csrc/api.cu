@@ -384,10 +384,16 @@ hios_status hios_ipc_import(hios_schedule s, int32_t rank, const void* blob, siz
       NEED(!s->s->owner.empty() && s->s->owner[l] == rank, HIOS_E_INVALID, "blob GPU not owned by rank");
       auto& L = E.lg[l];
       if (L.local || L.ipc_mapped) continue;
-      // map on every local device (the mapping is per device context)
+      // the mapping is made in the context of this rank's device: rank mode
+      // supports one device per rank (its logical GPUs may alias it), so the
+      // pointer is valid for every local kernel
       int dev = -1;
       for (auto& x : E.lg)
-        if (x.local) { dev = x.dev; break; }
+        if (x.local) {
+          NEED(dev < 0 || dev == x.dev, HIOS_E_UNSUPPORTED,
+               "rank mode: a rank's logical GPUs must share one device (IPC maps are per device)");
+          dev = x.dev;
+        }
       NEED(dev >= 0, HIOS_E_STATE, "no local GPU");
       hios::ck(cudaSetDevice(dev), "cudaSetDevice");
       void* a = nullptr;
