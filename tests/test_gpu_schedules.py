@@ -160,3 +160,26 @@ def test_grouped_stage_kernel_bit_identical(name, size):
         y2 = h.hios_run(S2, x)
         assert np.array_equal(y1, y2), (M, w)
         assert h.hios_kernel_count(S2) <= h.hios_kernel_count(S1)
+
+
+def test_time_ops_and_option_state_rules():
+    """hios_time_ops (bench.py's roofline source): a positive time for every
+    op with kernels, -1 for the input placeholder and zero-copy concats; the
+    schedule options are rejected after the first run (HIOS_E_STATE)."""
+    h = hios()
+    g = graphs.inception_v3(299)
+    W = gen.make_weights(g)
+    G = h.hios_graph_create(g.ops, g.edges, g.in_c, g.in_h, g.in_w, "bf16", W)
+    h.hios_profile(G, [0], 3)
+    S = h.hios_schedule_lp(G, 1, 3)
+    t = h.hios_time_ops(S, 3, 64 << 20)
+    for op in g.ops:
+        if op.kind in ("input", "concat"):
+            assert t[op.id] == -1, op.name
+        else:
+            assert 0 < t[op.id] < 10_000_000, (op.name, t[op.id])
+    h.hios_run(S, gen.make_input(g))
+    for fn, arg in ((h.hios_schedule_transport, "copy"), (h.hios_schedule_stage_mode, "grouped")):
+        with pytest.raises(h.HiosError) as ei:
+            fn(S, arg)
+        assert ei.value.code == 8
