@@ -449,6 +449,10 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--sweep", default="2048,4096,randwire_ws@2048,nasnet_a_large@2048,squeezenet@2048,4096:f32",
                     help="extra input sizes timed on 1 GPU (HIOS-LP / sequential / IOS-style), '' to skip")
+    ap.add_argument("--transport", default="peer", choices=["peer", "copy", "nccl"],
+                    help="cross-GPU edge transport (N > 1): fused peer stores, copy engine, NCCL send/recv")
+    ap.add_argument("--stage-mode", default="streams", choices=["streams", "grouped"],
+                    help="stage execution: per-op streams, or one grouped conv launch per stage (f2)")
     ap.add_argument("--ios-states", type=int, default=1 << 14,
                     help="state budget of the exact IOS DP in the size sweep (its t(S) are profiled lazily: "
                          "NASNet-A 2048^2 needs 2^18, ~5 min)")
@@ -515,7 +519,11 @@ def main():
     t_sched = time.perf_counter() - t0
     if world > 1:
         S = share_schedule(h, dist, G, g, S, M, args.window, rank)
-        bind_and_exchange(h, dist, S, M, world, rank, dev)
+    h.hios_schedule_transport(S, args.transport)
+    h.hios_schedule_stage_mode(S, args.stage_mode)
+    cfg["transport"], cfg["stage_mode"] = args.transport, args.stage_mode
+    if world > 1:
+        bind_and_exchange(h, dist, S, M, world, rank, dev, transport=args.transport)
     elif M > 1:
         ndev = torch.cuda.device_count()
         h.hios_schedule_place(S, [i % ndev for i in range(M)])
