@@ -107,6 +107,11 @@ CONV_CASES = [
     (24, 40, 33, 35, 3, 3, 2, 1, 1),      # tap mode, stride 2, C = 24
     (32, 96, 30, 30, 3, 3, 1, 1, 1),      # vgrid
     (32, 64, 50, 50, 1, 1, 1, 0, 0),      # tap 1x1
+    # C <= 32 (the box reads past C into zero weights) in halo / tap / vgrid modes
+    (16, 48, 40, 300, 3, 3, 1, 1, 1),
+    (24, 40, 33, 35, 3, 3, 2, 1, 1),
+    (32, 96, 30, 30, 3, 3, 1, 1, 1),
+    (32, 64, 50, 50, 1, 1, 1, 0, 0),
     # halo mode with resident weights (one N tile, > 148 output tiles per CTA wave)
     (32, 32, 160, 200, 3, 3, 1, 1, 1),
     (64, 80, 150, 130, 1, 1, 1, 0, 0),
