@@ -149,22 +149,6 @@ __device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr, int bo_mode 
   return d;
 }
 
-// the same for an A operand with 64-byte rows (32 channels, SWIZZLE_64B):
-// 8-row atoms 512 B apart
-__device__ __forceinline__ uint64_t umma_desc_sw64(uint32_t saddr) {
-  uint64_t d = 0;
-  d |= (uint64_t)((saddr & 0x3FFFFu) >> 4);        // start address
-  d |= (uint64_t)1 << 16;                          // LBO (unused for swizzled K-major)
-  d |= (uint64_t)(512 >> 4) << 32;                 // SBO = 512 B
-  d |= (uint64_t)1 << 46;                          // descriptor version (sm_100)
-  d |= (uint64_t)4 << 61;                          // SWIZZLE_64B
-  return d;
-}
-__device__ __forceinline__ uint64_t umma_desc_a(uint32_t saddr, int a_row) {
-  return a_row == 64 ? umma_desc_sw64(saddr) : umma_desc_sw128(saddr);
-}
-
-
 __device__ __forceinline__ void mma_bf16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
   asm volatile(
       "{\n"
@@ -349,9 +333,9 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int ST = a.stages;
-  const uint32_t A_BYTES = 128u * (uint32_t)a.a_row;
+  const uint32_t A_BYTES = 128 * 128;
   const uint32_t B_BYTES = (uint32_t)a.n_tile * 128;
-  const uint32_t H_BYTES = a.halo ? halo_bytes_of(a.hrows, a.halo_w, a.a_row) : 0u;
+  const uint32_t H_BYTES = a.halo ? halo_bytes_of(a.hrows, a.halo_w) : 0u;
   const uint32_t PITCH = stage_pitch(a.n_tile);
   uint8_t* sA = smem;  // halo: a_bufs x H_BYTES ; tap: ST x kps x A_BYTES
   uint8_t* sB = smem + (a.halo ? a.a_bufs * H_BYTES : ST * a.kps * A_BYTES);
@@ -473,7 +457,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
               if (a.dbg & 4) {  // timing experiment: no halo loads (stale smem)
                 mbar_arrive(afull0 + 8 * ab);
               } else {
-                mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.hrows * a.halo_w * (uint32_t)a.a_row);
+                mbar_expect_tx(afull0 + 8 * ab, (uint32_t)a.hrows * a.halo_w * 128u);
                 tma_load_3d(sA0 + ab * H_BYTES, pmx, afull0 + 8 * ab, cc * 64, x0, y0);
               }
             }
@@ -536,7 +520,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
                              | ((uint32_t)(128 >> 4) << 24);    // M = 128
       uint32_t st = 0, ph = 0, ab = 0, aph = 0, ks = 0, acc = 0, tph = 0;
       const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB) + (uint32_t)(j * n_sub) * 128u;
-      const uint32_t row_r = (uint32_t)a.hrow_px * (uint32_t)a.a_row, row_s = (uint32_t)a.dw * (uint32_t)a.a_row;
+      const uint32_t row_r = (uint32_t)a.hrow_px * 128u, row_s = (uint32_t)a.dw * 128u;
       int tcount = 0;
       if (a.bres) {
         mbar_wait(bres_bar, 0);
@@ -568,13 +552,13 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
           uint32_t xoff = 0;
           if (a.vgrid) {
             const int m0 = ((tile % tiles_mn) / a.tiles_n) * 128;
-            xoff = (uint32_t)(m0 - (m0 / a.vgrid) * a.vgrid) * (uint32_t)a.a_row;
+            xoff = (uint32_t)(m0 - (m0 / a.vgrid) * a.vgrid) * 128u;
           }
           for (int cc = 0; cc < nchunks; ++cc) {
             mbar_wait(afull0 + 8 * ab, aph);
             tc_fence_after();
             if (bres && lane == 0 && j == 0) TRACE2(1, tcount);
-            const uint64_t a0 = umma_desc_a(sA0 + ab * H_BYTES + xoff, a.a_row);
+            const uint64_t a0 = umma_desc_sw128(sA0 + ab * H_BYTES + xoff);
             const int kv = min(4, (C - cc * 64 + 15) >> 4);
             if (bres && fixed_rs) {
               // resident weights, common kernel shapes: the chunk's taps fully
@@ -656,7 +640,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
         const int C = a.C, kps = KPS;
         const uint32_t on = elect_one() ? 1u : 0u;
         const uint32_t ST_ = (uint32_t)ST;
-        const uint64_t aD0 = umma_desc_a(sA0, a.a_row), bD0 = umma_desc_sw128(sB0);
+        const uint64_t aD0 = umma_desc_sw128(sA0), bD0 = umma_desc_sw128(sB0);
         const uint64_t ast16 = A_STAGE >> 4, bst16 = B_STAGE >> 4, a16 = A_BYTES >> 4, b16 = B_BYTES >> 4;
         for (int tile = cta; tile < tiles; tile += ncta, ++tcount) {
           mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
@@ -1100,8 +1084,7 @@ void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st) {
 
 size_t conv_tc_smem_bytes(const ConvTcArgs& a) {
   const size_t B = a.bres ? (size_t)a.n_tile * 128 * a.c_chunks * a.R * a.S : (size_t)a.n_tile * 128 * a.kps * a.stages;
-  const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.hrows, a.halo_w, a.a_row)
-                          : (size_t)a.stages * a.kps * 128 * a.a_row;
+  const size_t A = a.halo ? (size_t)a.a_bufs * halo_bytes_of(a.hrows, a.halo_w) : (size_t)a.stages * a.kps * 128 * 128;
   return 1024 + A + B + (size_t)a.out_bufs * 128 * (size_t)stage_pitch(a.n_tile) +
          (2 * a.stages + 2 * kMaxABufs + 6) * 8 +
          2 * kScaleRes * 4;

@@ -446,10 +446,8 @@ void Executor::allocate() {
 // (waves x per-K-step time, where a K-step costs max(MMA, L2->SM bytes)).
 static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh, int sw, int dh, int dw) {
   ConvTcArgs c{};
-  // C <= 32: 32-channel A rows (64-byte swizzle), else 64-channel chunks
-  c.a_row = C <= 32 ? 64 : 128;
   int hw = 128 + (S - 1) * dw;
-  c.halo = (sw == 1 && Q >= 96 && hw <= 256 && R * dh <= 256 && halo_bytes_of(R, hw, c.a_row) <= 100 * 1024) ? 1 : 0;
+  c.halo = (sw == 1 && Q >= 96 && hw <= 256 && R * dh <= 256 && halo_bytes_of(R, hw) <= 100 * 1024) ? 1 : 0;
   // virtual-grid halo (narrow stride-1 square convs, see ConvTcArgs): tap
   // mode would stream the input R*S times through L2->SM; the box of whole
   // padded rows streams it ~(128 + (R-1) dh Wh + (S-1) dw) / 128 times.
@@ -460,7 +458,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   const int vrows = (Wh - 1 + 127 + (S - 1) * dw) / Wh + 1 + (R - 1) * dh;
   static const bool novgrid = getenv("HIOS_NOVGRID") != nullptr;  // A/B switch
   if (!c.halo && !novgrid && sh == 1 && sw == 1 && dh == 1 && dw == 1 && R == S && R >= 3 && Wh <= 256 && vrows <= 256 &&
-      halo_bytes_of(vrows, Wh, c.a_row) <= 96 * 1024) {
+      halo_bytes_of(vrows, Wh) <= 96 * 1024) {
     c.halo = 1;
     c.vgrid = Wh;
     hw = Wh;
@@ -500,7 +498,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     const int tn = (K + nt - 1) / nt;
     const int nm = n_mma_of(nt);
     const double mma = std::max(4.0 * nt / 2.0, 4.0 * 100.0 / nm);
-    const double a_bytes = c.halo ? (double)c.hrows * c.halo_w * c.a_row / (R * S) : 128.0 * c.a_row;
+    const double a_bytes = c.halo ? (double)c.hrows * c.halo_w * 128.0 / (R * S) : 16384.0;
     const double tma = std::max((c.halo ? 1.0 : 2.0) * 500.0 / 4.0, (a_bytes + nt * 128.0) / 64.0);
     const double epi = nt / 16.0 * 80.0 + 128.0 * nt * 2.0 / 64.0;
     const double tile = std::max(KI * std::max(mma, tma), epi) + 300.0;
@@ -552,18 +550,18 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   const size_t b_all = (size_t)c.c_chunks * R * S * B;
   c.bres = 0;
   if (c.halo && c.tiles_n == 1 && c.tiles_m > g_num_sms * c.occ && b_all <= 96 * 1024 &&
-      halo_bytes_of(c.hrows, hw, c.a_row) + b_all <= budget) {
+      halo_bytes_of(c.hrows, hw) + b_all <= budget) {
     c.bres = 1;
     c.kps = std::min(4, R * S);
     // as many input boxes in flight as fit (measured: the halo TMA latency,
     // ~2 us, bounds a 2-deep ring at small K; tools/conv_trace2.py)
     const int cap = kMaxABufs;
     c.a_bufs = 1;
-    while (c.a_bufs < cap && (c.a_bufs + 1) * halo_bytes_of(c.hrows, hw, c.a_row) + b_all <= budget) ++c.a_bufs;
+    while (c.a_bufs < cap && (c.a_bufs + 1) * halo_bytes_of(c.hrows, hw) + b_all <= budget) ++c.a_bufs;
     c.stages = 2;
   }
   if (c.halo && !c.bres) {
-    const size_t H = halo_bytes_of(c.hrows, hw, c.a_row);
+    const size_t H = halo_bytes_of(c.hrows, hw);
     if (!c.kps) c.kps = std::min(4, R * S);
     while (c.kps > 1 && H + 2 * c.kps * B > budget) --c.kps;
     c.a_bufs = (2 * H + 2 * c.kps * B <= budget) ? 2 : 1;
@@ -576,8 +574,8 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   }
   if (!c.halo) {
     if (!c.kps) c.kps = 4;
-    while (c.kps > 1 && 2 * c.kps * (128 * (size_t)c.a_row + B) > budget) --c.kps;
-    c.stages = (int)std::min<size_t>(8, budget / (c.kps * (128 * (size_t)c.a_row + B)));
+    while (c.kps > 1 && 2 * c.kps * (16384 + B) > budget) --c.kps;
+    c.stages = (int)std::min<size_t>(8, budget / (c.kps * (16384 + B)));
   }
   const int n_stage_steps = (KI + c.kps - 1) / c.kps;
   c.stages = std::max(2, std::min(c.stages, std::max(n_stage_steps, 2)));
@@ -647,15 +645,16 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   // ~16 B/cycle/SM whatever the number of issuing warps, 2-7x slower than an
   // in-bounds box.  Those channels meet zero weights (pitch rup(C, 64)) or are
   // skipped (K=16 slices past C are not issued).
-  const int cw = a.a_row / 2;  // channels per A smem row
-  const int Cm = C % cw ? rup(C, cw) : C;
-  const uint64_t rp = (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2;
+  const int Cm = C % 64 ? rup(C, 64) : C;
   if (a.vgrid)  // hrows whole padded input rows (x from -pw) per channel chunk
-    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, rp, cw, a.halo_w, a.hrows, 1, 1, a.a_row);
+    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w,
+                      a.hrows, 1, 1);
   else if (a.halo)  // R input rows (stride dh) x halo_w pixels per channel chunk
-    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, rp, cw, a.halo_w, R * dh, 1, dh, a.a_row);
+    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w, R * dh, 1,
+                      dh);
   else         // th x tw output positions of one (r, s) tap, conv stride as traversal stride
-    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, rp, cw, a.tw * sw, a.th * sh, sw, sh, a.a_row);
+    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.tw * sw, a.th * sh,
+                      sw, sh);
   if (!ok) fail(HIOS_E_CUDA, "tensor map (activation)");
   const int Cp = rup(C, 64);  // weight pitch: whole zero-padded 64-channel chunks (no TMA OOB fill)
   if (!make_tmap_3d(&mw, w, Cp, R * S, K, (uint64_t)Cp * 2, (uint64_t)R * S * Cp * 2, 64, 1, a.n_tile, 1, 1))

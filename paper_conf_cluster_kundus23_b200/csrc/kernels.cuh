@@ -94,10 +94,6 @@ struct ConvTcArgs {
   // box = whole padded input rows, tap (r, s) = the window at
   // v - v0 + r dh Wh + s dw; virtual columns q >= Q are computed and dropped
   int hrows, hrow_px, vgrid;
-  // bytes per A-operand smem row: 128 (64 channels, 128B swizzle) or, for
-  // C <= 32, 64 (32 channels, 64B swizzle): a 64-channel box over a 32-channel
-  // tensor would stream every input byte twice through L2 -> SM
-  int a_row;
 };
 constexpr int kScaleRes = 512;
 constexpr int kMaxABufs = 6;  // halo-mode input boxes in flight
@@ -176,8 +172,8 @@ struct ConvTcGroup {
 };
 void launch_conv_tc_group(const ConvTcGroup& G, size_t smem, cudaStream_t st);
 void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st);
-__host__ __device__ inline uint32_t halo_bytes_of(int R, int halo_w, int a_row = 128) {
-  return ((uint32_t)R * halo_w * (uint32_t)a_row + 1023u) & ~1023u;
+__host__ __device__ inline uint32_t halo_bytes_of(int R, int halo_w) {
+  return ((uint32_t)R * halo_w * 128u + 1023u) & ~1023u;
 }
 void launch_conv_simt(const ConvSimtArgs& a, cudaStream_t st);
 template <typename T> void launch_conv_small_c(const ConvSmallArgs<T>& a, cudaStream_t st);

@@ -102,11 +102,6 @@ CONV_CASES = [
     (40, 24, 13, 90, 3, 3, 1, 1, 1),      # Wh = 92, ragged last tile, small K
     (72, 200, 11, 7, 5, 5, 1, 2, 2),      # tiny image: one tile spans the whole output
     (64, 64, 20, 31, 3, 3, 1, 0, 0),      # no padding: Wh = Q + 2
-    # C <= 32: 32-channel A rows (64-byte swizzle) in tap / halo / vgrid modes
-    (16, 48, 40, 300, 3, 3, 1, 1, 1),     # halo, C = 16 (box reads 16 channels past C into zero weights)
-    (24, 40, 33, 35, 3, 3, 2, 1, 1),      # tap mode, stride 2, C = 24
-    (32, 96, 30, 30, 3, 3, 1, 1, 1),      # vgrid
-    (32, 64, 50, 50, 1, 1, 1, 0, 0),      # tap 1x1
     # C <= 32 (the box reads past C into zero weights) in halo / tap / vgrid modes
     (16, 48, 40, 300, 3, 3, 1, 1, 1),
     (24, 40, 33, 35, 3, 3, 2, 1, 1),
