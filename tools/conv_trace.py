@@ -54,6 +54,11 @@ for (name, C, K, H, W, kh, kw, s, ph, pw) in SHAPES:
             "tma_issued", "drained"]
     for c in range(min(3, t4.shape[0])):
         print(f"   cta{c} epi4  " + " ".join(f"{n}={v:.2f}" for n, v in zip(lab4, t4[c][:14]) if v > -1e6))
+    b5 = (ctypes.c_ulonglong * (32 * 48))()
+    lib.hios_debug_conv_trace5(b5)
+    t5 = (np.array(b5, dtype=np.int64).reshape(32, 3, 16)[0] - t0) / 1e3
+    print("   cta0 epi tfull", " ".join(f"{v:6.2f}" for v in t5[0]))
+    print("   cta0 epi done ", " ".join(f"{v:6.2f}" for v in t5[1]))
     print("   cta0 issue   ", " ".join(f"{v:6.2f}" for v in t2[0]))
     print("   cta0 full    ", " ".join(f"{v:6.2f}" for v in t2[1]))
     print("   cta0 emptyok ", " ".join(f"{v:6.2f}" for v in t2[2]))
