@@ -187,12 +187,14 @@ __device__ __forceinline__ void mma_commit(uint32_t bar) {
                : "memory");
 }
 
-// halo mode, B ring: one chunk's R_ x S_ taps, KPS_ taps per ring stage
-template <int R_, int S_, int KPS_>
+// halo mode, B ring: one chunk's R_ x S_ taps, KPS_ taps per ring stage;
+// HK_ output rows per tile: each weight stage feeds HK_ accumulators (TMEM
+// columns dstride apart), output row j reading the window one box row lower
+template <int R_, int S_, int KPS_, int HK_>
 __device__ __forceinline__ void halo_taps_ring(uint32_t d, uint64_t a0, uint64_t bD0, uint64_t bst16, uint64_t b16,
                                                uint32_t idesc, int kv, uint32_t on, uint64_t row_r16,
                                                uint64_t row_s16, uint32_t accum, uint32_t& st, uint32_t& ph,
-                                               uint32_t ST, uint32_t full0, uint32_t empty0) {
+                                               uint32_t ST, uint32_t full0, uint32_t empty0, uint32_t dstride) {
   uint64_t b0 = 0;
 #pragma unroll
   for (int t = 0; t < R_ * S_; ++t) {
@@ -201,12 +203,16 @@ __device__ __forceinline__ void halo_taps_ring(uint32_t d, uint64_t a0, uint64_t
       tc_fence_after();
       b0 = bD0 + (uint64_t)st * bst16;
     }
-    const uint64_t ad = a0 + (uint64_t)(t / S_) * row_r16 + (uint64_t)(t % S_) * row_s16;
     const uint64_t bd = b0 + (uint64_t)(t % KPS_) * b16;
-    mma_bf16_on(d, ad, bd, idesc, t == 0 ? accum : 1u, on);
-    if (kv > 1) mma_bf16_on(d, ad + 2, bd + 2, idesc, 1u, on);
-    if (kv > 2) mma_bf16_on(d, ad + 4, bd + 4, idesc, 1u, on);
-    if (kv > 3) mma_bf16_on(d, ad + 6, bd + 6, idesc, 1u, on);
+#pragma unroll
+    for (int j = 0; j < HK_; ++j) {
+      const uint64_t ad = a0 + (uint64_t)(t / S_ + j) * row_r16 + (uint64_t)(t % S_) * row_s16;
+      const uint32_t dj = d + (uint32_t)j * dstride;
+      mma_bf16_on(dj, ad, bd, idesc, t == 0 ? accum : 1u, on);
+      if (kv > 1) mma_bf16_on(dj, ad + 2, bd + 2, idesc, 1u, on);
+      if (kv > 2) mma_bf16_on(dj, ad + 4, bd + 4, idesc, 1u, on);
+      if (kv > 3) mma_bf16_on(dj, ad + 6, bd + 6, idesc, 1u, on);
+    }
     if (t % KPS_ == KPS_ - 1 || t == R_ * S_ - 1) {
       mma_commit_on(empty0 + 8 * st, on);
       if (++st == ST) { st = 0; ph ^= 1u; }
@@ -215,19 +221,23 @@ __device__ __forceinline__ void halo_taps_ring(uint32_t d, uint64_t a0, uint64_t
 }
 
 // halo mode, resident weights: one chunk's R_ x S_ taps (kv K=16 slices
-// each) with compile-time window offsets r * row_r16 + s * row_s16
-template <int R_, int S_>
+// each) with compile-time window offsets r * row_r16 + s * row_s16; HK_ rows
+template <int R_, int S_, int HK_>
 __device__ __forceinline__ void halo_taps_bres(uint32_t d, uint64_t a0, uint64_t b0, uint32_t idesc, int kv,
                                                uint32_t on, uint64_t row_r16, uint64_t row_s16, uint64_t b16,
-                                               uint32_t accum) {
+                                               uint32_t accum, uint32_t dstride) {
 #pragma unroll
   for (int t = 0; t < R_ * S_; ++t) {
-    const uint64_t ad = a0 + (uint64_t)(t / S_) * row_r16 + (uint64_t)(t % S_) * row_s16;
     const uint64_t bd = b0 + (uint64_t)t * b16;
-    mma_bf16_on(d, ad, bd, idesc, t == 0 ? accum : 1u, on);
-    if (kv > 1) mma_bf16_on(d, ad + 2, bd + 2, idesc, 1u, on);
-    if (kv > 2) mma_bf16_on(d, ad + 4, bd + 4, idesc, 1u, on);
-    if (kv > 3) mma_bf16_on(d, ad + 6, bd + 6, idesc, 1u, on);
+#pragma unroll
+    for (int j = 0; j < HK_; ++j) {
+      const uint64_t ad = a0 + (uint64_t)(t / S_ + j) * row_r16 + (uint64_t)(t % S_) * row_s16;
+      const uint32_t dj = d + (uint32_t)j * dstride;
+      mma_bf16_on(dj, ad, bd, idesc, t == 0 ? accum : 1u, on);
+      if (kv > 1) mma_bf16_on(dj, ad + 2, bd + 2, idesc, 1u, on);
+      if (kv > 2) mma_bf16_on(dj, ad + 4, bd + 4, idesc, 1u, on);
+      if (kv > 3) mma_bf16_on(dj, ad + 6, bd + 6, idesc, 1u, on);
+    }
   }
 }
 
@@ -540,13 +550,14 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
                                                   (a.R == 1 && a.S == 1 && KPS == 1) ||
                                                   (a.R * a.S == 7 && (a.R == 1 || a.S == 1) && KPS == 4) ||
                                                   (a.R * a.S == 3 && (a.R == 1 || a.S == 1) && KPS == 3));
+        const bool hk2 = a.hk == 2;  // (plan_conv_tc: hk > 1 only for fixed-loop shapes, hk <= 2)
         const bool fixed_rs = !(a.dbg & 32) && ((a.R == 3 && a.S == 3) || (a.R == 1 && a.S == 1) ||
                                                 (a.R == 2 && a.S == 1) || (a.R == 4 && a.S == 1) ||
                                                 (a.R == 5 && a.S == 5));
         for (int tile = cta; tile < tiles; tile += ncta, ++tcount) {
           mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
           tc_fence_after();
-          const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
+          const uint32_t d = tmem + acc * (uint32_t)(a.hk * a.n_tile) + (uint32_t)(j * n_sub);
           uint32_t accum = 0;
           // vgrid: the tile's window starts v0 mod Wh pixels into the box
           uint32_t xoff = 0;
@@ -565,11 +576,24 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
               // unrolled with compile-time window offsets (descriptor adds on
               // the uniform datapath, no loop-carried offsets)
               const uint64_t bc = bres0 + (uint64_t)(cc * RS) * b16;
-              if (a.R == 3 && S_ == 3) halo_taps_bres<3, 3>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
-              else if (a.R == 1 && S_ == 1) halo_taps_bres<1, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
-              else if (a.R == 2 && S_ == 1) halo_taps_bres<2, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
-              else if (a.R == 4 && S_ == 1) halo_taps_bres<4, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
-              else if (a.R == 5 && S_ == 5) halo_taps_bres<5, 5>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum);
+              const uint32_t dsx = (uint32_t)a.n_tile;
+              if (a.R == 3 && S_ == 3) {
+                if (hk2) halo_taps_bres<3, 3, 2>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+                else halo_taps_bres<3, 3, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+              }
+              else if (a.R == 1 && S_ == 1) halo_taps_bres<1, 1, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+              else if (a.R == 2 && S_ == 1) {
+                if (hk2) halo_taps_bres<2, 1, 2>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+                else halo_taps_bres<2, 1, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+              }
+              else if (a.R == 4 && S_ == 1) {
+                if (hk2) halo_taps_bres<4, 1, 2>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+                else halo_taps_bres<4, 1, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+              }
+              else if (a.R == 5 && S_ == 5) {
+                if (hk2) halo_taps_bres<5, 5, 2>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+                else halo_taps_bres<5, 5, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+              }
               else __trap();  // unreachable: fixed_rs lists exactly these shapes
               accum = 1;
               mma_commit_on(aempty0 + 8 * ab, on);
@@ -582,21 +606,41 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
               // compile-time tap boundaries (kps taps per stage)
               // (dispatch on R, S and kps together: each template's stage
               // boundaries must match the producer's)
-              if (a.R == 3 && S_ == 3 && kps == 3) halo_taps_ring<3, 3, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 3 && S_ == 3 && kps == 2) halo_taps_ring<3, 3, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 3 && S_ == 3 && kps == 4) halo_taps_ring<3, 3, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 5 && S_ == 5 && kps == 4) halo_taps_ring<5, 5, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 1 && S_ == 7 && kps == 4) halo_taps_ring<1, 7, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 7 && S_ == 1 && kps == 4) halo_taps_ring<7, 1, 4>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 1 && S_ == 3 && kps == 3) halo_taps_ring<1, 3, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 3 && S_ == 1 && kps == 3) halo_taps_ring<3, 1, 3>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
-              else if (a.R == 1 && S_ == 1 && kps == 1) halo_taps_ring<1, 1, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0);
+              const uint32_t dsr = (uint32_t)a.n_tile;
+              if (a.R == 3 && S_ == 3 && kps == 3) {
+                if (hk2) halo_taps_ring<3, 3, 3, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+                else halo_taps_ring<3, 3, 3, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+              }
+              else if (a.R == 3 && S_ == 3 && kps == 2) {
+                if (hk2) halo_taps_ring<3, 3, 2, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+                else halo_taps_ring<3, 3, 2, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+              }
+              else if (a.R == 3 && S_ == 3 && kps == 4) {
+                if (hk2) halo_taps_ring<3, 3, 4, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+                else halo_taps_ring<3, 3, 4, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+              }
+              else if (a.R == 5 && S_ == 5 && kps == 4) {
+                if (hk2) halo_taps_ring<5, 5, 4, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+                else halo_taps_ring<5, 5, 4, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+              }
+              else if (a.R == 1 && S_ == 7 && kps == 4) halo_taps_ring<1, 7, 4, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+              else if (a.R == 7 && S_ == 1 && kps == 4) {
+                if (hk2) halo_taps_ring<7, 1, 4, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+                else halo_taps_ring<7, 1, 4, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+              }
+              else if (a.R == 1 && S_ == 3 && kps == 3) halo_taps_ring<1, 3, 3, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+              else if (a.R == 3 && S_ == 1 && kps == 3) {
+                if (hk2) halo_taps_ring<3, 1, 3, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+                else halo_taps_ring<3, 1, 3, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+              }
+              else if (a.R == 1 && S_ == 1 && kps == 1) halo_taps_ring<1, 1, 1, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
               else __trap();  // unreachable: fixed_ring lists exactly these shapes
               accum = 1;
               mma_commit_on(aempty0 + 8 * ab, on);
               if (++ab == (uint32_t)abufs) { ab = 0; aph ^= 1u; }
               continue;
             }
+            if (a.hk != 1) __trap();  // plan_conv_tc: row groups only for the unrolled shapes
             uint64_t aoff_r = 0, aoff = 0;
             int s_ = 0;
             for (int t = 0; t < RS;) {
@@ -776,7 +820,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
       TRACE4(2);
       TRACE5(0, tcount);
       if (tcount == 0 && warp == kEpiWarp0 && lane == 0) TRACE(5);
-      const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)a.n_tile;
+      const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)(a.hk * a.n_tile);
       if (a.dbg & 16) {  // timing experiment: accumulator released unread
         tc_fence_before();
         mbar_arrive(tempty0 + 8 * acc);
@@ -791,16 +835,19 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
         // registers -- no staging, no proxy fence, no bulk-group waits
         const float* scs = s_scale + (a.sres ? n0 : 0);
         const float* shs = s_shift + (a.sres ? n0 : 0);
+        for (int jr = 0; jr < a.hk; ++jr) {  // output row jr of the tile's row group
+        const uint32_t tbj = tbase + (uint32_t)(jr * a.n_tile);
         int p, q;
         tile_pixel(a, m_blk, p0, q0, m, p, q);
+        p += jr;
         const bool valid = p < a.P && q < a.Q;
         const size_t pix = (size_t)p * a.Q + q;
         bf16* o1 = a.out + pix * a.ldo + n0;
         for (int col = 0; col < a.n_tile; col += 32) {
           const bool two = col + 16 < a.n_tile;  // warp-uniform
           uint32_t r0[16], r1[16];
-          tmem_ld16_nw(tbase + (uint32_t)col, r0);
-          if (two) tmem_ld16_nw(tbase + (uint32_t)col + 16u, r1);
+          tmem_ld16_nw(tbj + (uint32_t)col, r0);
+          if (two) tmem_ld16_nw(tbj + (uint32_t)col + 16u, r1);
           float sc[32], sf[32];
 #pragma unroll
           for (int q4 = 0; q4 < 8; ++q4) {
@@ -847,6 +894,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
             }
           }
         }
+        }  // jr
         tc_fence_before();
         mbar_arrive(tempty0 + 8 * acc);
         TRACE5(1, tcount);

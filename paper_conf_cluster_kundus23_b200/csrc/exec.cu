@@ -444,8 +444,10 @@ void Executor::allocate() {
 // Tile plan of one tcgen05 conv (see conv_tc.cu): halo mode for stride-1-in-W
 // convs with wide outputs, tap mode otherwise; n_tile from a small cost model
 // (waves x per-K-step time, where a K-step costs max(MMA, L2->SM bytes)).
-static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh, int sw, int dh, int dw) {
+static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh, int sw, int dh, int dw,
+                               bool allow_hk = true) {
   ConvTcArgs c{};
+  c.hk = 1;
   int hw = 128 + (S - 1) * dw;
   c.halo = (sw == 1 && Q >= 96 && hw <= 256 && R * dh <= 256 && halo_bytes_of(R, hw) <= 100 * 1024) ? 1 : 0;
   // virtual-grid halo (narrow stride-1 square convs, see ConvTcArgs): tap
@@ -478,6 +480,19 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
       if (best < 0 || cost < best) { best = cost; c.th = th; c.tw = tw; }
     }
     if (best < 0) fail(HIOS_E_UNSUPPORTED, "conv stride too large for the TMA box");
+  }
+  // row groups (classic halo, stride 1, shapes with an unrolled tap loop):
+  // two output rows per tile share one box of R + 1 input rows and every
+  // weight stage (B) -- per output row, R -> (R + 1) / 2 input rows and half
+  // the weight bytes cross L2 -> SM (the halo convs at 2048^2 / 4096^2 are
+  // bound by the TMA's per-row processing, profiles/README.md)
+  static const bool nohk = getenv("HIOS_NOHK") != nullptr;  // A/B switch
+  const bool hk_shape = (R == 3 && S == 3) || (R == 5 && S == 5) || (R == 7 && S == 1) || (R == 3 && S == 1) ||
+                        (R == 2 && S == 1) || (R == 4 && S == 1);
+  if (allow_hk && !nohk && c.halo && !c.vgrid && sh == 1 && dh == 1 && hk_shape && P >= 4) {
+    c.hk = 2;
+    c.th = 2;
+    c.hrows = R + 1;
   }
   c.tiles_q = (Q + c.tw - 1) / c.tw;
   c.tiles_m = ((P + c.th - 1) / c.th) * c.tiles_q;
@@ -526,6 +541,10 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     const int nb = (K + cap - 1) / cap;
     c.n_tile = rup((K + nb - 1) / nb, 16);
   }
+  if (c.hk > 1 && c.n_tile > 128) {  // hk accumulators double-buffered: 2 * hk * n_tile <= 512 TMEM columns
+    const int nb = (K + 127) / 128;
+    c.n_tile = rup((K + nb - 1) / nb, 16);
+  }
   c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
   c.n_mma = 1;  // measured: splitting N over several MMA warps does not pay (tools/conv_micro.py)
   const size_t B = (size_t)c.n_tile * 128;
@@ -569,7 +588,10 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
       const int cap = 4;
       while (c.a_bufs < cap && (c.a_bufs + 1) * H + 4 * c.kps * B <= budget) ++c.a_bufs;
     }
-    if (H + 2 * c.kps * B > budget) fail(HIOS_E_UNSUPPORTED, "conv halo plan does not fit shared memory");
+    if (H + 2 * c.kps * B > budget) {
+      if (c.hk > 1) return plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw, false);
+      fail(HIOS_E_UNSUPPORTED, "conv halo plan does not fit shared memory");
+    }
     else c.stages = (int)std::min<size_t>(8, (budget - c.a_bufs * H) / (c.kps * B));
   }
   if (!c.halo) {
@@ -589,6 +611,16 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   // small-spatial conv faster alone (7c_3x3 18.3 -> 14.5 us) but the step
   // slower (0.865 -> 0.88-0.90 ms): the extra CTAs and the finalize launch
   // crowd out the stage's concurrent ops.  So it is opt-in (HIOS_SPLITK=1).
+  if (c.hk > 1) {
+    // the kernel's row-group loops exist only for the unrolled (R, S, kps)
+    // shapes (conv_tc.cu halo_taps_ring / halo_taps_bres) and the direct-store
+    // epilogue; anything else plans without row groups
+    const bool ring_ok = (R == 3 && S == 3 && c.kps >= 2 && c.kps <= 4) || (R == 5 && S == 5 && c.kps == 4) ||
+                         (R == 7 && S == 1 && c.kps == 4) || (R == 3 && S == 1 && c.kps == 3);
+    const bool bres_ok = (R == 3 && S == 3) || (R == 2 && S == 1) || (R == 4 && S == 1) || (R == 5 && S == 5);
+    if (c.epi != 2 || !(c.bres ? bres_ok : ring_ok))
+      return plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw, false);
+  }
   if (!c.halo && getenv("HIOS_SPLITK") && tiles < 48 && KI >= 16) {
     // at most one wave of CTAs, >= ~6 K-steps each; splits may start at any
     // (chunk, tap) K-step
@@ -650,8 +682,8 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
     ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w,
                       a.hrows, 1, 1);
   else if (a.halo)  // R input rows (stride dh) x halo_w pixels per channel chunk
-    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w, R * dh, 1,
-                      dh);
+    ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.halo_w,
+                      a.hrows * dh, 1, dh);
   else         // th x tw output positions of one (r, s) tap, conv stride as traversal stride
     ok = make_tmap_3d(&mx, in.p, Cm, W, H, (uint64_t)in.ldc * 2, (uint64_t)(in.row_px ? in.row_px : W) * in.ldc * 2, 64, a.tw * sw, a.th * sh,
                       sw, sh);

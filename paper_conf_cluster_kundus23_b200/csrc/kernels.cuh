@@ -94,6 +94,11 @@ struct ConvTcArgs {
   // box = whole padded input rows, tap (r, s) = the window at
   // v - v0 + r dh Wh + s dw; virtual columns q >= Q are computed and dropped
   int hrows, hrow_px, vgrid;
+  // classic halo, stride 1: hk consecutive output rows per tile (hk > 1: one
+  // box of R + hk - 1 input rows feeds hk accumulators, so every input row and
+  // every weight stage crosses L2 -> SM once per hk output rows instead of R /
+  // once per row; tile_row = output-row group, th = hk)
+  int hk;
 };
 constexpr int kScaleRes = 512;
 constexpr int kMaxABufs = 6;  // halo-mode input boxes in flight
