@@ -541,11 +541,13 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     const int nb = (K + cap - 1) / cap;
     c.n_tile = rup((K + nb - 1) / nb, 16);
   }
-  if (c.hk > 1 && c.n_tile > 128) {  // hk accumulators double-buffered: 2 * hk * n_tile <= 512 TMEM columns
-    const int nb = (K + 127) / 128;
-    c.n_tile = rup((K + nb - 1) / nb, 16);
-  }
   c.tiles_n = (K + c.n_tile - 1) / c.n_tile;
+  // row groups need 2 * hk * n_tile <= 512 TMEM columns and pay only with
+  // enough tiles to fill the SMs twice (measured, tools/conv_micro.py: forcing
+  // n_tile <= 128 made Mixed_7b 3x3 at 126^2 49.7 -> 59.4 us; halving the tiles
+  // of Conv2d_4a at 254^2 29.6 -> 31.8 us; 2a / 2b / 5x5 at 4096^2 -16..-23 %)
+  if (c.hk > 1 && (c.n_tile > 128 || (int64_t)c.tiles_m * c.tiles_n < 2LL * g_num_sms))
+    return plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw, false);
   c.n_mma = 1;  // measured: splitting N over several MMA warps does not pay (tools/conv_micro.py)
   const size_t B = (size_t)c.n_tile * 128;
   const size_t stage_out = 128 * ((size_t)c.n_tile * 2 + 16);
