@@ -675,7 +675,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
           mma_commit_on(tfull0 + 8 * acc, on);
           __syncwarp();
           if (lane == 0 && tcount == 0 && j == 0) TRACE(4);
-          acc ^= 1u;
+          if (a.nacc == 2) acc ^= 1u;
           if (acc == 0) tph ^= 1u;
         }
       } else {
@@ -721,7 +721,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
           mma_commit_on(tfull0 + 8 * acc, on);
           __syncwarp();
           if (lane == 0 && tcount == 0 && j == 0) TRACE(4);
-          acc ^= 1u;
+          if (a.nacc == 2) acc ^= 1u;
           if (acc == 0) tph ^= 1u;
         }
       }
@@ -779,7 +779,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
         }
         tc_fence_before();
         mbar_arrive(tempty0 + 8 * acc);
-        acc ^= 1u;
+        if (a.nacc == 2) acc ^= 1u;
         if (acc == 0) tph ^= 1u;
         continue;
       }
@@ -825,7 +825,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
         tc_fence_before();
         mbar_arrive(tempty0 + 8 * acc);
         TRACE5(1, tcount);
-        acc ^= 1u;
+        if (a.nacc == 2) acc ^= 1u;
         if (acc == 0) tph ^= 1u;
         continue;
       }
@@ -898,7 +898,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
         tc_fence_before();
         mbar_arrive(tempty0 + 8 * acc);
         TRACE5(1, tcount);
-        acc ^= 1u;
+        if (a.nacc == 2) acc ^= 1u;
         if (acc == 0) tph ^= 1u;
         continue;
       }
@@ -960,7 +960,7 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
       tc_fence_before();
       mbar_arrive(tempty0 + 8 * acc);  // TMEM accumulator free for the next tile
       if (tcount == 0 && warp == kEpiWarp0 && lane == 0) TRACE(6);
-      acc ^= 1u;
+      if (a.nacc == 2) acc ^= 1u;
       if (acc == 0) tph ^= 1u;
       TRACE4(9);
       if (a.tma_out) {

@@ -546,8 +546,11 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   // enough tiles to fill the SMs twice (measured, tools/conv_micro.py: forcing
   // n_tile <= 128 made Mixed_7b 3x3 at 126^2 49.7 -> 59.4 us; halving the tiles
   // of Conv2d_4a at 254^2 29.6 -> 31.8 us; 2a / 2b / 5x5 at 4096^2 -16..-23 %)
-  if (c.hk > 1 && (c.n_tile > 128 || (int64_t)c.tiles_m * c.tiles_n < 2LL * g_num_sms))
+  if (c.hk > 1 && (c.n_tile > 256 || (int64_t)c.tiles_m * c.tiles_n < 2LL * g_num_sms))
     return plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw, false);
+  // TMEM: 2 accumulator sets of hk x n_tile columns when they fit in 512,
+  // else one (the epilogue then does not overlap the next tile's MMAs)
+  c.nacc = 2 * c.hk * c.n_tile <= 512 ? 2 : 1;
   c.n_mma = 1;  // measured: splitting N over several MMA warps does not pay (tools/conv_micro.py)
   const size_t B = (size_t)c.n_tile * 128;
   const size_t stage_out = 128 * ((size_t)c.n_tile * 2 + 16);
@@ -558,7 +561,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   c.occ = 1;
   // epilogue mode (HIOS_EPI overrides): direct register stores for N tiles
   // <= 128 (no staging tile), TMA bulk-tensor stores for wider tiles
-  c.epi = c.n_tile <= 128 ? 2 : 1;
+  c.epi = (c.n_tile <= 128 || c.hk > 1) ? 2 : 1;  // row groups: direct stores (any n_tile)
   c.out_bufs = c.epi == 2 ? 0 : (c.n_tile <= (c.occ == 2 ? 48 : 128) ? 2 : 1);
   c.sres = c.tiles_n * c.n_tile <= kScaleRes ? 1 : 0;
   // occupancy: 1 CTA/SM (212 KB) or 2 CTAs/SM (104 KB each, TMEM <= 256 cols)
@@ -620,7 +623,7 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     const bool ring_ok = (R == 3 && S == 3 && c.kps >= 2 && c.kps <= 4) || (R == 5 && S == 5 && c.kps == 4) ||
                          (R == 7 && S == 1 && c.kps == 4) || (R == 3 && S == 1 && c.kps == 3);
     const bool bres_ok = (R == 3 && S == 3) || (R == 2 && S == 1) || (R == 4 && S == 1) || (R == 5 && S == 5);
-    if (c.epi != 2 || !(c.bres ? bres_ok : ring_ok))
+    if (c.epi != 2 || !(c.bres ? bres_ok : ring_ok) || (c.nacc == 1 && c.bres))
       return plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw, false);
   }
   if (!c.halo && getenv("HIOS_SPLITK") && tiles < 48 && KI >= 16) {

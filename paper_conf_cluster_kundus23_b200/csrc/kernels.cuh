@@ -99,6 +99,8 @@ struct ConvTcArgs {
   // every weight stage crosses L2 -> SM once per hk output rows instead of R /
   // once per row; tile_row = output-row group, th = hk)
   int hk;
+  int nacc;  // TMEM accumulator sets (2: the epilogue of tile i overlaps the MMAs of tile i+1; 1 when
+             // 2 * hk * n_tile > 512 columns)
 };
 constexpr int kScaleRes = 512;
 constexpr int kMaxABufs = 6;  // halo-mode input boxes in flight

@@ -102,6 +102,11 @@ CONV_CASES = [
     (40, 24, 13, 90, 3, 3, 1, 1, 1),      # Wh = 92, ragged last tile, small K
     (72, 200, 11, 7, 5, 5, 1, 2, 2),      # tiny image: one tile spans the whole output
     (64, 64, 20, 31, 3, 3, 1, 0, 0),      # no padding: Wh = Q + 2
+    # row-group halo tiles (two output rows per box; >= 2 x 148 tiles)
+    (32, 64, 300, 150, 3, 3, 1, 1, 1),    # resident weights, two accumulator sets
+    (64, 192, 300, 200, 3, 3, 1, 1, 1),   # n_tile 192: one accumulator set (nacc 1)
+    (48, 64, 201, 300, 5, 5, 1, 2, 2),    # 5x5, odd P (last group half empty)
+    (64, 160, 401, 130, 7, 1, 1, 3, 0),   # 7x1 weight ring
     # C <= 32 (the box reads past C into zero weights) in halo / tap / vgrid modes
     (16, 48, 40, 300, 3, 3, 1, 1, 1),
     (24, 40, 33, 35, 3, 3, 2, 1, 1),
