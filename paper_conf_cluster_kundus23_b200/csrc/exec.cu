@@ -546,10 +546,12 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   // enough tiles to fill the SMs twice (measured, tools/conv_micro.py: forcing
   // n_tile <= 128 made Mixed_7b 3x3 at 126^2 49.7 -> 59.4 us; halving the tiles
   // of Conv2d_4a at 254^2 29.6 -> 31.8 us; 2a / 2b / 5x5 at 4096^2 -16..-23 %)
-  if (c.hk > 1 && (c.n_tile > 256 || (int64_t)c.tiles_m * c.tiles_n < 2LL * g_num_sms))
+  // (measured: with n_tile 192 and one accumulator set -- no epilogue overlap
+  // -- Conv2d_4a at 4096^2 371 -> 379 us, so row groups keep two sets)
+  if (c.hk > 1 && (c.n_tile > 128 || (int64_t)c.tiles_m * c.tiles_n < 2LL * g_num_sms))
     return plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw, false);
-  // TMEM: 2 accumulator sets of hk x n_tile columns when they fit in 512,
-  // else one (the epilogue then does not overlap the next tile's MMAs)
+  // TMEM accumulator sets of hk x n_tile columns (the kernel supports 1 when
+  // 2 sets do not fit in 512 columns)
   c.nacc = 2 * c.hk * c.n_tile <= 512 ? 2 : 1;
   c.n_mma = 1;  // measured: splitting N over several MMA warps does not pay (tools/conv_micro.py)
   const size_t B = (size_t)c.n_tile * 128;
