@@ -581,7 +581,10 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
                 if (hk2) halo_taps_bres<3, 3, 2>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
                 else halo_taps_bres<3, 3, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
               }
-              else if (a.R == 1 && S_ == 1) halo_taps_bres<1, 1, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+              else if (a.R == 1 && S_ == 1) {
+                if (hk2) halo_taps_bres<1, 1, 2>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+                else halo_taps_bres<1, 1, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
+              }
               else if (a.R == 2 && S_ == 1) {
                 if (hk2) halo_taps_bres<2, 1, 2>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
                 else halo_taps_bres<2, 1, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
@@ -633,7 +636,10 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
                 if (hk2) halo_taps_ring<3, 1, 3, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
                 else halo_taps_ring<3, 1, 3, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
               }
-              else if (a.R == 1 && S_ == 1 && kps == 1) halo_taps_ring<1, 1, 1, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+              else if (a.R == 1 && S_ == 1 && kps == 1) {
+                if (hk2) halo_taps_ring<1, 1, 1, 2>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+                else halo_taps_ring<1, 1, 1, 1>(d, a0, bD0h, bst16, b16, idesc, kv, on, row_r16, row_s16, accum, st, ph, ST_, full0, empty0, dsr);
+              }
               else __trap();  // unreachable: fixed_ring lists exactly these shapes
               accum = 1;
               mma_commit_on(aempty0 + 8 * ab, on);
@@ -839,7 +845,8 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
         const uint32_t tbj = tbase + (uint32_t)(jr * a.n_tile);
         int p, q;
         tile_pixel(a, m_blk, p0, q0, m, p, q);
-        p += jr;
+        if (a.hk_px) q += jr * 128;  // pixel pairs (1x1): the second 128 pixels of the row segment
+        else p += jr;                 // row groups: the next output row
         const bool valid = p < a.P && q < a.Q;
         const size_t pix = (size_t)p * a.Q + q;
         bf16* o1 = a.out + pix * a.ldo + n0;

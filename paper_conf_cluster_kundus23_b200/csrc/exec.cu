@@ -494,6 +494,17 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     c.th = 2;
     c.hrows = R + 1;
   }
+  // pixel pairs (1x1, stride 1, wide rows): a tile is 256 consecutive pixels of
+  // one output row as two 128-pixel accumulators sharing every weight stage
+  // (one box of 256 pixels per channel chunk): half the weight bytes per output
+  if (allow_hk && !nohk && c.halo && !c.vgrid && R == 1 && S == 1 && sh == 1 && Q >= 192) {
+    c.hk = 2;
+    c.hk_px = 1;
+    c.tw = 256;
+    c.halo_w = 256;
+    hw = 256;
+    c.hrow_px = 128;  // accumulator j reads the window j * 128 pixels into the box
+  }
   c.tiles_q = (Q + c.tw - 1) / c.tw;
   c.tiles_m = ((P + c.th - 1) / c.th) * c.tiles_q;
   if (c.vgrid) {
@@ -624,8 +635,10 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     // epilogue; anything else plans without row groups
     const bool ring_ok = (R == 3 && S == 3 && c.kps >= 2 && c.kps <= 4) || (R == 5 && S == 5 && c.kps == 4) ||
                          (R == 7 && S == 1 && c.kps == 4) || (R == 3 && S == 1 && c.kps == 3);
-    const bool bres_ok = (R == 3 && S == 3) || (R == 2 && S == 1) || (R == 4 && S == 1) || (R == 5 && S == 5);
-    if (c.epi != 2 || !(c.bres ? bres_ok : ring_ok) || (c.nacc == 1 && c.bres))
+    const bool bres_ok = (R == 3 && S == 3) || (R == 2 && S == 1) || (R == 4 && S == 1) || (R == 5 && S == 5) ||
+                         (R == 1 && S == 1);
+    const bool ring_ok1 = R == 1 && S == 1 && c.kps == 1;
+    if (c.epi != 2 || !(c.bres ? bres_ok : (ring_ok || ring_ok1)) || (c.nacc == 1 && c.bres))
       return plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw, false);
   }
   if (!c.halo && getenv("HIOS_SPLITK") && tiles < 48 && KI >= 16) {

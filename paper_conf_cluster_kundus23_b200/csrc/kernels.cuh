@@ -99,6 +99,7 @@ struct ConvTcArgs {
   // every weight stage crosses L2 -> SM once per hk output rows instead of R /
   // once per row; tile_row = output-row group, th = hk)
   int hk;
+  int hk_px;  // hk > 1 for a 1x1 conv: the tile is 2 x 128 consecutive pixels of one row (box 256 px)
   int nacc;  // TMEM accumulator sets (2: the epilogue of tile i overlaps the MMAs of tile i+1; 1 when
              // 2 * hk * n_tile > 512 columns)
 };

@@ -107,6 +107,9 @@ CONV_CASES = [
     (64, 192, 300, 200, 3, 3, 1, 1, 1),   # n_tile 192: one accumulator set (nacc 1)
     (48, 64, 201, 300, 5, 5, 1, 2, 2),    # 5x5, odd P (last group half empty)
     (64, 160, 401, 130, 7, 1, 1, 3, 0),   # 7x1 weight ring
+    # pixel pairs (1x1, rows >= 192 px: two 128-pixel accumulators per 256-pixel box)
+    (192, 64, 150, 509, 1, 1, 1, 0, 0),   # ragged last pair, resident weights
+    (288, 96, 160, 600, 1, 1, 1, 0, 0),   # C tail (288 = 4.5 chunks), weight ring
     # C <= 32 (the box reads past C into zero weights) in halo / tap / vgrid modes
     (16, 48, 40, 300, 3, 3, 1, 1, 1),
     (24, 40, 33, 35, 3, 3, 2, 1, 1),

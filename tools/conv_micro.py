@@ -28,6 +28,9 @@ SHAPES = [  # name, C, K, H, W, kh, kw, s, ph, pw
     ("5b5x5_4096", 48, 64, 509, 509, 5, 5, 1, 2, 2),
     ("7c1x1_4096", 2048, 448, 126, 126, 1, 1, 1, 0, 0),
     ("7b3x3_4096", 448, 384, 126, 126, 3, 3, 1, 1, 1),
+    ("5b1x1_4096", 192, 64, 509, 509, 1, 1, 1, 0, 0),
+    ("6e1x1_4096", 768, 192, 254, 254, 1, 1, 1, 0, 0),
+    ("3b_4096", 64, 80, 1022, 1022, 1, 1, 1, 0, 0),
 ]
 
 
