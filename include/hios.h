@@ -313,6 +313,18 @@ hios_status hios_time_ops(hios_schedule s, int32_t reps, int64_t flush_bytes, in
  * that are kernels written in this library). */
 hios_status hios_kernel_count(hios_schedule s, int64_t* n);
 
+/* Tile plan of op `op`'s tcgen05 convolution as lowered for Q ("the
+ * convolution ... operators"), for inspection and tests:
+ * solo = 0 the plan used inside its stage, 1 the plan used when the op runs
+ * alone (a singleton stage, t(v) profiling).  plan[8] (caller-owned) =
+ * {A-operand mode: 1 tap, 2 halo, 3 virtual-grid halo; N tile; output tiles;
+ * epilogue: 0 smem staging, 1 TMA bulk-tensor stores, 2 direct stores;
+ * 1 = 256-bit direct stores; output rows per tile; pipeline stages;
+ * K-steps per stage}; all zero for ops without a tcgen05
+ * conv (other kinds, fp32 graphs, CUDA-core stems).  Errors: HIOS_E_INVALID
+ * (NULL, op out of range), HIOS_E_STATE (Q not run yet). */
+hios_status hios_op_plan(hios_schedule s, int32_t op, int32_t solo, int32_t* plan);
+
 /* ------------------------------------------------------------------ misc */
 const char* hios_last_error(void);
 int32_t hios_abi_version(void);

@@ -508,6 +508,15 @@ hios_status hios_time_ops(hios_schedule s, int32_t reps, int64_t flush_bytes, in
   });
 }
 
+hios_status hios_op_plan(hios_schedule s, int32_t op, int32_t solo, int32_t* plan) {
+  return guard([&] {
+    NEED(s && plan && op >= 0 && op < s->s->g->n, HIOS_E_INVALID, "bad argument");
+    NEED(s->s->exec && s->s->exec->captured, HIOS_E_STATE, "run first");
+    const hios::OpExec& x = s->s->exec->ox[op];
+    for (int i = 0; i < 8; ++i) plan[i] = solo ? x.plan_solo[i] : x.plan[i];
+  });
+}
+
 hios_status hios_kernel_count(hios_schedule s, int64_t* n) {
   return guard([&] {
     NEED(s && n, HIOS_E_INVALID, "NULL argument");

@@ -79,6 +79,20 @@ __device__ __forceinline__ uint4 lds128(uint32_t addr) {
                : "memory");
   return v;
 }
+// folded-BN epilogue of two accumulator columns: + shift (the scale is folded
+// into the weights at upload, exec.cu conv_layout), optional ReLU, rounded to
+// bf16x2; lo -> bits [0,16)
+__device__ __forceinline__ uint32_t bias_relu_pack(uint32_t lo, uint32_t hi, float b_lo, float b_hi, int relu) {
+  float y0 = __uint_as_float(lo) + b_lo, y1 = __uint_as_float(hi) + b_hi;
+  if (relu) { y0 = fmaxf(y0, 0.f); y1 = fmaxf(y1, 0.f); }
+  __nv_bfloat162 b2 = __floats2bfloat162_rn(y0, y1);
+  return *reinterpret_cast<uint32_t*>(&b2);
+}
+__device__ __forceinline__ void st_global_256(void* p, const uint32_t (&v)[8]) {
+  asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(p), "r"(v[0]), "r"(v[1]), "r"(v[2]),
+               "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+               : "memory");
+}
 __device__ __forceinline__ uint16_t lds16(uint32_t addr) {
   uint16_t v;
   asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(addr) : "memory");
@@ -307,6 +321,12 @@ __device__ __forceinline__ unsigned long long gtimer() {
     if (a.trace && blockIdx.x < 256) g_conv_trace[blockIdx.x * 8 + (k)] = gtimer(); \
   } while (0)
 
+// split and output-tile index of persistent tile number `tile`
+__device__ __forceinline__ void split_of(const ConvTcArgs& a, int tile, int tiles_mn, int& split, int& tmn) {
+  split = tile / tiles_mn;
+  tmn = tile - split * tiles_mn;
+}
+
 static __host__ __device__ inline uint32_t tmem_cols(int n) {
   uint32_t c = 32;
   while ((int)c < n) c <<= 1;
@@ -447,7 +467,8 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
       }
       if (a.bres) mine = 1 << 30;  // no B ring
       for (int tile = cta; tile < tiles; tile += ncta) {
-        const int split = tile / tiles_mn, tmn = tile - split * tiles_mn;
+        int split, tmn;
+        split_of(a, tile, tiles_mn, split, tmn);
         const int m_blk = tmn / a.tiles_n, n_blk = tmn - m_blk * a.tiles_n;
         const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
         const int p0 = tp * a.th, q0 = tq * a.tw, n0 = n_blk * a.n_tile;
@@ -561,11 +582,16 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
           uint32_t accum = 0;
           // vgrid: the tile's window starts v0 mod Wh pixels into the box
           uint32_t xoff = 0;
+          int split_, tmn_;
+          split_of(a, tile, tiles_mn, split_, tmn_);
           if (a.vgrid) {
-            const int m0 = ((tile % tiles_mn) / a.tiles_n) * 128;
+            const int m0 = (tmn_ / a.tiles_n) * 128;
             xoff = (uint32_t)(m0 - (m0 / a.vgrid) * a.vgrid) * 128u;
           }
-          for (int cc = 0; cc < nchunks; ++cc) {
+          // the tile's channel chunks [c_lo, c_hi) (a K split of whole chunks;
+          // kpsplit = R * S * c_chunks without split-K)
+          const int c_lo = split_ * a.kpsplit / RS, c_hi = min(nchunks, c_lo + a.kpsplit / RS);
+          for (int cc = c_lo; cc < c_hi; ++cc) {
             mbar_wait(afull0 + 8 * ab, aph);
             tc_fence_after();
             if (bres && lane == 0 && j == 0) TRACE2(1, tcount);
@@ -697,7 +723,8 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
           tc_fence_after();
           const uint32_t d = tmem + acc * (uint32_t)a.n_tile + (uint32_t)(j * n_sub);
           uint32_t accum = 0;
-          const int split = tile / tiles_mn;
+          int split, tmn_;
+          split_of(a, tile, tiles_mn, split, tmn_);
           const int k_lo = split * a.kpsplit, k_hi = min(a.c_chunks * RS, k_lo + a.kpsplit);
           int cc = k_lo / RS, rs = k_lo - (k_lo / RS) * RS;
           int kv = min(4, (C - cc * 64 + 15) >> 4);
@@ -745,50 +772,22 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
     const int et = threadIdx.x - 32 * kEpiWarp0;  // 0..127
     uint32_t tcount = 0, acc = 0, tph = 0;
     if (a.sres) {
-      // all K channels' folded BN once per CTA (rounded up to the N tile;
+      // all K channels' BN shift once per CTA (rounded up to the N tile;
       // channels past K read the last one and are clipped at the store)
       const int kr = a.tiles_n * a.n_tile;
       for (int jj = et; jj < kr; jj += 128) {
         const int nj = min(jj, a.K - 1);
-        asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_scale + jj)), "f"(__ldg(a.scale + nj)) : "memory");
         asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_shift + jj)), "f"(__ldg(a.shift + nj)) : "memory");
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
     }
     for (int tile = cta; tile < tiles; tile += ncta, ++tcount) {
-      const int split = tile / tiles_mn, tmn = tile - split * tiles_mn;
+      int split, tmn;
+      split_of(a, tile, tiles_mn, split, tmn);
       const int m_blk = tmn / a.tiles_n, n_blk = tmn - m_blk * a.tiles_n;
       const int tp = m_blk / a.tiles_q, tq = m_blk - tp * a.tiles_q;
       const int p0 = tp * a.th, q0 = tq * a.tw, n0 = n_blk * a.n_tile;
       const int n_valid = min(a.n_tile, a.K - n0);
-      if (a.ksplit > 1) {
-        // split-K: raw fp32 partial sums to the workspace (scale/shift/ReLU
-        // are applied by conv_splitk_finalize after all splits)
-        mbar_wait(tfull0 + 8 * acc, tph);
-        __syncwarp();
-        tc_fence_after();
-        const uint32_t tbase = tmem + ((uint32_t)(lw * 32) << 16) + acc * (uint32_t)a.n_tile;
-        int p, q;
-        tile_pixel(a, m_blk, p0, q0, m, p, q);
-        const bool valid = p < a.P && q < a.Q;
-        float* wrow = a.ws + (size_t)split * a.ws_split + ((size_t)p * a.Q + q) * a.ws_ld + n0;
-        for (int col = 0; col < a.n_tile; col += 16) {
-          uint32_t r[16];
-          tmem_ld16(tbase + (uint32_t)col, r);
-          if (valid) {
-            uint4* d4 = reinterpret_cast<uint4*>(wrow + col);
-            d4[0] = make_uint4(r[0], r[1], r[2], r[3]);
-            d4[1] = make_uint4(r[4], r[5], r[6], r[7]);
-            d4[2] = make_uint4(r[8], r[9], r[10], r[11]);
-            d4[3] = make_uint4(r[12], r[13], r[14], r[15]);
-          }
-        }
-        tc_fence_before();
-        mbar_arrive(tempty0 + 8 * acc);
-        if (a.nacc == 2) acc ^= 1u;
-        if (acc == 0) tph ^= 1u;
-        continue;
-      }
       // staging tile of this tile (two alternate when out_bufs == 2, so the
       // bulk stores of tile i drain while tile i+1 is staged)
       const uint32_t ob = a.out_bufs == 2 ? (tcount & 1u) : 0u;
@@ -806,14 +805,13 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
           __syncwarp();
         }
       } else {
-        // previous tile fully copied out of sOut / s_scale (all 128 threads;
+        // previous tile fully copied out of sOut / s_shift (all 128 threads;
         // TMA-store mode: the bulk stores have finished reading sOut)
         if (a.tma_out && lane == 0) bulk_wait_read0();
         asm volatile("bar.sync 1, 128;" ::: "memory");
         if (!a.sres) {
           for (int jj = et; jj < a.n_tile; jj += 128) {
             const int nj = min(n0 + jj, a.K - 1);
-            asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_scale + jj)), "f"(__ldg(a.scale + nj)) : "memory");
             asm volatile("st.shared.f32 [%0], %1;" ::"r"(smem_u32(s_shift + jj)), "f"(__ldg(a.shift + nj)) : "memory");
           }
           asm volatile("bar.sync 1, 128;" ::: "memory");
@@ -839,7 +837,8 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
         // direct stores: each thread owns one output pixel (its TMEM lane)
         // and writes its n_valid channels as 16-byte vectors straight from
         // registers -- no staging, no proxy fence, no bulk-group waits
-        const float* scs = s_scale + (a.sres ? n0 : 0);
+        // (measured slower: warp-staged coalesced copy-out, Inception-1024
+        // HIOS-LP 0.86 -> 1.00 ms)
         const float* shs = s_shift + (a.sres ? n0 : 0);
         for (int jr = 0; jr < a.hk; ++jr) {  // output row jr of the tile's row group
         const uint32_t tbj = tbase + (uint32_t)(jr * a.n_tile);
@@ -855,18 +854,17 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
           uint32_t r0[16], r1[16];
           tmem_ld16_nw(tbj + (uint32_t)col, r0);
           if (two) tmem_ld16_nw(tbj + (uint32_t)col + 16u, r1);
-          float sc[32], sf[32];
+          float sf[32];
 #pragma unroll
           for (int q4 = 0; q4 < 8; ++q4) {
-            const uint4 u = lds128(smem_u32(scs + col + 4 * q4));
             const uint4 w = lds128(smem_u32(shs + col + 4 * q4));
-            sc[4 * q4] = __uint_as_float(u.x); sc[4 * q4 + 1] = __uint_as_float(u.y);
-            sc[4 * q4 + 2] = __uint_as_float(u.z); sc[4 * q4 + 3] = __uint_as_float(u.w);
             sf[4 * q4] = __uint_as_float(w.x); sf[4 * q4 + 1] = __uint_as_float(w.y);
             sf[4 * q4 + 2] = __uint_as_float(w.z); sf[4 * q4 + 3] = __uint_as_float(w.w);
           }
+          if (jr == 0 && col < 64) TRACE4(3 + 2 * (col >> 5));
           tmem_wait_pin(r0);
           pin16(r1);
+          if (jr == 0 && col < 64) TRACE4(4 + 2 * (col >> 5));
 #pragma unroll
           for (int hlf = 0; hlf < 2; ++hlf) {
             const int c16 = col + 16 * hlf;
@@ -874,14 +872,16 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
             const uint32_t* r = hlf ? r1 : r0;
             uint32_t pk[8];
 #pragma unroll
-            for (int e = 0; e < 8; ++e) {
-              float y0 = __uint_as_float(r[2 * e]) * sc[16 * hlf + 2 * e] + sf[16 * hlf + 2 * e];
-              float y1 = __uint_as_float(r[2 * e + 1]) * sc[16 * hlf + 2 * e + 1] + sf[16 * hlf + 2 * e + 1];
-              if (a.relu) { y0 = fmaxf(y0, 0.f); y1 = fmaxf(y1, 0.f); }
-              __nv_bfloat162 b2 = __floats2bfloat162_rn(y0, y1);
-              pk[e] = *reinterpret_cast<uint32_t*>(&b2);
-            }
+            for (int e = 0; e < 8; ++e)
+              pk[e] = bias_relu_pack(r[2 * e], r[2 * e + 1], sf[16 * hlf + 2 * e], sf[16 * hlf + 2 * e + 1], a.relu);
             if (!valid) continue;
+            if (a.st256 && c16 + 16 <= n_valid) {
+              // 32-byte stores (one full sector per thread and instruction:
+              // half the L1 store requests of 16-byte vectors)
+              st_global_256(o1 + c16, pk);
+              for (int d_ = 0; d_ < a.out2.n; ++d_) st_global_256(a.out2.p[d_] + pix * a.out2.ld[d_] + n0 + c16, pk);
+              continue;
+            }
 #pragma unroll
             for (int v8 = 0; v8 < 2; ++v8) {
               const int c8 = c16 + 8 * v8;
@@ -900,8 +900,10 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
               }
             }
           }
+          if (jr == 0 && col < 64) TRACE4(7 + (col >> 5));
         }
         }  // jr
+        TRACE4(9);
         tc_fence_before();
         mbar_arrive(tempty0 + 8 * acc);
         TRACE5(1, tcount);
@@ -914,20 +916,13 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
       // 16-byte chunks XOR-swizzled like the tensor map (bits 4.. ^= bits 7..)
       const uint32_t SWB = (uint32_t)a.out_sw * 2u, swm = SWB / 16u - 1u;
       const uint32_t sw_log = a.out_sw == 64 ? 6u : (a.out_sw == 32 ? 5u : 4u);
-      // resident scale/shift are indexed by absolute channel (n0 + col)
-      const uint32_t s_sc = smem_u32(s_scale) + (a.sres ? (uint32_t)n0 * 4u : 0u),
-                     s_sh = smem_u32(s_shift) + (a.sres ? (uint32_t)n0 * 4u : 0u);
+      // resident shifts are indexed by absolute channel (n0 + col)
+      const uint32_t s_sh = smem_u32(s_shift) + (a.sres ? (uint32_t)n0 * 4u : 0u);
       // one 16-column group: folded BN + ReLU -> bf16 -> staging tile
-      auto emit16 = [&](int col, const uint32_t (&r)[16], const float* sc, const float* sf) {
+      auto emit16 = [&](int col, const uint32_t (&r)[16], const float* sf) {
         uint32_t pk[8];
 #pragma unroll
-        for (int q = 0; q < 8; ++q) {
-          float y0 = __uint_as_float(r[2 * q]) * sc[2 * q] + sf[2 * q];
-          float y1 = __uint_as_float(r[2 * q + 1]) * sc[2 * q + 1] + sf[2 * q + 1];
-          if (a.relu) { y0 = fmaxf(y0, 0.f); y1 = fmaxf(y1, 0.f); }
-          __nv_bfloat162 b2 = __floats2bfloat162_rn(y0, y1);
-          pk[q] = *reinterpret_cast<uint32_t*>(&b2);
-        }
+        for (int q = 0; q < 8; ++q) pk[q] = bias_relu_pack(r[2 * q], r[2 * q + 1], sf[2 * q], sf[2 * q + 1], a.relu);
         if (a.tma_out) {
           const uint32_t slab = (uint32_t)col >> sw_log;
           const uint32_t cb = ((uint32_t)col - (slab << sw_log)) * 2u;  // byte in the slab row
@@ -948,21 +943,18 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
         uint32_t r0[16], r1[16];
         tmem_ld16_nw(tbase + (uint32_t)col, r0);
         if (two) tmem_ld16_nw(tbase + (uint32_t)col + 16u, r1);
-        float sc[32], sf[32];
+        float sf[32];
 #pragma unroll
         for (int q = 0; q < 8; ++q) {
-          const uint4 u = lds128(s_sc + (uint32_t)(col + 4 * q) * 4u);
           const uint4 w = lds128(s_sh + (uint32_t)(col + 4 * q) * 4u);
-          sc[4 * q] = __uint_as_float(u.x); sc[4 * q + 1] = __uint_as_float(u.y);
-          sc[4 * q + 2] = __uint_as_float(u.z); sc[4 * q + 3] = __uint_as_float(u.w);
           sf[4 * q] = __uint_as_float(w.x); sf[4 * q + 1] = __uint_as_float(w.y);
           sf[4 * q + 2] = __uint_as_float(w.z); sf[4 * q + 3] = __uint_as_float(w.w);
         }
         tmem_wait_pin(r0);
         pin16(r1);
         if (col < 16 * 6) TRACE4(3 + col / 32);
-        emit16(col, r0, sc, sf);
-        if (two) emit16(col + 16, r1, sc + 16, sf + 16);
+        emit16(col, r0, sf);
+        if (two) emit16(col + 16, r1, sf + 16);
       }
       tc_fence_before();
       mbar_arrive(tempty0 + 8 * acc);  // TMEM accumulator free for the next tile
@@ -1092,49 +1084,6 @@ __global__ void __launch_bounds__(kThreads, 1) conv_tc_group_kernel(const __grid
     case 4: conv_tc_group_op<4>(G); break;
     default: conv_tc_group_op<5>(G); break;
   }
-}
-
-// sum the split-K partials, folded BN + ReLU, bf16, 16-byte stores
-__global__ void conv_splitk_finalize(const float* __restrict__ ws, int ksplit, size_t ws_split, int ws_ld, int PQ,
-                                     int K, const float* __restrict__ scale, const float* __restrict__ shift,
-                                     int relu, bf16* out, int ldo, Dst<bf16> out2) {
-  pdl_enter();
-  const int KG = (K + 7) / 8;
-  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= PQ * KG) return;
-  const int pix = idx / KG, n = (idx - pix * KG) * 8;
-  float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
-  const float* src = ws + (size_t)pix * ws_ld + n;
-  for (int s = 0; s < ksplit; ++s) {
-    const float4 a0 = *reinterpret_cast<const float4*>(src + s * ws_split);
-    const float4 a1 = *reinterpret_cast<const float4*>(src + s * ws_split + 4);
-    acc[0] += a0.x; acc[1] += a0.y; acc[2] += a0.z; acc[3] += a0.w;
-    acc[4] += a1.x; acc[5] += a1.y; acc[6] += a1.z; acc[7] += a1.w;
-  }
-  __align__(16) bf16 v[8];
-#pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    const int nj = min(n + j, K - 1);
-    float y = acc[j] * __ldg(scale + nj) + __ldg(shift + nj);
-    v[j] = __float2bfloat16_rn(relu ? fmaxf(y, 0.f) : y);
-  }
-  bf16* d = out + (size_t)pix * ldo + n;
-  if (n + 8 <= K) {
-    *reinterpret_cast<uint4*>(d) = *reinterpret_cast<const uint4*>(v);
-    for (int d_ = 0; d_ < out2.n; ++d_)
-      *reinterpret_cast<uint4*>(out2.p[d_] + (size_t)pix * out2.ld[d_] + n) = *reinterpret_cast<const uint4*>(v);
-  } else {
-    for (int j = 0; n + j < K; ++j) {
-      d[j] = v[j];
-      for (int d_ = 0; d_ < out2.n; ++d_) out2.p[d_][(size_t)pix * out2.ld[d_] + n + j] = v[j];
-    }
-  }
-}
-
-void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st) {
-  const int PQ = a.P * a.Q, KG = (a.K + 7) / 8;
-  launch_pdl(conv_splitk_finalize, dim3((PQ * KG + 255) / 256), dim3(256), 0, st, (const float*)a.ws, a.ksplit,
-             a.ws_split, a.ws_ld, PQ, a.K, a.scale, a.shift, a.relu, a.out, a.ldo, a.out2);
 }
 
 size_t conv_tc_smem_bytes(const ConvTcArgs& a) {

@@ -55,6 +55,8 @@ static thread_local int g_num_sms = 148;
 // group-context build only), so a stage's convs can share one launch
 static thread_local std::vector<ConvTcOp>* g_tc_out = nullptr;
 static thread_local size_t* g_tc_smem = nullptr;
+// where conv_closure<bf16> records its tile plan (OpExec::plan / plan_solo)
+static thread_local int* g_plan_out = nullptr;
 
 void ck(cudaError_t e, const char* what) {
   if (e != cudaSuccess) fail(HIOS_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
@@ -267,14 +269,19 @@ static void* upload(LGpu& L, const std::vector<T>& h) {
 
 // conv weights W[k][c][r][s] -> tensor-core layout [k][r*S+s][Cp] (Cp = C rounded to 8, zero pad)
 //                             -> SIMT layout [k][r][s][c]
+// fold (tcgen05 convs): the folded-BN scale of output channel k is multiplied
+// into its weights before rounding to bf16 (scale * (W * x) = (scale W) * x),
+// so the conv_tc epilogue adds the shift only
 template <typename T>
-static std::vector<T> conv_layout(const float* W, int K, int C, int R, int S, int Cp) {
+static std::vector<T> conv_layout(const float* W, int K, int C, int R, int S, int Cp, const float* fold = nullptr) {
   std::vector<T> out((size_t)K * R * S * Cp, to_dev_t<T>(0.f));
-  for (int k = 0; k < K; ++k)
+  for (int k = 0; k < K; ++k) {
+    const float f = fold ? fold[k] : 1.f;
     for (int c = 0; c < C; ++c)
       for (int r = 0; r < R; ++r)
         for (int s2 = 0; s2 < S; ++s2)
-          out[((size_t)k * R * S + r * S + s2) * Cp + c] = to_dev_t<T>(W[(((size_t)k * C + c) * R + r) * S + s2]);
+          out[((size_t)k * R * S + r * S + s2) * Cp + c] = to_dev_t<T>(f * W[(((size_t)k * C + c) * R + r) * S + s2]);
+  }
   return out;
 }
 
@@ -305,7 +312,7 @@ static void upload_weights_T(Executor& ex, int v) {
               for (int s2 = 0; s2 < o.kw; ++s2) {
                 const int ch = ((r & 1) * 2 + (s2 & 1)) * C + c;
                 w2[((size_t)k * R2 * S2 + (r >> 1) * S2 + (s2 >> 1)) * Cp2 + ch] =
-                    to_dev_t<T>(o.weight[(((size_t)k * C + c) * o.kh + r) * o.kw + s2]);
+                    to_dev_t<T>(o.scale[k] * o.weight[(((size_t)k * C + c) * o.kh + r) * o.kw + s2]);
               }
         x.w = upload(L, w2);
         if (rup(4 * C, 8) == 16 && S2 <= 4) {
@@ -323,7 +330,7 @@ static void upload_weights_T(Executor& ex, int v) {
         x.shift.push_back((float*)upload(L, o.shift));
         break;
       }
-      x.w = upload(L, conv_layout<T>(o.weight.data(), o.out_c, o.in_c, o.kh, o.kw, Cp));
+      x.w = upload(L, conv_layout<T>(o.weight.data(), o.out_c, o.in_c, o.kh, o.kw, Cp, tc ? o.scale.data() : nullptr));
       if (small_c_conv(o)) x.w_small = (float*)upload(L, conv_layout<float>(o.weight.data(), o.out_c, o.in_c, o.kh, o.kw, o.in_c));
       x.scale.push_back((float*)upload(L, o.scale));
       x.shift.push_back((float*)upload(L, o.shift));
@@ -340,7 +347,8 @@ static void upload_weights_T(Executor& ex, int v) {
         off += (size_t)c * RS;
         x.dw.push_back((float*)upload(L, dw));
         const int Cp = tc ? rup(c, 64) : rup(c, 16);
-        x.pw.push_back(upload(L, conv_layout<T>(o.weight.data() + off, o.out_c, c, 1, 1, Cp)));
+        x.pw.push_back(upload(L, conv_layout<T>(o.weight.data() + off, o.out_c, c, 1, 1, Cp,
+                                                tc ? o.scale.data() + (size_t)r * o.out_c : nullptr)));
         off += (size_t)o.out_c * c;
         std::vector<float> sc(o.scale.begin() + (size_t)r * o.out_c, o.scale.begin() + (size_t)(r + 1) * o.out_c);
         std::vector<float> sh(o.shift.begin() + (size_t)r * o.out_c, o.shift.begin() + (size_t)(r + 1) * o.out_c);
@@ -619,16 +627,11 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
   }
   const int n_stage_steps = (KI + c.kps - 1) / c.kps;
   c.stages = std::max(2, std::min(c.stages, std::max(n_stage_steps, 2)));
-  // split-K (tap mode): deep layers with few output tiles can split their
-  // K-steps across CTAs; fp32 partials are reduced by a finalize kernel that
-  // applies the folded BN + ReLU.
+  // no split-K (measured: a workspace + finalize kernel and a cluster /
+  // distributed-shared-memory reduction both lost under HIOS stages,
+  // DESIGN.md §6)
   c.ksplit = 1;
   c.kpsplit = KI;
-  const int tiles = c.tiles_m * c.tiles_n;
-  // Measured (Inception-v3 1024, HIOS w=4, same box): split-K makes a deep
-  // small-spatial conv faster alone (7c_3x3 18.3 -> 14.5 us) but the step
-  // slower (0.865 -> 0.88-0.90 ms): the extra CTAs and the finalize launch
-  // crowd out the stage's concurrent ops.  So it is opt-in (HIOS_SPLITK=1).
   if (c.hk > 1) {
     // the kernel's row-group loops exist only for the unrolled (R, S, kps)
     // shapes (conv_tc.cu halo_taps_ring / halo_taps_bres) and the direct-store
@@ -640,18 +643,6 @@ static ConvTcArgs plan_conv_tc(int P, int Q, int K, int C, int R, int S, int sh,
     const bool ring_ok1 = R == 1 && S == 1 && c.kps == 1;
     if (c.epi != 2 || !(c.bres ? bres_ok : (ring_ok || ring_ok1)) || (c.nacc == 1 && c.bres))
       return plan_conv_tc(P, Q, K, C, R, S, sh, sw, dh, dw, false);
-  }
-  if (!c.halo && getenv("HIOS_SPLITK") && tiles < 48 && KI >= 16) {
-    // at most one wave of CTAs, >= ~6 K-steps each; splits may start at any
-    // (chunk, tap) K-step
-    const int cta_cap = g_num_sms;
-    const int min_k = 6;
-    int want = std::max(1, (cta_cap * c.occ) / tiles);
-    want = std::min(want, KI / min_k);
-    if (want >= 2) {
-      c.kpsplit = (KI + want - 1) / want;
-      c.ksplit = (KI + c.kpsplit - 1) / c.kpsplit;
-    }
   }
   return c;
 }
@@ -719,6 +710,11 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
   a.dbg = 0;
   a.out = (bf16*)out.p; a.ldo = out.ldc;
   a.out2 = dst_of<bf16>(out2);
+  // 256-bit epilogue stores need every pixel row of every destination
+  // 32-byte aligned (16-channel groups of the tile start at n0 % 16 == 0)
+  a.st256 = ((uintptr_t)out.p % 32 == 0 && out.ldc % 16 == 0 && !getenv("HIOS_NOST256")) ? 1 : 0;
+  for (auto& v : out2)
+    if ((uintptr_t)v.p % 32 != 0 || v.ldc % 16 != 0) a.st256 = 0;
   // epilogue by TMA bulk-tensor stores: output tensor map {K, Q, P} over the
   // destination slice (clips the ragged pixel / channel edges of a tile)
   CUtensorMap mo = mx, mo2 = mx;
@@ -738,20 +734,12 @@ std::function<void(cudaStream_t)> conv_closure<bf16>(Executor& ex, const View& i
     if (!a.tma_out) a.epi = 0;
   }
   const size_t smem = conv_tc_smem_bytes(a);
-  const int grid = std::min(a.tiles_m * a.tiles_n * a.ksplit, g_num_sms * a.occ);
-  if (a.ksplit > 1) {
-    a.ws_ld = a.tiles_n * a.n_tile;
-    a.ws_split = (size_t)P * Q * a.ws_ld;
-    void* ws = nullptr;
-    ck(cudaMalloc(&ws, a.ws_split * a.ksplit * sizeof(float)), "cudaMalloc split-K workspace");
-    ex.lg[ex.cur_lgpu].allocs.push_back(ws);
-    a.ws = (float*)ws;
-    nk += 2;
-    return [mx, mw, a, smem, grid](cudaStream_t st) {
-      launch_conv_tc(mx, mw, mx, mx, a, grid, smem, st);
-      launch_conv_splitk_finalize(a, st);
-    };
+  if (g_plan_out) {
+    const int pl[8] = {a.vgrid ? 3 : (a.halo ? 2 : 1), a.n_tile, a.tiles_m * a.tiles_n, a.epi, a.st256, a.hk,
+                       a.stages, a.kps};
+    std::memcpy(g_plan_out, pl, sizeof(pl));
   }
+  const int grid = std::min(a.tiles_m * a.tiles_n * a.ksplit, g_num_sms * a.occ);
   nk += 1;
   if (g_tc_out) {
     ConvTcOp op;
@@ -1016,9 +1004,11 @@ void Executor::build_op_closures(int v) {
   ck(cudaSetDevice(lg[l].dev), "cudaSetDevice");
   cur_lgpu = l;
   g_num_sms = lg[l].num_sms;
+  OpExec& x = ox[v];
+  g_plan_out = x.plan;
   if (g.dtype == HIOS_BF16) build_op<bf16>(*this, v);
   else build_op<float>(*this, v);
-  OpExec& x = ox[v];
+  g_plan_out = nullptr;
   const int k = g.ops[v].kind;
   if (g.dtype == HIOS_BF16 && (k == HIOS_OP_CONV || k == HIOS_OP_SEPCONV)) {
     auto run = x.run;
@@ -1026,7 +1016,9 @@ void Executor::build_op_closures(int v) {
     auto tc = x.tc;
     const size_t tcs = x.tc_smem;
     g_conv_solo = true;
+    g_plan_out = x.plan_solo;
     build_op<bf16>(*this, v);
+    g_plan_out = nullptr;
     g_conv_solo = false;
     x.run_solo = x.run;
     x.n_kernels_solo = x.n_kernels;

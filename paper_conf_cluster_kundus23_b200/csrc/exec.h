@@ -64,6 +64,11 @@ struct OpExec {
   // tap-mode convs take narrower N tiles there (more CTAs); empty = run
   std::function<void(cudaStream_t)> run_solo;
   int n_kernels_solo = 0;
+  // tcgen05 conv tile plan (hios_op_plan): {A mode (1 tap, 2 halo, 3 vgrid
+  // halo), n_tile, output tiles, epilogue mode, 256-bit stores, rows per
+  // tile, stages, K-steps per stage}; [0] = 0 for any other op / path
+  int plan[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  int plan_solo[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   // a plain tcgen05 conv (one launch, group-context plan): its descriptor for
   // the stage's grouped launch (conv_tc_group_kernel); empty otherwise
   std::vector<ConvTcOp> tc;

@@ -71,12 +71,9 @@ struct ConvTcArgs {
   int n_mma;                 // MMA warps splitting the N tile (n_tile % (16 * n_mma) == 0)
   int occ;                   // co-resident CTAs per SM the smem plan allows (1 or 2)
   int dbg;                   // debug switches (timing experiments; 0 in production)
-  int ksplit, kpsplit;       // split-K: splits and K-steps (chunk x tap) per split
+  int ksplit, kpsplit;       // K splits (1) and K-steps (chunk x tap) per split
   int kps;                   // K-steps (64-channel x tap) per pipeline stage
-  float* ws;                 // split-K fp32 workspace [ksplit][P*Q][ws_ld]
-  size_t ws_split;           // elements per split
-  int ws_ld;                 // row pitch (tiles_n * n_tile)
-  const float* scale;  // [K]
+  const float* scale;  // [K] (conv_tc: folded into the weights at upload, unused by the kernel)
   const float* shift;  // [K]
   bf16* out;  int ldo; // primary output (channel offset applied)
   Dst<bf16> out2;      // remote replicas (fused cross-GPU stores)
@@ -102,6 +99,7 @@ struct ConvTcArgs {
   int hk_px;  // hk > 1 for a 1x1 conv: the tile is 2 x 128 consecutive pixels of one row (box 256 px)
   int nacc;  // TMEM accumulator sets (2: the epilogue of tile i overlaps the MMAs of tile i+1; 1 when
              // 2 * hk * n_tile > 512 columns)
+  int st256;  // direct-store epilogue: every destination 32-byte aligned per pixel (256-bit stores)
 };
 constexpr int kScaleRes = 512;
 constexpr int kMaxABufs = 6;  // halo-mode input boxes in flight
@@ -179,7 +177,6 @@ struct ConvTcGroup {
   int cta0[kMaxGroup + 1];  // op i owns CTAs [cta0[i], cta0[i+1])
 };
 void launch_conv_tc_group(const ConvTcGroup& G, size_t smem, cudaStream_t st);
-void launch_conv_splitk_finalize(const ConvTcArgs& a, cudaStream_t st);
 __host__ __device__ inline uint32_t halo_bytes_of(int R, int halo_w) {
   return ((uint32_t)R * halo_w * 128u + 1023u) & ~1023u;
 }

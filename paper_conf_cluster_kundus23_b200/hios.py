@@ -80,6 +80,7 @@ def load() -> C.CDLL:
         "hios_run_timed": [VP, VP, VP, VP, P(I64)],
         "hios_read_op_output": [VP, I32, P(C.c_float), I64],
         "hios_kernel_count": [VP, P(I64)],
+        "hios_op_plan": [VP, I32, I32, P(I32)],
         "hios_time_ops": [VP, I32, I64, P(I64)],
         "hios_schedule_transport": [VP, I32],
         "hios_schedule_stage_mode": [VP, I32],
@@ -432,6 +433,14 @@ def hios_kernel_count(s: Schedule) -> int:
     v = C.c_int64()
     _ck(load().hios_kernel_count(s.h, C.byref(v)))
     return v.value
+
+
+def hios_op_plan(s: Schedule, op: int, solo: bool = False) -> dict:
+    """The tcgen05 conv tile plan of `op` (hios_op_plan); mode 0 = no tcgen05 conv."""
+    v = (C.c_int32 * 8)()
+    _ck(load().hios_op_plan(s.h, op, 1 if solo else 0, v))
+    keys = ("mode", "n_tile", "tiles", "epilogue", "st256", "rows", "stages", "kps")
+    return dict(zip(keys, list(v)))
 
 
 def hios_abi_version() -> int:

@@ -120,41 +120,21 @@ CONV_CASES = [
     (64, 80, 150, 130, 1, 1, 1, 0, 0),
 ]
 
-SPLITK_CASES = [
-    (448, 384, 19, 19, 3, 3, 2, 1, 1),    # split boundaries inside a chunk's taps (stride 2: tap mode)
-    (2048, 384, 8, 8, 1, 1, 1, 0, 0),
-    (288, 384, 35, 35, 3, 3, 2, 0, 0),
-]
-
-
-def conv_case(dtype, case):
-    """(normwise error vs the oracle, kernels in the schedule's graph)."""
-    C, K, H, Wd, kh, kw, s, ph, pw = case
+def test_op_plan_reports_the_conv_tile_plan():
+    """hios_op_plan: a tcgen05 conv reports its A-operand mode and N tile; other
+    ops report zeros."""
+    C, K, H, Wd = 64, 96, 40, 300
     g = graphs.GraphSpec("conv", C, H, Wd)
     x0 = g.input()
-    g.conv(x0, K, (kh, kw), s=s, p=(ph, pw), relu=1)
+    c = g.conv(x0, K, (3, 3), s=1, p=(1, 1), relu=1)
+    g.maxpool(c, 3, 2)
     W = gen.make_weights(g)
-    x = gen.make_input(g) - 0.5
-    _, S, y = run_graph_gpu(g, W, x, dtype, profile=False)
-    ref = infer.run_graph(g, W, x)[1]
-    return nerr(y.reshape(ref.shape), ref), hios().hios_kernel_count(S)
-
-
-@pytest.mark.parametrize("dtype", ["bf16", "f32"])
-@pytest.mark.parametrize("case", CONV_CASES)
-def test_conv_parity(dtype, case):
-    err, _ = conv_case(dtype, case)
-    assert err <= TOL[dtype] / (4 if dtype == "bf16" else 1)
-
-
-@pytest.mark.parametrize("case", SPLITK_CASES)
-def test_conv_parity_splitk(case, monkeypatch):
-    """The opt-in split-K path (K-step-granular splits + finalize kernel)."""
-    _, n_plain = conv_case("bf16", case)
-    monkeypatch.setenv("HIOS_SPLITK", "1")
-    err, n_split = conv_case("bf16", case)
-    assert n_split == n_plain + 1  # the finalize kernel: split-K really ran
-    assert err <= TOL["bf16"] / 4
+    x = gen.make_input(g)
+    _, S, _ = run_graph_gpu(g, W, x, "bf16", profile=False)
+    h = hios()
+    p = h.hios_op_plan(S, 1, solo=True)
+    assert p["mode"] == 2 and p["n_tile"] % 16 == 0 and p["tiles"] >= 40 and p["stages"] >= 2, p
+    assert h.hios_op_plan(S, 2)["mode"] == 0
 
 
 SEP_CASES = [

@@ -13,6 +13,8 @@ from workloads import gen, graphs  # noqa: E402
 
 SHAPES = [  # name, C, K, H, W, kh, kw, s, ph, pw
     ("stem2a", 32, 32, 511, 511, 3, 3, 1, 0, 0),
+    ("tiny1x1", 64, 64, 11, 11, 1, 1, 1, 0, 0),     # one tile, one K-step: the fixed cost of a launch
+    ("tiny1x1_c256", 256, 64, 11, 11, 1, 1, 1, 0, 0),
     ("4a", 80, 192, 254, 254, 3, 3, 1, 0, 0),
     ("5b_5x5", 48, 64, 125, 125, 5, 5, 1, 2, 2),
     ("5b_1x1", 192, 64, 125, 125, 1, 1, 1, 0, 0),
@@ -21,6 +23,10 @@ SHAPES = [  # name, C, K, H, W, kh, kw, s, ph, pw
     ("6e_1x7", 192, 192, 62, 62, 1, 7, 1, 0, 3),
     ("7c_1x1", 2048, 384, 30, 30, 1, 1, 1, 0, 0),
     ("7c_3x3", 448, 384, 30, 30, 3, 3, 1, 1, 1),
+    ("7c_1x3", 384, 384, 30, 30, 1, 3, 1, 0, 1),
+    ("7c_pool", 2048, 192, 30, 30, 1, 1, 1, 0, 0),
+    ("6e_7x1", 192, 192, 62, 62, 7, 1, 1, 3, 0),
+    ("7a_s2", 192, 320, 62, 62, 3, 3, 2, 0, 0),
     # Inception-v3 at 4096^2 (compute-heavy)
     ("4a_4096", 80, 192, 1022, 1022, 3, 3, 1, 0, 0),
     ("2a_4096", 32, 32, 2047, 2047, 3, 3, 1, 0, 0),
