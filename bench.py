@@ -393,6 +393,7 @@ def measure_workload(h, torch, model, sz, M, args, dev, stream, flush, pk, dtype
         else:
             Sx = h.hios_schedule_lp(Gs, m_, w_)
         t_s = time.perf_counter() - t0
+        h.hios_schedule_stage_mode(Sx, args.stage_mode)
         if m_ > 1:
             ndev = torch.cuda.device_count()
             h.hios_schedule_place(Sx, [i % ndev for i in range(m_)])
@@ -400,6 +401,8 @@ def measure_workload(h, torch, model, sz, M, args, dev, stream, flush, pk, dtype
             dout = torch.empty(h.hios_output_numel(Sx), dtype=torch.float32, device=f"cuda:{dev}")
         for _ in range(3):
             h.hios_run_device(Sx, din.data_ptr(), dout.data_ptr(), stream.cuda_stream)
+        if name == "hios_lp":
+            row["stage_mode"] = h.hios_schedule_stage_mode_used(Sx)
         ev = []
         for i in range(max(5, args.steps // 3)):
             flush.fill_(float(i))
@@ -451,8 +454,10 @@ def main():
                     help="extra input sizes timed on 1 GPU (HIOS-LP / sequential / IOS-style), '' to skip")
     ap.add_argument("--transport", default="peer", choices=["peer", "copy", "nccl"],
                     help="cross-GPU edge transport (N > 1): fused peer stores, copy engine, NCCL send/recv")
-    ap.add_argument("--stage-mode", default="streams", choices=["streams", "grouped"],
-                    help="stage execution: per-op streams, or one grouped conv launch per stage (f2)")
+    ap.add_argument("--stage-mode", default="auto", choices=["streams", "grouped", "dataflow", "auto"],
+                    help="stage execution: per-op streams joined per stage, one grouped conv launch per stage "
+                         "(f2), per-op input waits (dataflow), or auto (both captured, the faster kept after "
+                         "the first run); applied to every schedule the bench times")
     ap.add_argument("--ios-states", type=int, default=1 << 14,
                     help="state budget of the exact IOS DP in the size sweep (its t(S) are profiled lazily: "
                          "NASNet-A 2048^2 needs 2^18, ~5 min)")
@@ -558,6 +563,8 @@ def main():
     for _ in range(args.warmup):
         run_dev(S)
     barrier()
+    if args.stage_mode == "auto":
+        cfg["stage_mode"] = "auto->" + h.hios_schedule_stage_mode_used(S)
     clk = Clocks(dev)
     barrier()
     ncu = bool(os.environ.get("HIOS_NCU"))
@@ -678,6 +685,7 @@ def main():
                 extra[name] = {"unavailable": str(ex)}
                 continue
             t_sched_x = time.perf_counter() - t_s0
+            h.hios_schedule_stage_mode(Sx, args.stage_mode)
             if m_ > 1:
                 ndev = torch.cuda.device_count()
                 h.hios_schedule_place(Sx, [i % ndev for i in range(m_)])

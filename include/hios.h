@@ -241,9 +241,28 @@ hios_status hios_schedule_transport(hios_schedule s, int32_t transport);
  *     (hios_profile measures t(S) with streams.)  (Measured on one B200,
  *     Inception-v3 HIOS-LP w = 5: 0.80 ms grouped vs 0.74 ms streams at 1024^2;
  *     DESIGN.md §6.)
+ *   HIOS_STAGE_DATAFLOW: the stages' ops in the schedule's order, op i of a
+ *     stage on stream i of its GPU, each waiting only for its own inputs and
+ *     the previous op of its stream instead of the whole previous stage (the
+ *     stage boundary join of P:86 relaxed to the data dependencies; at
+ *     most |S| <= w ops in flight per GPU as in the stage model).
+ *   HIOS_STAGE_AUTO: both STREAMS and DATAFLOW graphs are captured; the first
+ *     run (its results are STREAMS') then replays each 9 times and keeps the
+ *     faster (median wall time of launch + synchronize) for every later run --
+ *     measured selection, like the profiler's t(S).  One process
+ *     driving all its logical GPUs only (otherwise STREAMS).
  * Errors: HIOS_E_INVALID (unknown mode), HIOS_E_STATE (already run). */
-typedef enum { HIOS_STAGE_STREAMS = 0, HIOS_STAGE_GROUPED = 1 } hios_stage_mode;
+typedef enum {
+  HIOS_STAGE_STREAMS = 0,
+  HIOS_STAGE_GROUPED = 1,
+  HIOS_STAGE_DATAFLOW = 2,
+  HIOS_STAGE_AUTO = 3
+} hios_stage_mode;
 hios_status hios_schedule_stage_mode(hios_schedule s, int32_t mode);
+/* The stage mode the schedule's graphs execute (after the first run; AUTO
+ * resolves to STREAMS or DATAFLOW).  Errors: HIOS_E_INVALID, HIOS_E_STATE
+ * (not run yet). */
+hios_status hios_schedule_stage_mode_used(hios_schedule s, int32_t* mode);
 
 /* NCCL transport set-up.  hios_nccl_unique_id writes a 128-byte ncclUniqueId
  * (call on one rank, broadcast the bytes); hios_schedule_nccl_init creates

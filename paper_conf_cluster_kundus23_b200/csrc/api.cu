@@ -275,7 +275,9 @@ hios_status hios_schedule_transport(hios_schedule s, int32_t transport) {
 hios_status hios_schedule_stage_mode(hios_schedule s, int32_t mode) {
   return guard([&] {
     NEED(s, HIOS_E_INVALID, "NULL schedule");
-    NEED(mode == HIOS_STAGE_STREAMS || mode == HIOS_STAGE_GROUPED, HIOS_E_INVALID, "unknown stage mode");
+    NEED(mode == HIOS_STAGE_STREAMS || mode == HIOS_STAGE_GROUPED || mode == HIOS_STAGE_DATAFLOW ||
+             mode == HIOS_STAGE_AUTO,
+         HIOS_E_INVALID, "unknown stage mode");
     NEED(!s->s->exec, HIOS_E_STATE, "set the stage mode before the first run");
     s->s->stage_mode = mode;
   });
@@ -505,6 +507,14 @@ hios_status hios_time_ops(hios_schedule s, int32_t reps, int64_t flush_bytes, in
     auto& E = ensure_exec(*s->s);
     if (!s->s->owner.empty()) check_remote_mapped(E);
     E.time_ops(reps, flush_bytes, op_ns);
+  });
+}
+
+hios_status hios_schedule_stage_mode_used(hios_schedule s, int32_t* mode) {
+  return guard([&] {
+    NEED(s && mode, HIOS_E_INVALID, "NULL argument");
+    NEED(s->s->exec && s->s->exec->captured, HIOS_E_STATE, "run first");
+    *mode = s->s->exec->mode_used;
   });
 }
 

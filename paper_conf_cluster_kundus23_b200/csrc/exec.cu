@@ -15,6 +15,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdlib>
+#include <chrono>
 #include <cstring>
 #include <numeric>
 #include <set>
@@ -68,6 +69,9 @@ static inline int64_t rup64(int64_t x, int64_t m) { return (x + m - 1) / m * m; 
 Executor::Executor(Schedule& sch) : s(sch), g(*sch.g), M(sch.M) {
   esz = g.dtype == HIOS_BF16 ? 2 : 4;
   group_convs = sch.stage_mode == HIOS_STAGE_GROUPED;
+  dataflow = sch.stage_mode == HIOS_STAGE_DATAFLOW;
+  auto_pending = sch.stage_mode == HIOS_STAGE_AUTO;
+  mode_used = auto_pending ? HIOS_STAGE_STREAMS : sch.stage_mode;
   transport = sch.transport;
   int ndev = 0;
   ck(cudaGetDeviceCount(&ndev), "cudaGetDeviceCount");
@@ -95,6 +99,8 @@ Executor::~Executor() {
     }
     if (L.gexec) cudaGraphExecDestroy(L.gexec);
     if (L.gexec_timed) cudaGraphExecDestroy(L.gexec_timed);
+    if (L.gexec_alt) cudaGraphExecDestroy(L.gexec_alt);
+    if (L.gexec_timed_alt) cudaGraphExecDestroy(L.gexec_timed_alt);
     for (auto st : L.streams) cudaStreamDestroy(st);
     if (L.ev_fork) cudaEventDestroy(L.ev_fork);
     for (auto e : L.ev_join) cudaEventDestroy(e);
@@ -1125,12 +1131,13 @@ static std::vector<int> partition_ctas(const std::vector<int>& tiles, const std:
 }
 
 void Executor::enqueue_stage(int l, const std::vector<int>& S, bool timed, int64_t& nk,
-                             const std::function<void(int, cudaStream_t)>& post) {
+                             const std::function<void(int, cudaStream_t)>& post, cudaStream_t lane,
+                             bool singleton) {
   LGpu& L = lg[l];
-  cudaStream_t s0 = L.streams[0];
+  cudaStream_t s0 = lane ? lane : L.streams[0];
   auto run_one = [&](int v, cudaStream_t st) {
     if (timed) ck(cudaEventRecordWithFlags(op_ev0[v], st, cudaEventRecordExternal), "event record");
-    const bool solo = S.size() == 1 && ox[v].run_solo;
+    const bool solo = singleton && S.size() == 1 && ox[v].run_solo;
     (solo ? ox[v].run_solo : ox[v].run)(st);
     if (timed) ck(cudaEventRecordWithFlags(op_ev1[v], st, cudaEventRecordExternal), "event record");
     nk += solo ? ox[v].n_kernels_solo : ox[v].n_kernels;
@@ -1286,40 +1293,78 @@ void Executor::capture_device(const std::vector<int>& ls, bool timed) {
     for (int j = 0; j < (int)s.Q[l].size(); ++j) order.emplace_back(rank[l][j], l, j);
   std::sort(order.begin(), order.end());
   cur_graph = lset;
+  // a cross-GPU input u of an op on logical GPU l, waited for on stream st
+  auto wait_remote = [&](int u, int l, cudaStream_t st) {
+    const int p = s.gpu_of[u];
+    if (lset.count(p)) {
+      ck(cudaStreamWaitEvent(st, edge_event(u, l), 0), "wait edge");
+    } else if (flag_index[u][l] < 0) {  // NCCL: post up to this receive, then wait for it
+      for (size_t i = 0; i < acts.size(); ++i) {
+        const NcclXfer& x = xfers[acts[i]];
+        if (x.u == u && x.dst == l) {
+          post(std::max(next, i + 1));
+          ck(cudaStreamWaitEvent(st, x.ev_recv, 0), "wait recv");
+        }
+      }
+    } else {
+      launch_wait(lg[l].sync, lg[l].sync + 1 + M + flag_index[u][l], 0, st);
+      ++nk;
+    }
+  };
+  auto deliver = [&](int v, cudaStream_t st) {
+    nk += enqueue_deliver(*this, v, st);
+    for (int k : acts)
+      if (xfers[k].u == v && lset.count(xfers[k].src)) ready[k] = 1;
+  };
+  // dataflow stage mode: op i of a stage runs on lane (stream) i and waits only
+  // for its own inputs (done events of same-GPU producers on other lanes) and
+  // the previous op of its lane -- no join at the stage boundary
+  std::vector<char> lanes_forked(M, 0);
   for (auto& it : order) {
     const int l = std::get<1>(it), j = std::get<2>(it);
     LGpu& L = lg[l];
     cudaStream_t s0 = L.streams[0];
     const auto& S = s.Q[l][j];
+    if (dataflow) {
+      if (!lanes_forked[l]) {
+        lanes_forked[l] = 1;
+        ck(cudaEventRecord(L.ev_fork, s0), "fork lanes");
+        for (size_t k = 1; k < L.streams.size(); ++k) ck(cudaStreamWaitEvent(L.streams[k], L.ev_fork, 0), "fork");
+      }
+      for (size_t i = 0; i < S.size(); ++i) {
+        const int v = S[i];
+        cudaStream_t st = L.streams[i];
+        std::set<int> ins;
+        for (int e : g.ops[v].in_edges) ins.insert(g.edges[e].src);
+        for (int u : ins) {
+          if (s.gpu_of[u] != l) wait_remote(u, l, st);
+          else if (lane_of[u] != (int)i && g.ops[u].kind != HIOS_OP_INPUT)
+            ck(cudaStreamWaitEvent(st, done_ev[u], 0), "wait input");
+        }
+        enqueue_stage(l, std::vector<int>{v}, timed, nk, deliver, st, S.size() == 1);
+        ck(cudaEventRecord(done_ev[v], st), "done");
+        lane_of[v] = (int)i;
+      }
+      continue;
+    }
     std::set<int> waits;
     for (int v : S)
       for (int e : g.ops[v].in_edges) {
         const int u = g.edges[e].src;
         if (s.gpu_of[u] != l) waits.insert(u);
       }
-    for (int u : waits) {
-      const int p = s.gpu_of[u];
-      if (lset.count(p)) {
-        ck(cudaStreamWaitEvent(s0, edge_event(u, l), 0), "wait edge");
-      } else if (flag_index[u][l] < 0) {  // NCCL: post up to this receive, then wait for it
-        for (size_t i = 0; i < acts.size(); ++i) {
-          const NcclXfer& x = xfers[acts[i]];
-          if (x.u == u && x.dst == l) {
-            post(std::max(next, i + 1));
-            ck(cudaStreamWaitEvent(s0, x.ev_recv, 0), "wait recv");
-          }
-        }
-      } else {
-        launch_wait(L.sync, L.sync + 1 + M + flag_index[u][l], 0, s0);
-        ++nk;
+    for (int u : waits) wait_remote(u, l, s0);
+    enqueue_stage(l, S, timed, nk, deliver);
+  }
+  if (dataflow)
+    for (int l : ls) {
+      LGpu& L = lg[l];
+      if (!lanes_forked[l]) continue;
+      for (size_t k = 1; k < L.streams.size(); ++k) {
+        ck(cudaEventRecord(L.ev_join[k], L.streams[k]), "join lane");
+        ck(cudaStreamWaitEvent(L.streams[0], L.ev_join[k], 0), "join lane wait");
       }
     }
-    enqueue_stage(l, S, timed, nk, [&](int v, cudaStream_t st) {
-      nk += enqueue_deliver(*this, v, st);
-      for (int k : acts)
-        if (xfers[k].u == v && lset.count(xfers[k].src)) ready[k] = 1;
-    });
-  }
   cur_graph.clear();
   if (!acts.empty()) {
     post(acts.size());
@@ -1354,6 +1399,8 @@ void Executor::capture() {
   if (op_ev0.empty()) {
     op_ev0.assign(g.n, nullptr);
     op_ev1.assign(g.n, nullptr);
+    done_ev.assign(g.n, nullptr);
+    lane_of.assign(g.n, -1);
   }
   kernels_per_run = 0;
   for (int l = 0; l < M; ++l) {
@@ -1364,13 +1411,69 @@ void Executor::capture() {
       if (s.gpu_of[v] == l && !op_ev0[v]) {
         ck(cudaEventCreate(&op_ev0[v]), "event");
         ck(cudaEventCreate(&op_ev1[v]), "event");
+        ck(cudaEventCreateWithFlags(&done_ev[v], cudaEventDisableTiming), "event");
       }
   }
-  for (auto& kv : graphs_by_dev) {
-    ck(cudaSetDevice(kv.first), "cudaSetDevice");
-    for (int timed = 0; timed < 2; ++timed) capture_device(kv.second, timed != 0);
+  // HIOS_STAGE_AUTO (one process driving all its GPUs): the dataflow variant
+  // is captured first and parked in gexec*_alt, then the streams variant
+  const bool both = auto_pending && std::all_of(lg.begin(), lg.end(), [](const LGpu& L) { return L.local; });
+  if (!both) auto_pending = false;
+  for (int pass = both ? 0 : 1; pass < 2; ++pass) {
+    dataflow = pass == 0 ? true : (both ? false : dataflow);
+    const int64_t kpr = kernels_per_run;
+    for (auto& kv : graphs_by_dev) {
+      ck(cudaSetDevice(kv.first), "cudaSetDevice");
+      for (int timed = 0; timed < 2; ++timed) capture_device(kv.second, timed != 0);
+      if (pass == 0) {
+        LGpu& L0 = lg[kv.second[0]];
+        std::swap(L0.gexec, L0.gexec_alt);
+        std::swap(L0.gexec_timed, L0.gexec_timed_alt);
+      }
+    }
+    if (pass == 0) kernels_per_run = kpr;  // counted once (the variants launch the same kernels)
   }
   captured = true;
+}
+
+// HIOS_STAGE_AUTO: replay both captured variants (graphs only, on the arena's
+// current contents) and keep the faster; wall time of launch-all + sync-all,
+// median of 7 after 2 warm-ups each.
+void Executor::choose_variant() {
+  auto run_all = [&](bool alt) {
+    const auto t0 = std::chrono::steady_clock::now();
+    for (auto& kv : graphs_by_dev) {
+      LGpu& L = lg[kv.second[0]];
+      ck(cudaSetDevice(L.dev), "cudaSetDevice");
+      ck(cudaGraphLaunch(alt ? L.gexec_alt : L.gexec, L.streams[0]), "graph launch");
+    }
+    for (auto& kv : graphs_by_dev) {
+      LGpu& L = lg[kv.second[0]];
+      ck(cudaSetDevice(L.dev), "cudaSetDevice");
+      ck(cudaStreamSynchronize(L.streams[0]), "synchronize");
+    }
+    return std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+  };
+  double med[2];
+  for (int alt = 0; alt < 2; ++alt) {
+    std::vector<double> t;
+    for (int i = 0; i < 9; ++i) {
+      const double x = run_all(alt != 0);
+      if (i >= 2) t.push_back(x);
+    }
+    std::sort(t.begin(), t.end());
+    med[alt] = t[t.size() / 2];
+  }
+  if (med[1] < med[0]) {
+    for (auto& kv : graphs_by_dev) {
+      LGpu& L = lg[kv.second[0]];
+      std::swap(L.gexec, L.gexec_alt);
+      std::swap(L.gexec_timed, L.gexec_timed_alt);
+    }
+    mode_used = HIOS_STAGE_DATAFLOW;
+  } else {
+    mode_used = HIOS_STAGE_STREAMS;
+  }
+  auto_pending = false;
 }
 
 void Executor::run_device(const void* d_in, void* d_out, cudaStream_t user, bool timed) {
@@ -1432,6 +1535,15 @@ void Executor::run_device(const void* d_in, void* d_out, cudaStream_t user, bool
   }
   if (ev_user) cudaEventDestroy(ev_user);
   ck(cudaGetLastError(), "run");
+  if (auto_pending) {
+    // the first run's results stand; the variants are then timed on its data
+    for (auto& kv : graphs_by_dev) {
+      ck(cudaSetDevice(lg[kv.second[0]].dev), "cudaSetDevice");
+      ck(cudaStreamSynchronize(lg[kv.second[0]].streams[0]), "synchronize");
+    }
+    choose_variant();
+    ck(cudaSetDevice(cur), "cudaSetDevice");
+  }
 }
 
 // Uninstrumented per-op device time of the schedule's own kernels (bench.py's

@@ -86,6 +86,9 @@ struct LGpu {
   std::vector<cudaEvent_t> ev_join;
   cudaEvent_t ev_start = nullptr, ev_done = nullptr;
   cudaGraphExec_t gexec = nullptr, gexec_timed = nullptr;
+  // HIOS_STAGE_AUTO: the other executor variant's graphs until the first run
+  // has measured both (then the faster one is gexec / gexec_timed)
+  cudaGraphExec_t gexec_alt = nullptr, gexec_timed_alt = nullptr;
   char* arena = nullptr;       // local: owned; remote (rank mode): IPC-mapped
   size_t arena_bytes = 0;
   unsigned* sync = nullptr;    // [0] epoch, [1 .. 1+M) acks, then flags
@@ -157,9 +160,18 @@ struct Executor {
   // launch on s0 with an explicit SM partition, the other ops forked onto
   // streams 1.. (or every op on its own stream: group == false); post(v, st)
   // runs after op v on the stream v ran on
+  // (lane != nullptr: the ops run on that stream instead of stream 0;
+  // singleton: a one-op stage takes the op's solo plan)
   void enqueue_stage(int l, const std::vector<int>& S, bool timed, int64_t& nk,
-                     const std::function<void(int, cudaStream_t)>& post);
+                     const std::function<void(int, cudaStream_t)>& post, cudaStream_t lane = nullptr,
+                     bool singleton = true);
   bool group_convs = false;  // hios_schedule_stage_mode
+  bool dataflow = false;     // HIOS_STAGE_DATAFLOW: per-op input waits instead of stage joins
+  bool auto_pending = false; // HIOS_STAGE_AUTO: streams vs dataflow not measured yet
+  int mode_used = 0;         // the stage mode the graphs execute (hios_schedule_stage_mode_used)
+  void choose_variant();     // HIOS_STAGE_AUTO: time both variants' graphs, keep the faster
+  std::vector<cudaEvent_t> done_ev;  // dataflow: op v finished on its lane
+  std::vector<int> lane_of;          // dataflow: the lane (stream index) op v ran on
 };
 
 void ck(cudaError_t e, const char* what);

@@ -81,6 +81,7 @@ def load() -> C.CDLL:
         "hios_read_op_output": [VP, I32, P(C.c_float), I64],
         "hios_kernel_count": [VP, P(I64)],
         "hios_op_plan": [VP, I32, I32, P(I32)],
+        "hios_schedule_stage_mode_used": [VP, P(I32)],
         "hios_time_ops": [VP, I32, I64, P(I64)],
         "hios_schedule_transport": [VP, I32],
         "hios_schedule_stage_mode": [VP, I32],
@@ -344,7 +345,7 @@ def hios_schedule_transport(s: Schedule, transport):
     _ck(load().hios_schedule_transport(s.h, t))
 
 
-STAGE_MODE = {"streams": 0, "grouped": 1}
+STAGE_MODE = {"streams": 0, "grouped": 1, "dataflow": 2, "auto": 3}
 
 
 def hios_schedule_stage_mode(s: Schedule, mode):
@@ -433,6 +434,13 @@ def hios_kernel_count(s: Schedule) -> int:
     v = C.c_int64()
     _ck(load().hios_kernel_count(s.h, C.byref(v)))
     return v.value
+
+
+def hios_schedule_stage_mode_used(s: Schedule) -> str:
+    """The stage mode the schedule's graphs execute (AUTO resolved after the first run)."""
+    v = C.c_int32()
+    _ck(load().hios_schedule_stage_mode_used(s.h, C.byref(v)))
+    return {m: k for k, m in STAGE_MODE.items()}[v.value]
 
 
 def hios_op_plan(s: Schedule, op: int, solo: bool = False) -> dict:

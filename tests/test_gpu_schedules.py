@@ -162,6 +162,33 @@ def test_grouped_stage_kernel_bit_identical(name, size):
         assert h.hios_kernel_count(S2) <= h.hios_kernel_count(S1)
 
 
+@pytest.mark.parametrize("name,size", [("inception_v3", 299), ("randwire_ws", 224), ("nasnet_a_large", 331)])
+def test_dataflow_and_auto_stage_modes_bit_identical(name, size):
+    """HIOS_STAGE_DATAFLOW (per-op input waits instead of stage joins) and
+    HIOS_STAGE_AUTO (both captured, the faster kept after the first run)
+    compute exactly what the stage-joined streams compute, on 1 GPU and on 2
+    logical GPUs, on every run; AUTO reports which variant it kept."""
+    h = hios()
+    g = graphs.build(name, size)
+    W = gen.make_weights(g)
+    x = gen.make_input(g)
+    G = h.hios_graph_create(g.ops, g.edges, g.in_c, g.in_h, g.in_w, "bf16", W)
+    h.hios_profile(G, [0], 3)
+    for M, w in [(1, 5), (2, 3)]:
+        S1 = h.hios_schedule_lp(G, M, w)
+        y1 = h.hios_run(S1, x)
+        assert h.hios_schedule_stage_mode_used(S1) == "streams"
+        for mode in ("dataflow", "auto"):
+            S2 = h.hios_schedule_lp(G, M, w)
+            h.hios_schedule_stage_mode(S2, mode)
+            for _ in range(2):  # AUTO: the first run measures, the second uses the kept variant
+                y2 = h.hios_run(S2, x)
+                assert np.array_equal(y1, y2), (M, w, mode)
+            used = h.hios_schedule_stage_mode_used(S2)
+            assert used == ("dataflow" if mode == "dataflow" else used) and used in ("streams", "dataflow")
+            assert h.hios_kernel_count(S2) == h.hios_kernel_count(S1)
+
+
 def test_time_ops_and_option_state_rules():
     """hios_time_ops (bench.py's roofline source): a positive time for every
     op with kernels, -1 for the input placeholder and zero-copy concats; the

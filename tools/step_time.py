@@ -20,6 +20,7 @@ def main():
     ap.add_argument("--size", type=int, default=1024)
     ap.add_argument("--windows", default="1,5")
     ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--stage-mode", default="streams")
     args = ap.parse_args()
     import torch
     from paper_conf_cluster_kundus23_b200 import hios as h
@@ -35,6 +36,8 @@ def main():
     out = []
     for w in [int(v) for v in args.windows.split(",")]:
         S = h.hios_schedule_lp(G, 1, w)
+        if args.stage_mode != "streams":
+            h.hios_schedule_stage_mode(S, args.stage_mode)
         d_out = torch.empty(h.hios_output_numel(S), device="cuda")
         for _ in range(5):
             h.hios_run_device(S, d_in.data_ptr(), d_out.data_ptr(), st.cuda_stream)
@@ -50,7 +53,8 @@ def main():
         ms = [a.elapsed_time(b) for a, b in ts]
         out.append(f"w={w}: {np.mean(ms):.4f} ms (median {np.median(ms):.4f}, predicted "
                    f"{h.hios_schedule_latency_ns(S) / 1e6:.4f})")
-    print(f"{args.model}@{args.size} lib={os.environ.get('HIOS_LIB', 'in-tree')}: " + "; ".join(out), flush=True)
+    print(f"{args.model}@{args.size} lib={os.environ.get('HIOS_LIB', 'in-tree')} mode={args.stage_mode}: " + "; ".join(out),
+          flush=True)
 
 
 if __name__ == "__main__":
