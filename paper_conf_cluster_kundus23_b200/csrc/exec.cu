@@ -1320,6 +1320,14 @@ void Executor::capture_device(const std::vector<int>& ls, bool timed) {
   // for its own inputs (done events of same-GPU producers on other lanes) and
   // the previous op of its lane -- no join at the stage boundary
   std::vector<char> lanes_forked(M, 0);
+  std::vector<std::vector<double>> lane_free(M);  // dataflow: predicted time each lane is free
+  std::vector<std::vector<int>> lane_last(M);     // dataflow: last op on each lane
+  std::vector<double> pred_fin(g.n, 0.0);         // dataflow: predicted finish of op v
+  for (int l : ls) {
+    lane_free[l].assign(lg[l].streams.size(), 0.0);
+    lane_last[l].assign(lg[l].streams.size(), -1);
+  }
+  std::fill(lane_of.begin(), lane_of.end(), -1);
   for (auto& it : order) {
     const int l = std::get<1>(it), j = std::get<2>(it);
     LGpu& L = lg[l];
@@ -1331,19 +1339,45 @@ void Executor::capture_device(const std::vector<int>& ls, bool timed) {
         ck(cudaEventRecord(L.ev_fork, s0), "fork lanes");
         for (size_t k = 1; k < L.streams.size(); ++k) ck(cudaStreamWaitEvent(L.streams[k], L.ev_fork, 0), "fork");
       }
+      // lane choice (list scheduling on the measured t(v)): the lane whose
+      // last op is v's latest-finishing same-GPU producer (the stream order is
+      // then a real dependency), else the lane free earliest; one lane per op
+      // of the stage
+      std::vector<char> taken(L.streams.size(), 0);
       for (size_t i = 0; i < S.size(); ++i) {
         const int v = S[i];
-        cudaStream_t st = L.streams[i];
         std::set<int> ins;
         for (int e : g.ops[v].in_edges) ins.insert(g.edges[e].src);
+        double ready = 0;
+        int prod_lane = -1;
+        double prod_fin = -1;
+        for (int u : ins)
+          if (s.gpu_of[u] == l && lane_of[u] >= 0) {
+            ready = std::max(ready, pred_fin[u]);
+            if (pred_fin[u] > prod_fin && lane_last[l][lane_of[u]] == u && !taken[lane_of[u]]) {
+              prod_fin = pred_fin[u];
+              prod_lane = lane_of[u];
+            }
+          }
+        int k = prod_lane;
+        if (k < 0) {
+          for (size_t c = 0; c < L.streams.size(); ++c)
+            if (!taken[c] && (k < 0 || lane_free[l][c] < lane_free[l][k])) k = (int)c;
+        }
+        taken[k] = 1;
+        cudaStream_t st = L.streams[k];
         for (int u : ins) {
           if (s.gpu_of[u] != l) wait_remote(u, l, st);
-          else if (lane_of[u] != (int)i && g.ops[u].kind != HIOS_OP_INPUT)
+          else if (g.ops[u].kind != HIOS_OP_INPUT && !(lane_of[u] == k && lane_last[l][k] == u))
             ck(cudaStreamWaitEvent(st, done_ev[u], 0), "wait input");
         }
         enqueue_stage(l, std::vector<int>{v}, timed, nk, deliver, st, S.size() == 1);
         ck(cudaEventRecord(done_ev[v], st), "done");
-        lane_of[v] = (int)i;
+        lane_of[v] = k;
+        lane_last[l][k] = v;
+        const double t = std::max<double>(1.0, (double)g.ops[v].cost);
+        pred_fin[v] = std::max(ready, lane_free[l][k]) + t;
+        lane_free[l][k] = pred_fin[v];
       }
       continue;
     }
