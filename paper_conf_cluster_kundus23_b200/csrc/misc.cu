@@ -97,8 +97,10 @@ static inline unsigned grid_for(long long n, int block) {
 // ---------------------------------------------------------------- pooling
 // grid = (ceil(Q * CG / 256), P): one output row per blockIdx.y; KH/KW > 0
 // unroll the window (loads hoisted, accumulated immediately).
+// (<= 64 registers: four 256-thread CTAs per SM; measured 66 registers
+// limited the 3x3 stride-2 max pools at 4096^2 to 37.5 % occupancy)
 template <typename T, int KH, int KW>
-__global__ void pool_kernel(const PoolArgs<T> a) {
+__global__ void __launch_bounds__(256, 4) pool_kernel(const PoolArgs<T> a) {
   pdl_enter();
   constexpr int N = Vec<T>::N;
   const int kh = KH > 0 ? KH : a.kh, kw = KW > 0 ? KW : a.kw;
@@ -376,6 +378,8 @@ __global__ void __launch_bounds__(256) pool_tiled_kernel(const PoolArgs<T> a) {
 // bytes per pixel: whole cache lines per load, vs 32-byte pieces in
 // pool_tiled_kernel) and each thread reduces four outputs (columns lane/8 +
 // 4j of row warp, channel vector lane%8) with FHADD.BF16 from smem.
+// (Measured slower: four consecutive columns per thread sharing their vertical
+// 3-sums -- avgpool 5d at 4096^2 75.5 -> 81.2 us, more registers.)
 constexpr int kP64TP = 8, kP64TQ = 16;
 __global__ void __launch_bounds__(256) pool_avg64_kernel(const PoolArgs<bf16> a) {
   __shared__ __align__(16) uint4 tile[(kP64TP + 2) * (kP64TQ + 2) * 8];
@@ -539,7 +543,7 @@ __host__ __device__ inline int dw_tile_rows(int R, int sh) { return (kDwTP - 1) 
 __host__ __device__ inline int dw_tile_cols(int S, int sw) { return (kDwTQ - 1) * sw + S; }
 
 template <typename T, int KS>
-__global__ void __launch_bounds__(256) dw_tiled_kernel(const DwArgs<T> a) {
+__global__ void __launch_bounds__(256, 4) dw_tiled_kernel(const DwArgs<T> a) {
   extern __shared__ __align__(16) uint8_t dsm[];
   constexpr int N = 8;                       // channels per vector (16 B bf16, 32 B fp32)
   constexpr int VB = N * (int)sizeof(T);     // bytes per staged vector
@@ -645,7 +649,7 @@ __global__ void __launch_bounds__(256) dw_tiled_kernel(const DwArgs<T> a) {
 // fma.rn.f32.bf16 (FHFMA.BF16, sm_100) multiplies the bf16 halves directly
 // into fp32 accumulators: no conversions in the inner loop.
 template <int KS, int SS, int KR>
-__global__ void __launch_bounds__(256) dw_reg_kernel(const DwArgs<bf16> a) {
+__global__ void __launch_bounds__(256, 4) dw_reg_kernel(const DwArgs<bf16> a) {
   extern __shared__ __align__(16) uint8_t dsm[];
   constexpr int TP = 4 * KR, N = 8, VB = 16;
   constexpr int IH = (TP - 1) * SS + KS, IW = (kDwTQ - 1) * SS + KS;

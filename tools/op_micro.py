@@ -17,6 +17,8 @@ PEAK_TF, PEAK_GBS = 1645.7, 6554.2
 # name, kind, C, H, W, params
 SHAPES = [
     ("i4096_maxpool1", "maxpool", 64, 2045, 2045, dict(k=3, s=2, p=0)),
+    ("i4096_maxpool2", "maxpool", 192, 1020, 1020, dict(k=3, s=2, p=0)),
+    ("i4096_6a_maxpool", "maxpool", 288, 509, 509, dict(k=3, s=2, p=0)),
     ("i4096_avgpool5d", "avgpool", 288, 509, 509, dict(k=3, s=1, p=1)),
     ("i4096_avgpool6b", "avgpool", 768, 254, 254, dict(k=3, s=1, p=1)),
     ("sq_maxpool2", "maxpool", 96, 1021, 1021, dict(k=3, s=2, p=0, ceil=1)),
