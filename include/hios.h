@@ -344,6 +344,15 @@ hios_status hios_kernel_count(hios_schedule s, int64_t* n);
  * (NULL, op out of range), HIOS_E_STATE (Q not run yet). */
 hios_status hios_op_plan(hios_schedule s, int32_t op, int32_t solo, int32_t* plan);
 
+/* *relu = 1 when op `op`'s stored output (hios_read_op_output) is ReLU(y)
+ * rather than y: every consumer applies ReLU to it first (pre-ReLU convs,
+ * single-input separable convs and ReLU adds, or a concat whose consumers all
+ * do -- NASNet's ReLU -> conv -> BN cell inputs), so the executor applies the
+ * ReLU in the producer's epilogue instead of making a ReLU'd copy for the
+ * consumers; the network output never is.  Errors: HIOS_E_INVALID,
+ * HIOS_E_STATE (not run yet). */
+hios_status hios_op_output_relu(hios_schedule s, int32_t op, int32_t* relu);
+
 /* ------------------------------------------------------------------ misc */
 const char* hios_last_error(void);
 int32_t hios_abi_version(void);

@@ -518,6 +518,14 @@ hios_status hios_schedule_stage_mode_used(hios_schedule s, int32_t* mode) {
   });
 }
 
+hios_status hios_op_output_relu(hios_schedule s, int32_t op, int32_t* relu) {
+  return guard([&] {
+    NEED(s && relu && op >= 0 && op < s->s->g->n, HIOS_E_INVALID, "bad argument");
+    NEED(s->s->exec && s->s->exec->captured, HIOS_E_STATE, "run first");
+    *relu = s->s->exec->relu_out[op] ? 1 : 0;
+  });
+}
+
 hios_status hios_op_plan(hios_schedule s, int32_t op, int32_t solo, int32_t* plan) {
   return guard([&] {
     NEED(s && plan && op >= 0 && op < s->s->g->n, HIOS_E_INVALID, "bad argument");

@@ -189,12 +189,59 @@ void Executor::plan() {
       }
     }
   }
+  // ReLU hoisting (relu_out): an op whose every consumer applies ReLU to it
+  // first stores its output ReLU'd (its epilogue has a ReLU flag: conv,
+  // separable conv, add, identity); a concat qualifies when its consumers all
+  // do and each of its inputs qualifies with the concat counted as ReLU-first
+  relu_out.assign(n, 0);
+  {
+    auto relu_first = [&](int v) {
+      const Op& c = g.ops[v];
+      // (a separable conv aggregates its inputs before the ReLU: one input only)
+      const bool single = c.in_edges.size() == 1 && (c.agg.empty() || c.agg[0] == 1.f);
+      if (c.kind == HIOS_OP_CONV && c.pre_relu) return true;
+      if (c.kind == HIOS_OP_SEPCONV && c.pre_relu && single) return true;
+      return c.kind == HIOS_OP_ADD && c.relu && single;
+    };
+    auto can_relu = [&](int u) {
+      const int k = g.ops[u].kind;
+      return u != g.sink_op && (k == HIOS_OP_CONV || k == HIOS_OP_SEPCONV || k == HIOS_OP_ADD || k == HIOS_OP_IDENTITY);
+    };
+    auto all_relu_first = [&](int u, int except) {
+      if (g.ops[u].out_edges.empty()) return false;
+      for (int e : g.ops[u].out_edges) {
+        const int v = g.edges[e].dst;
+        if (v != except && !relu_first(v)) return false;
+      }
+      return true;
+    };
+    std::vector<char> concat_ok(n, 0);
+    for (int c = 0; c < n; ++c) {
+      if (g.ops[c].kind != HIOS_OP_CONCAT || c == g.sink_op || !all_relu_first(c, -1)) continue;
+      bool ok = true;
+      for (int e : g.ops[c].in_edges) {
+        const int p = g.edges[e].src;
+        if (!can_relu(p) || !all_relu_first(p, c)) ok = false;
+        for (int e2 : g.ops[p].out_edges)  // a producer of two concats: keep it simple
+          if (g.edges[e2].dst != c && g.ops[g.edges[e2].dst].kind == HIOS_OP_CONCAT) ok = false;
+      }
+      concat_ok[c] = ok;
+    }
+    for (int c = 0; c < n; ++c)
+      if (concat_ok[c]) {
+        relu_out[c] = 1;
+        for (int e : g.ops[c].in_edges) relu_out[g.edges[e].src] = 1;
+      }
+    for (int u = 0; u < n; ++u)
+      if (!relu_out[u] && can_relu(u) && all_relu_first(u, -1)) relu_out[u] = 1;
+  }
   // pre-ReLU convs: one ReLU'd copy of the input per (producer, GPU) when the
   // producer runs on that GPU (made right after it), else a per-consumer scratch
   relu_loc.clear();
   for (int v = 0; v < n; ++v) {
     const Op& o = g.ops[v];
     if (o.kind != HIOS_OP_CONV || !o.pre_relu) continue;
+    if (relu_out[g.edges[o.in_edges[0]].src]) continue;  // stored ReLU'd already
     const int u = g.edges[o.in_edges[0]].src, l = s.gpu_of[v];
     const Op& ou = g.ops[u];
     const int ldc = rup(ou.C, 8);
@@ -777,6 +824,7 @@ static void build_op(Executor& ex, int v) {
   const Op& o = g.ops[v];
   const int l = ex.s.gpu_of[v];
   OpExec& x = ex.ox[v];
+  const int relu_v = (o.relu || ex.relu_out[v]) ? 1 : 0;  // the op's own ReLU, or its consumers' (hoisted)
   auto view_of = [&](int u, int on) { return View{ex.ptr(on, ex.loc[u][on].off), ex.loc[u][on].ldc}; };
   auto in_op = [&](int k) { return g.edges[o.in_edges[k]].src; };
   const View out = view_of(v, l);
@@ -798,7 +846,7 @@ static void build_op(Executor& ex, int v) {
       // made once after u on u's GPU (shared by every pre-ReLU consumer there)
       // or, for a remote / input producer, here into this op's scratch
       View cin = view_of(u, l);
-      if (o.pre_relu) {
+      if (o.pre_relu && !ex.relu_out[u]) {
         auto it = ex.relu_loc.find((int64_t)u * ex.M + l);
         if (it != ex.relu_loc.end()) {
           cin = View{ex.ptr(l, it->second.off), it->second.ldc};
@@ -815,7 +863,7 @@ static void build_op(Executor& ex, int v) {
         if (iv.ldc < (int)(16 / sizeof(T))) fail(HIOS_E_UNSUPPORTED, "stem input pixel pitch below 16 bytes");
         ConvStem3Args<T> c{};
         c.x = (const T*)iv.p; c.H = xi.H; c.W = xi.W; c.ldx = iv.ldc;
-        c.P = o.H; c.Q = o.W; c.K = o.out_c; c.ph = o.ph; c.pw = o.pw; c.relu = o.relu;
+        c.P = o.H; c.Q = o.W; c.K = o.out_c; c.ph = o.ph; c.pw = o.pw; c.relu = relu_v;
         // whole 16-byte vectors (zeros into the pad channels) unless an output
         // is a concat slice, whose pad channels belong to the next producer
         bool own = true;
@@ -851,10 +899,10 @@ static void build_op(Executor& ex, int v) {
           // 4-pixel window j..j+3 of the s2d tensor (pixel stride 32 B)
           View pv{sv.p, sv.ldc, W2};
           fns.push_back(conv_closure<T>(ex, pv, H2, o.W, 64, x.w_pack, x.scale[0], x.shift[0], o.out_c, R2, 1, 1, 1,
-                                        0, 0, 1, 1, o.H, o.W, o.relu, out, out2, nk));
+                                        0, 0, 1, 1, o.H, o.W, relu_v, out, out2, nk));
         } else {
           fns.push_back(conv_closure<T>(ex, sv, H2, W2, 4 * xi.C, x.w, x.scale[0], x.shift[0], o.out_c, R2, S2, 1, 1,
-                                        0, 0, 1, 1, o.H, o.W, o.relu, out, out2, nk));
+                                        0, 0, 1, 1, o.H, o.W, relu_v, out, out2, nk));
         }
         break;
       }
@@ -864,7 +912,7 @@ static void build_op(Executor& ex, int v) {
         c.x = (const T*)iv.p; c.H = xi.H; c.W = xi.W; c.C = xi.C; c.ldx = iv.ldc;
         c.w = x.w_small; c.scale = x.scale[0]; c.shift = x.shift[0];
         c.P = o.H; c.Q = o.W; c.K = o.out_c; c.R = o.kh; c.S = o.kw; c.sh = o.sh; c.sw = o.sw;
-        c.ph = o.ph; c.pw = o.pw; c.relu = o.relu;
+        c.ph = o.ph; c.pw = o.pw; c.relu = relu_v;
         c.out = (T*)out.p; c.ldo = out.ldc;
         c.out2 = dst_of<T>(out2);
         fns.push_back([c](cudaStream_t st) { launch_conv_small_c<T>(c, st); });
@@ -878,7 +926,7 @@ static void build_op(Executor& ex, int v) {
         g_tc_smem = &x.tc_smem;
       }
       fns.push_back(conv_closure<T>(ex, cin, xi.H, xi.W, xi.C, x.w, x.scale[0], x.shift[0], o.out_c, o.kh,
-                                    o.kw, o.sh, o.sw, o.ph, o.pw, o.dh, o.dw, o.H, o.W, o.relu, out, out2, nk));
+                                    o.kw, o.sh, o.sw, o.ph, o.pw, o.dh, o.dw, o.H, o.W, relu_v, out, out2, nk));
       g_tc_out = nullptr;
       g_tc_smem = nullptr;
       break;
@@ -911,7 +959,7 @@ static void build_op(Executor& ex, int v) {
         ++nk;
         const bool last = r == o.reps - 1;
         fns.push_back(conv_closure<T>(ex, dwv, o.H, o.W, c, x.pw[r], x.scale[r], x.shift[r], o.out_c, 1, 1, 1, 1, 0,
-                                      0, 1, 1, o.H, o.W, last ? o.relu : 0, last ? out : midv,
+                                      0, 1, 1, o.H, o.W, last ? relu_v : 0, last ? out : midv,
                                       last ? out2 : std::vector<View>(), nk));
       }
       break;
@@ -976,7 +1024,7 @@ static void build_op(Executor& ex, int v) {
         View iv = view_of(in_op(k), l);
         a.x[k] = (const T*)iv.p; a.ldx[k] = iv.ldc; a.agg[k] = o.agg[k];
       }
-      a.n_in = nin; a.HW = o.H * o.W; a.C = o.C; a.relu = o.relu;
+      a.n_in = nin; a.HW = o.H * o.W; a.C = o.C; a.relu = relu_v;
       a.out = (T*)out.p; a.ldo = out.ldc;
       a.out2 = dst_of<T>(out2);
       fns.push_back([a](cudaStream_t st) { launch_add<T>(a, st); });
@@ -986,7 +1034,8 @@ static void build_op(Executor& ex, int v) {
     case HIOS_OP_IDENTITY: {
       View iv = view_of(in_op(0), l);
       CopyArgs<T> c{(const T*)iv.p, iv.ldc, o.H * o.W, o.C, (T*)out.p, out.ldc};
-      fns.push_back([c](cudaStream_t st) { launch_copy<T>(c, st); });
+      if (relu_v) fns.push_back([c](cudaStream_t st) { launch_relu_copy<T>(c, st); });
+      else fns.push_back([c](cudaStream_t st) { launch_copy<T>(c, st); });
       ++nk;
       break;
     }

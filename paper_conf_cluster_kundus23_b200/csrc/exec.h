@@ -117,6 +117,11 @@ struct Executor {
   std::vector<std::vector<Loc>> loc;   // loc[op][lgpu]
   std::map<int64_t, Loc> relu_loc;     // (producer * M + lgpu) -> ReLU'd copy for pre-ReLU convs
   std::vector<char> inplace;           // per edge: producer writes into the concat slice
+  // per op: every consumer applies ReLU to this output first (pre-ReLU convs /
+  // separable convs, single-input ReLU adds, or a concat whose own consumers
+  // all do), so the op stores its output already ReLU'd and the consumers
+  // read it without a ReLU'd copy (ReLU(bf16(y)) = bf16(ReLU(y)): exact)
+  std::vector<char> relu_out;
   std::vector<OpExec> ox;
   std::vector<std::vector<int>> flag_index;  // [op][lgpu] flag slot on that lgpu (-1 none)
   int n_streams = 1;

@@ -81,6 +81,7 @@ def load() -> C.CDLL:
         "hios_read_op_output": [VP, I32, P(C.c_float), I64],
         "hios_kernel_count": [VP, P(I64)],
         "hios_op_plan": [VP, I32, I32, P(I32)],
+        "hios_op_output_relu": [VP, I32, P(I32)],
         "hios_schedule_stage_mode_used": [VP, P(I32)],
         "hios_time_ops": [VP, I32, I64, P(I64)],
         "hios_schedule_transport": [VP, I32],
@@ -441,6 +442,13 @@ def hios_schedule_stage_mode_used(s: Schedule) -> str:
     v = C.c_int32()
     _ck(load().hios_schedule_stage_mode_used(s.h, C.byref(v)))
     return {m: k for k, m in STAGE_MODE.items()}[v.value]
+
+
+def hios_op_output_relu(s: Schedule, op: int) -> bool:
+    """True when op's stored output is ReLU'd (its consumers' ReLU hoisted into it)."""
+    v = C.c_int32()
+    _ck(load().hios_op_output_relu(s.h, op, C.byref(v)))
+    return bool(v.value)
 
 
 def hios_op_plan(s: Schedule, op: int, solo: bool = False) -> dict:
