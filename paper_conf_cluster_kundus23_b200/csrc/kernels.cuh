@@ -187,8 +187,8 @@ template <typename T> void launch_conv_small_c(const ConvSmallArgs<T>& a, cudaSt
 // kernel's parameter bank, so every multiply-add is one FFMA with a constant
 // operand (no shared-memory weight loads); see misc.cu conv_stem3_kernel
 constexpr int kStem3MaxK = 40;
-struct Stem3W {
-  float w[27][kStem3MaxK];  // [(r*3+s)*3+c][k]
+struct __align__(8) Stem3W {
+  float w[27][kStem3MaxK];  // [(r*3+s)*3+c][k]  (channel pairs 8-byte aligned: fma.rn.f32x2)
   float scale[kStem3MaxK], shift[kStem3MaxK];
 };
 template <typename T>

@@ -1352,11 +1352,16 @@ __global__ void __launch_bounds__(128) conv_stem3_kernel(const ConvStem3Args<T> 
   float x[3][XW][3];
   stem3_load<T, PX>(a, QP, it, x);
   const int kb = KT < KK ? (int)blockIdx.y * KT : 0;
-  float acc[PX][KT];
+  static_assert(KT % 2 == 0, "channel pairs");
+  // packed fp32x2 FMAs (FFMA2, sm_100): output channels (k, k+1) of one pixel
+  // per instruction -- the input value broadcast to both halves, the weight
+  // pair {w[i][k], w[i][k+1]} read from the parameter bank; two independent
+  // round-to-nearest FMAs, the same arithmetic as fmaf in the same order
+  uint64_t acc2[PX][KT / 2];
 #pragma unroll
   for (int u = 0; u < PX; ++u)
 #pragma unroll
-    for (int k = 0; k < KT; ++k) acc[u][k] = 0.f;
+    for (int k = 0; k < KT / 2; ++k) acc2[u][k] = 0ull;
 #pragma unroll
   for (int r = 0; r < 3; ++r)
 #pragma unroll
@@ -1364,13 +1369,30 @@ __global__ void __launch_bounds__(128) conv_stem3_kernel(const ConvStem3Args<T> 
 #pragma unroll
       for (int c = 0; c < 3; ++c) {
         const int i = (r * 3 + s) * 3 + c;
+        uint64_t xb[PX];
 #pragma unroll
-        for (int k = 0; k < KT; ++k) {
-          const float wv = w.w[i][kb + k];  // uniform-register operand of the FFMA
+        for (int u = 0; u < PX; ++u) {
+          const float xv = x[r][2 * u + s][c];
+          asm("mov.b64 %0, {%1, %1};" : "=l"(xb[u]) : "f"(xv));
+        }
 #pragma unroll
-          for (int u = 0; u < PX; ++u) acc[u][k] = fmaf(x[r][2 * u + s][c], wv, acc[u][k]);
+        for (int k = 0; k < KT; k += 2) {
+          const uint64_t wv = *reinterpret_cast<const uint64_t*>(&w.w[i][kb + k]);  // uniform operand
+#pragma unroll
+          for (int u = 0; u < PX; ++u)
+            asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(acc2[u][k / 2]) : "l"(xb[u]), "l"(wv));
         }
       }
+  float acc[PX][KT];
+#pragma unroll
+  for (int u = 0; u < PX; ++u)
+#pragma unroll
+    for (int k = 0; k < KT / 2; ++k) {
+      float lo, hi;
+      asm("mov.b64 {%0, %1}, %2;" : "=f"(lo), "=f"(hi) : "l"(acc2[u][k]));
+      acc[u][2 * k] = lo;
+      acc[u][2 * k + 1] = hi;
+    }
   const int p = (int)(it / QP), q0 = (int)(it - (long long)p * QP) * PX;
 #pragma unroll
   for (int u = 0; u < PX; ++u) {
