@@ -255,6 +255,43 @@ __device__ __forceinline__ void halo_taps_bres(uint32_t d, uint64_t a0, uint64_t
   }
 }
 
+// the same for ONE elected lane (the caller branches on elect_one()): plain,
+// unpredicated tcgen05.mma with a compile-time K=16 slice count KV_.  With a
+// single active thread ptxas keeps the descriptors in uniform registers and
+// issues the MMAs back to back; issued lane-predicated from the converged warp
+// every descriptor went through R2UR (~150 cycles per MMA in the kernel).
+// Measured: Conv2d_2a-4096 298 -> 192 us, Conv2d_2b 291 -> 262 us, Conv2d_2a
+// at 1024^2 21.9 -> 16.0 us.  (The whole issue loop on one lane -- ring and
+// tap modes too -- measured slower for the weight-ring convs: Conv2d_4a-4096
+// 367 -> 379 us, NASNet-2048 10.78 -> 11.10 ms.)
+template <int R_, int S_, int HK_, int KV_>
+__device__ __forceinline__ void halo_taps_bres_lane(uint32_t d, uint64_t a0, uint64_t b0, uint32_t idesc,
+                                                    uint64_t row_r16, uint64_t row_s16, uint64_t b16, uint32_t accum,
+                                                    uint32_t dstride) {
+#pragma unroll
+  for (int t = 0; t < R_ * S_; ++t) {
+    const uint64_t bd = b0 + (uint64_t)t * b16;
+#pragma unroll
+    for (int j = 0; j < HK_; ++j) {
+      const uint64_t ad = a0 + (uint64_t)(t / S_ + j) * row_r16 + (uint64_t)(t % S_) * row_s16;
+      const uint32_t dj = d + (uint32_t)j * dstride;
+#pragma unroll
+      for (int q = 0; q < KV_; ++q) mma_bf16(dj, ad + 2 * q, bd + 2 * q, idesc, (t == 0 && q == 0) ? accum : 1u);
+    }
+  }
+}
+// dispatch on the chunk's K=16 slice count (1, 2 or 4; 3 -> false: the caller
+// issues the lane-predicated loop)
+template <int R_, int S_, int HK_, int KVMIN>
+__device__ __forceinline__ void halo_taps_bres_lane_kv(int kv, uint32_t d, uint64_t a0, uint64_t b0, uint32_t idesc,
+                                                       uint64_t row_r16, uint64_t row_s16, uint64_t b16, uint32_t accum,
+                                                       uint32_t dstride) {
+  if (kv == 4) halo_taps_bres_lane<R_, S_, HK_, 4>(d, a0, b0, idesc, row_r16, row_s16, b16, accum, dstride);
+  else if (KVMIN <= 3 && kv == 3) halo_taps_bres_lane<R_, S_, HK_, 3>(d, a0, b0, idesc, row_r16, row_s16, b16, accum, dstride);
+  else if (KVMIN <= 2 && kv == 2) halo_taps_bres_lane<R_, S_, HK_, 2>(d, a0, b0, idesc, row_r16, row_s16, b16, accum, dstride);
+  else if (KVMIN <= 1) halo_taps_bres_lane<R_, S_, HK_, 1>(d, a0, b0, idesc, row_r16, row_s16, b16, accum, dstride);
+}
+
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
@@ -599,11 +636,29 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
             const int kv = min(4, (C - cc * 64 + 15) >> 4);
             if (bres && fixed_rs) {
               // resident weights, common kernel shapes: the chunk's taps fully
-              // unrolled with compile-time window offsets (descriptor adds on
-              // the uniform datapath, no loop-carried offsets)
+              // unrolled with compile-time window offsets, issued by the
+              // elected lane alone (halo_taps_bres_lane)
               const uint64_t bc = bres0 + (uint64_t)(cc * RS) * b16;
               const uint32_t dsx = (uint32_t)a.n_tile;
-              if (a.R == 3 && S_ == 3) {
+              // (3x3 with 2 or 4 K=16 slices, 1x1 with any: the lane-issued
+              // instantiations; other shapes / slice counts the predicated loop)
+              const bool lane_ok = (a.R == 3 && S_ == 3 && (kv == 2 || kv == 4)) || (a.R == 1 && S_ == 1);
+              bool done = false;
+              if (lane_ok) {
+                if (on) {
+                  if (a.R == 3) {
+                    if (hk2) halo_taps_bres_lane_kv<3, 3, 2, 2>(kv, d, a0, bc, idesc, row_r16, row_s16, b16, accum, dsx);
+                    else halo_taps_bres_lane_kv<3, 3, 1, 2>(kv, d, a0, bc, idesc, row_r16, row_s16, b16, accum, dsx);
+                  } else {
+                    if (hk2) halo_taps_bres_lane_kv<1, 1, 2, 1>(kv, d, a0, bc, idesc, row_r16, row_s16, b16, accum, dsx);
+                    else halo_taps_bres_lane_kv<1, 1, 1, 1>(kv, d, a0, bc, idesc, row_r16, row_s16, b16, accum, dsx);
+                  }
+                }
+                __syncwarp();
+                done = true;
+              }
+              if (done) {
+              } else if (a.R == 3 && S_ == 3) {
                 if (hk2) halo_taps_bres<3, 3, 2>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
                 else halo_taps_bres<3, 3, 1>(d, a0, bc, idesc, kv, on, row_r16, row_s16, b16, accum, dsx);
               }
