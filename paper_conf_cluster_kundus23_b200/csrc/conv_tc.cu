@@ -768,11 +768,14 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
       } else {
         // tap mode, lean issue loop: a stage carries up to kps K-steps (may
         // cross a 64-channel chunk); descriptors are stage bases + strides
+        // (the whole loop on the elected lane: waits, MMAs, commits -- the
+        // descriptors stay in uniform registers, see halo_taps_bres_lane)
         const int C = a.C, kps = KPS;
-        const uint32_t on = elect_one() ? 1u : 0u;
+        const uint32_t on = 1u;
         const uint32_t ST_ = (uint32_t)ST;
         const uint64_t aD0 = umma_desc_sw128(sA0), bD0 = umma_desc_sw128(sB0);
         const uint64_t ast16 = A_STAGE >> 4, bst16 = B_STAGE >> 4, a16 = A_BYTES >> 4, b16 = B_BYTES >> 4;
+        if (elect_one())
         for (int tile = cta; tile < tiles; tile += ncta, ++tcount) {
           mbar_wait(tempty0 + 8 * acc, tph ^ 1u);
           tc_fence_after();
@@ -807,11 +810,11 @@ __device__ __forceinline__ void conv_tc_body(const CUtensorMap* pmx, const CUten
             if (++st == ST_) { st = 0; ph ^= 1u; }
           }
           mma_commit_on(tfull0 + 8 * acc, on);
-          __syncwarp();
-          if (lane == 0 && tcount == 0 && j == 0) TRACE(4);
+          if (tcount == 0 && j == 0) TRACE(4);
           if (a.nacc == 2) acc ^= 1u;
           if (acc == 0) tph ^= 1u;
         }
+        __syncwarp();
       }
     }
     __syncwarp();
