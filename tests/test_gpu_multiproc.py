@@ -49,6 +49,18 @@ def test_two_process_ipc_run(model, size, transport):
     assert "bit-identical to 1-process run: True" in r.stdout
 
 
+@pytest.mark.parametrize("transport", ["peer", "copy"])
+def test_two_process_ipc_run_dataflow(transport):
+    """HIOS_STAGE_DATAFLOW across processes: per-op lanes wait on the IPC
+    flags of their own cross-GPU inputs; bit-identical to one process."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr=127.0.0.1", "--master-port=29535", os.path.join(ROOT, "tools", "mp_check.py"),
+           "inception_v3", "299", transport, "dataflow"]
+    r = _run_group(cmd, 300)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
+    assert "bit-identical to 1-process run: True" in r.stdout
+
+
 def test_bench_two_ranks_smoke():
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", "--master-port=29534", os.path.join(ROOT, "bench.py"),

@@ -22,6 +22,7 @@ def main():
     model = sys.argv[1] if len(sys.argv) > 1 else "tiny"
     size = int(sys.argv[2]) if len(sys.argv) > 2 and sys.argv[2] != "-" else None
     transport = sys.argv[3] if len(sys.argv) > 3 else "peer"
+    stage_mode = sys.argv[4] if len(sys.argv) > 4 else "streams"
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
     dev = int(os.environ.get("LOCAL_RANK", "0")) % torch.cuda.device_count()
@@ -41,6 +42,7 @@ def main():
         S = h.hios_schedule_lp(G, world, 2)
     S = bench.share_schedule(h, dist, G, g, S, world, 2, rank)
     h.hios_schedule_transport(S, transport)
+    h.hios_schedule_stage_mode(S, stage_mode)
     own = bench.bind_and_exchange(h, dist, S, world, world, rank, dev, transport=transport)
     op_gpu, _, _ = h.hios_schedule_stages(S)
     used = sorted(set(op_gpu.tolist()))
@@ -62,7 +64,8 @@ def main():
         S1 = h.hios_schedule_lp(G1, 1, 1)
         y1 = h.hios_run(S1, x)
         ok = all(np.array_equal(y, y1) for y in ys)
-        print(f"rank {rank}: world {world}, transport {transport}, GPUs used {used}, sink on rank {sink_rank}, "
+        print(f"rank {rank}: world {world}, transport {transport}, stage mode {stage_mode}, GPUs used {used}, "
+              f"sink on rank {sink_rank}, "
               f"bit-identical to 1-process run: {ok}", flush=True)
     flag = torch.tensor([1 if ok else 0])
     dist.all_reduce(flag, op=dist.ReduceOp.MIN)
