@@ -381,7 +381,7 @@ __global__ void __launch_bounds__(256) pool_tiled_kernel(const PoolArgs<T> a) {
 // (Measured slower: four consecutive columns per thread sharing their vertical
 // 3-sums -- avgpool 5d at 4096^2 75.5 -> 81.2 us, more registers.)
 constexpr int kP64TP = 8, kP64TQ = 16;
-__global__ void __launch_bounds__(256) pool_avg64_kernel(const PoolArgs<bf16> a) {
+__global__ void __launch_bounds__(256, 6) pool_avg64_kernel(const PoolArgs<bf16> a) {
   __shared__ __align__(16) uint4 tile[(kP64TP + 2) * (kP64TQ + 2) * 8];
   const int c0 = blockIdx.x * 64, q0 = blockIdx.y * kP64TQ, p0 = blockIdx.z * kP64TP;
   pdl_enter();
