@@ -142,6 +142,51 @@ void Executor::plan() {
     cursor[l] += rup64(std::max<int64_t>(bytes, 16) + 128, 256);
     return off;
   };
+  // ReLU hoisting (relu_out): an op whose every consumer applies ReLU to it
+  // first stores its output ReLU'd (its epilogue has a ReLU flag: conv,
+  // separable conv, add, identity).  A concat whose consumers all do is stored
+  // ReLU'd: each input that qualifies (the concat counted as ReLU-first) writes
+  // its slice ReLU'd in place; any other input keeps its raw output in its own
+  // buffer and the concat ReLU-copies that slice (relu_copy_in) -- NASNet's
+  // cell outputs: the five branch adds in place, the fitted input copied
+  relu_out.assign(n, 0);
+  relu_copy_in.assign(g.edges.size(), 0);
+  {
+    auto relu_first = [&](int v) {
+      const Op& c = g.ops[v];
+      // (a separable conv aggregates its inputs before the ReLU: one input only)
+      const bool single = c.in_edges.size() == 1 && (c.agg.empty() || c.agg[0] == 1.f);
+      if (c.kind == HIOS_OP_CONV && c.pre_relu) return true;
+      if (c.kind == HIOS_OP_SEPCONV && c.pre_relu && single) return true;
+      return c.kind == HIOS_OP_ADD && c.relu && single;
+    };
+    auto can_relu = [&](int u) {
+      const int k = g.ops[u].kind;
+      return u != g.sink_op && (k == HIOS_OP_CONV || k == HIOS_OP_SEPCONV || k == HIOS_OP_ADD || k == HIOS_OP_IDENTITY);
+    };
+    auto all_relu_first = [&](int u, int except) {
+      if (g.ops[u].out_edges.empty()) return false;
+      for (int e : g.ops[u].out_edges) {
+        const int v = g.edges[e].dst;
+        if (v != except && !relu_first(v)) return false;
+      }
+      return true;
+    };
+    for (int c = 0; c < n; ++c) {
+      if (g.ops[c].kind != HIOS_OP_CONCAT || c == g.sink_op || !all_relu_first(c, -1)) continue;
+      relu_out[c] = 1;
+      for (int e : g.ops[c].in_edges) {
+        const int p = g.edges[e].src;
+        bool ok = can_relu(p) && all_relu_first(p, c);
+        for (int e2 : g.ops[p].out_edges)  // a producer of two concats: copy
+          if (g.edges[e2].dst != c && g.ops[g.edges[e2].dst].kind == HIOS_OP_CONCAT) ok = false;
+        if (ok) relu_out[p] = 1;
+        else relu_copy_in[e] = 1;
+      }
+    }
+    for (int u = 0; u < n; ++u)
+      if (!relu_out[u] && can_relu(u) && all_relu_first(u, -1)) relu_out[u] = 1;
+  }
   // reverse topological order: a concat consumer's buffer exists before its producers are placed
   for (int k = n - 1; k >= 0; --k) {
     const int u = g.topo[k];
@@ -152,7 +197,7 @@ void Executor::plan() {
       for (int e : o.out_edges) {
         const int v = g.edges[e].dst;
         const Op& ov = g.ops[v];
-        if (ov.kind != HIOS_OP_CONCAT || s.gpu_of[v] != l || loc[v][l].off < 0) continue;
+        if (ov.kind != HIOS_OP_CONCAT || s.gpu_of[v] != l || loc[v][l].off < 0 || relu_copy_in[e]) continue;
         int c_off = 0;
         for (int e2 : ov.in_edges) {
           if (g.edges[e2].slot >= g.edges[e].slot) break;
@@ -188,52 +233,6 @@ void Executor::plan() {
         x.midbuf = alloc(l, (int64_t)o.H * o.W * x.mid_ldc * esz);
       }
     }
-  }
-  // ReLU hoisting (relu_out): an op whose every consumer applies ReLU to it
-  // first stores its output ReLU'd (its epilogue has a ReLU flag: conv,
-  // separable conv, add, identity); a concat qualifies when its consumers all
-  // do and each of its inputs qualifies with the concat counted as ReLU-first
-  relu_out.assign(n, 0);
-  {
-    auto relu_first = [&](int v) {
-      const Op& c = g.ops[v];
-      // (a separable conv aggregates its inputs before the ReLU: one input only)
-      const bool single = c.in_edges.size() == 1 && (c.agg.empty() || c.agg[0] == 1.f);
-      if (c.kind == HIOS_OP_CONV && c.pre_relu) return true;
-      if (c.kind == HIOS_OP_SEPCONV && c.pre_relu && single) return true;
-      return c.kind == HIOS_OP_ADD && c.relu && single;
-    };
-    auto can_relu = [&](int u) {
-      const int k = g.ops[u].kind;
-      return u != g.sink_op && (k == HIOS_OP_CONV || k == HIOS_OP_SEPCONV || k == HIOS_OP_ADD || k == HIOS_OP_IDENTITY);
-    };
-    auto all_relu_first = [&](int u, int except) {
-      if (g.ops[u].out_edges.empty()) return false;
-      for (int e : g.ops[u].out_edges) {
-        const int v = g.edges[e].dst;
-        if (v != except && !relu_first(v)) return false;
-      }
-      return true;
-    };
-    std::vector<char> concat_ok(n, 0);
-    for (int c = 0; c < n; ++c) {
-      if (g.ops[c].kind != HIOS_OP_CONCAT || c == g.sink_op || !all_relu_first(c, -1)) continue;
-      bool ok = true;
-      for (int e : g.ops[c].in_edges) {
-        const int p = g.edges[e].src;
-        if (!can_relu(p) || !all_relu_first(p, c)) ok = false;
-        for (int e2 : g.ops[p].out_edges)  // a producer of two concats: keep it simple
-          if (g.edges[e2].dst != c && g.ops[g.edges[e2].dst].kind == HIOS_OP_CONCAT) ok = false;
-      }
-      concat_ok[c] = ok;
-    }
-    for (int c = 0; c < n; ++c)
-      if (concat_ok[c]) {
-        relu_out[c] = 1;
-        for (int e : g.ops[c].in_edges) relu_out[g.edges[e].src] = 1;
-      }
-    for (int u = 0; u < n; ++u)
-      if (!relu_out[u] && can_relu(u) && all_relu_first(u, -1)) relu_out[u] = 1;
   }
   // pre-ReLU convs: one ReLU'd copy of the input per (producer, GPU) when the
   // producer runs on that GPU (made right after it), else a per-consumer scratch
@@ -1009,7 +1008,9 @@ static void build_op(Executor& ex, int v) {
         if (!ex.inplace[e]) {
           View iv = view_of(u, l);
           CopyArgs<T> c{(const T*)iv.p, iv.ldc, o.H * o.W, xu.C, (T*)(out.p + (size_t)c_off * ex.esz), out.ldc};
-          fns.push_back([c](cudaStream_t st) { launch_copy<T>(c, st); });
+          // a ReLU'd concat (relu_out) whose input keeps its raw output: ReLU'd slice copy
+          if (ex.relu_out[v] && !ex.relu_out[u]) fns.push_back([c](cudaStream_t st) { launch_relu_copy<T>(c, st); });
+          else fns.push_back([c](cudaStream_t st) { launch_copy<T>(c, st); });
           ++nk;
         }
         c_off += xu.C;

@@ -122,6 +122,7 @@ struct Executor {
   // all do), so the op stores its output already ReLU'd and the consumers
   // read it without a ReLU'd copy (ReLU(bf16(y)) = bf16(ReLU(y)): exact)
   std::vector<char> relu_out;
+  std::vector<char> relu_copy_in;  // per edge: the ReLU'd concat copies this raw input's slice
   std::vector<OpExec> ox;
   std::vector<std::vector<int>> flag_index;  // [op][lgpu] flag slot on that lgpu (-1 none)
   int n_streams = 1;
