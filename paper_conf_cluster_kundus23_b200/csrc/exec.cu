@@ -382,6 +382,30 @@ static void upload_weights_T(Executor& ex, int v) {
         x.shift.push_back((float*)upload(L, o.shift));
         break;
       }
+      if (!small_c_conv(o) && o.kh * o.kw > 1 && !o.weight.empty()) {
+        // single non-zero tap: keep only that tap (x.tap_r / tap_s)
+        int nz = 0, r0 = -1, s0 = -1;
+        for (int r = 0; r < o.kh && nz < 2; ++r)
+          for (int s2 = 0; s2 < o.kw && nz < 2; ++s2) {
+            bool any = false;
+            for (int k = 0; k < o.out_c && !any; ++k)
+              for (int c = 0; c < o.in_c; ++c)
+                if (o.weight[(((size_t)k * o.in_c + c) * o.kh + r) * o.kw + s2] != 0.f) { any = true; break; }
+            if (any) { ++nz; r0 = r; s0 = s2; }
+          }
+        if (nz == 1) {
+          std::vector<float> w1((size_t)o.out_c * o.in_c);
+          for (int k = 0; k < o.out_c; ++k)
+            for (int c = 0; c < o.in_c; ++c)
+              w1[(size_t)k * o.in_c + c] = o.weight[(((size_t)k * o.in_c + c) * o.kh + r0) * o.kw + s0];
+          x.w = upload(L, conv_layout<T>(w1.data(), o.out_c, o.in_c, 1, 1, Cp, tc ? o.scale.data() : nullptr));
+          x.tap_r = r0;
+          x.tap_s = s0;
+          x.scale.push_back((float*)upload(L, o.scale));
+          x.shift.push_back((float*)upload(L, o.shift));
+          break;
+        }
+      }
       x.w = upload(L, conv_layout<T>(o.weight.data(), o.out_c, o.in_c, o.kh, o.kw, Cp, tc ? o.scale.data() : nullptr));
       if (small_c_conv(o)) x.w_small = (float*)upload(L, conv_layout<float>(o.weight.data(), o.out_c, o.in_c, o.kh, o.kw, o.in_c));
       x.scale.push_back((float*)upload(L, o.scale));
@@ -924,8 +948,13 @@ static void build_op(Executor& ex, int v) {
         g_tc_out = &x.tc;
         g_tc_smem = &x.tc_smem;
       }
-      fns.push_back(conv_closure<T>(ex, cin, xi.H, xi.W, xi.C, x.w, x.scale[0], x.shift[0], o.out_c, o.kh,
-                                    o.kw, o.sh, o.sw, o.ph, o.pw, o.dh, o.dw, o.H, o.W, relu_v, out, out2, nk));
+      if (x.tap_r >= 0)  // single-tap conv: 1x1 on the tap-shifted input (same P x Q outputs)
+        fns.push_back(conv_closure<T>(ex, cin, xi.H, xi.W, xi.C, x.w, x.scale[0], x.shift[0], o.out_c, 1, 1, o.sh,
+                                      o.sw, o.ph - x.tap_r * o.dh, o.pw - x.tap_s * o.dw, 1, 1, o.H, o.W, relu_v, out,
+                                      out2, nk));
+      else
+        fns.push_back(conv_closure<T>(ex, cin, xi.H, xi.W, xi.C, x.w, x.scale[0], x.shift[0], o.out_c, o.kh,
+                                      o.kw, o.sh, o.sw, o.ph, o.pw, o.dh, o.dw, o.H, o.W, relu_v, out, out2, nk));
       g_tc_out = nullptr;
       g_tc_smem = nullptr;
       break;

@@ -51,6 +51,11 @@ struct OpExec {
   int relu_ldc = 0;
   int dw_ldc = 0, mid_ldc = 0;
   // stride-2 small-C stem (bf16): space-to-depth copy of the input (arena offset)
+  // a conv whose weights are zero at every tap but (tap_r, tap_s) (NASNet's
+  // factorized-reduction path 2: a shifted, strided 1x1 conv written as a
+  // 3x3 conv): x.w holds that tap only and the conv runs as 1x1 on the input
+  // shifted by the tap (padding ph - tap_r * dh, pw - tap_s * dw)
+  int tap_r = -1, tap_s = -1;
   int64_t s2dbuf = -1;
   int s2d_ldc = 0;
   // s2d stem with its S' taps packed into one 64-element K row (overlapping
