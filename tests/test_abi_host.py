@@ -196,6 +196,39 @@ def test_missing_costs_is_state_error():
     assert e.value.code == 8
 
 
+def test_executor_queries_and_stage_modes_host_rules():
+    """Host-side rules of the executor queries (no GPU): the stage mode
+    accepts STREAMS / GROUPED / DATAFLOW / AUTO and rejects others
+    (HIOS_E_INVALID); the mode used, the conv tile plan and the hoisted-ReLU
+    flag exist only after a run (HIOS_E_STATE); bad op ids are HIOS_E_INVALID."""
+    g = graphs.tiny(8, 8, 8)
+    G = hios.hios_graph_create(g.ops, g.edges, g.in_c, g.in_h, g.in_w, "bf16", gen.make_weights(g))
+    for op in g.ops:
+        hios.hios_set_op_cost(G, op.id, 1000)
+    for e in range(g.n_edges):
+        hios.hios_set_edge_cost(G, e, 100)
+    hios.hios_set_group_model(G, 7, 10)
+    for mode in ("streams", "grouped", "dataflow", "auto"):
+        S = hios.hios_schedule_lp(G, 1, 2)
+        hios.hios_schedule_stage_mode(S, mode)
+    S = hios.hios_schedule_lp(G, 1, 2)
+    with pytest.raises(hios.HiosError) as e:
+        hios.hios_schedule_stage_mode(S, 7)
+    assert e.value.code == 1
+    with pytest.raises(hios.HiosError) as e:
+        hios.hios_schedule_stage_mode_used(S)
+    assert e.value.code == 8
+    with pytest.raises(hios.HiosError) as e:
+        hios.hios_op_plan(S, 1)
+    assert e.value.code == 8
+    with pytest.raises(hios.HiosError) as e:
+        hios.hios_op_output_relu(S, 1)
+    assert e.value.code == 8
+    with pytest.raises(hios.HiosError) as e:
+        hios.hios_op_output_relu(S, g.n_ops)
+    assert e.value.code == 1
+
+
 def test_import_rejects_infeasible():
     n, t, E = 4, [5, 5, 5, 5], [(0, 2, 0), (3, 1, 0)]
     G, N, t_all, E_all = _cost_graph(n, t, E)
